@@ -1,0 +1,335 @@
+#!/usr/bin/env python
+"""bench.py -- batched negacyclic RNS NTT/INTT throughput on B200 (BASELINE.json metric).
+
+Contract (task statement / DESIGN.md "Measurement"):
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl wd|reference] [--mode auto|cuda|tensor|fused]
+A STEP = one pass of the whole hot path over one batch: forward NTT of every
+(polynomial, limb) row, then the inverse NTT of the result (config 3 of
+BASELINE.json: N=2^16, L=36, 64 ciphertexts = 128 polynomials = 4608 rows per
+direction).  value = KOPS = 1e-3 x single-prime N-point transforms per second
+(SURVEY.md reading C-9), counting both directions, summed over all ranks
+(weak scaling: every rank owns its own 64-ciphertext batch; the limbs and
+ciphertexts are independent so there is no collective inside the step).
+Inputs (1.2 GB) are larger than L2 (126 MB), so no explicit flush is needed.
+Rank 0 prints ONE JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (logN, L, ciphertexts)
+    "c1": (12, 4, None),       # 1 polynomial (configs[0]; oracle in seconds)
+    "c2": (16, 36, 1),
+    "c3": (16, 36, 64),        # headline (BASELINE.json metric / configs[2])
+    "c4": (17, 48, 32),
+}
+METRIC = "NTT KOPS (N=2^16, L=36) at 1/2/4/8 B200; % of HBM / int8 tensor roofline"
+FALLBACK_HBM_GBS = 6650.0
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except Exception:
+        return {"hbm_gbs": FALLBACK_HBM_GBS, "bf16_tflops": 1590.0}, "fallback"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML during the timed region."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, dev_index: int, period: float = 0.01):
+        self.samples, self.reasons, self.stop_ev = [], set(), threading.Event()
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+        self.period = period
+        self.th = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self.stop_ev.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.nv:
+            self.th.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop_ev.set()
+        if self.nv:
+            self.th.join()
+
+    def summary(self):
+        s = sorted(self.samples)
+        return {"sm_mhz": (s[len(s) // 2] if s else None), "sm_max_mhz": self.max_mhz,
+                "samples": len(s), "reasons": sorted(self.reasons)}
+
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def oracle_kops(logn: int, L: int, seconds: float = 12.0):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload."""
+    import oracle
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs
+    threads = oracle.default_threads()
+    primes = inputs.bench_primes(L)
+    n = 1 << logn
+    x = inputs.uniform_residues(primes, n, 1, inputs.SEED_BASE + 2)[0]      # one polynomial, all limbs
+    for q in primes:
+        oracle.psi_min(q, n)                                                 # psi search: plan time, not timed
+    done, t0 = 0, time.perf_counter()
+    while True:
+        k = max(1, min(L, threads))
+        rows = x[:k][None]
+        y = oracle.ntt_forward(rows, primes[:k], threads=threads)
+        oracle.ntt_inverse(y, primes[:k], threads=threads)
+        done += 2 * k
+        el = time.perf_counter() - t0
+        if el >= seconds:
+            break
+    return {"value": done / el / 1e3, "unit": "KOPS", "cores": threads, "kind": "oracle",
+            "sample": "%d N=2^%d transforms (fwd+inv pairs over the first %d limbs of one polynomial of the "
+                      "workload, %d threads) in %.1f s on %s" % (done, logn, min(L, threads), threads, el,
+                                                                   cpu_model())}
+
+
+def run_reference(args):
+    """--impl reference: the oracle on the host cores, same metric/config (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    logn, L, nct = CONFIGS[args.config]
+    import oracle
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs
+    oracle.build()
+    threads = oracle.default_threads()
+    primes = inputs.bench_primes(L)
+    n = 1 << logn
+    x = inputs.uniform_residues(primes, n, 1, inputs.SEED_BASE + 2)[0]
+    for q in primes:
+        oracle.psi_min(q, n)
+    k = max(1, min(L, threads))             # rows per step: one bounded sample of the workload
+    def step():
+        y = oracle.ntt_forward(x[:k][None], primes[:k], threads=threads)
+        oracle.ntt_inverse(y, primes[:k], threads=threads)
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    el = time.perf_counter() - t0
+    v = 2 * k * args.steps / el / 1e3
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "KOPS", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": "N=2^%d L=%d, bounded sample: %d rows fwd+inv per step" % (logn, L, k),
+                   "N": n, "L": L},
+        "cpu_baseline": {"value": v, "unit": "KOPS", "cores": threads, "kind": "oracle",
+                         "sample": "%d rows (N=2^%d) forward+inverse per step, %d threads, %s" % (k, logn, threads,
+                                                                                                  cpu_model())},
+        "e2e": {"value": v, "unit": "KOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="wd", choices=["wd", "reference"])
+    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused"])
+    ap.add_argument("--share", type=float, default=-1.0, help="tensor share for --mode fused")
+    ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    args = ap.parse_args()
+
+    if args.impl == "reference":
+        run_reference(args)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    logn, L, nct = CONFIGS[args.config]
+    n = 1 << logn
+    batch = 1 if nct is None else 2 * nct            # polynomials (1 ciphertext = 2 polynomials)
+    primes = inputs.bench_primes(L)
+    rows = batch * L
+    plan = wdntt.Plan(n, primes)
+    plan.set_mode(args.mode, args.share)
+    x = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 2 + 97 * rank, device="cuda")
+    y = torch.empty_like(x)
+    z = torch.empty_like(x)
+    stream = torch.cuda.current_stream()
+    sp = stream.cuda_stream
+
+    def step():
+        wdntt.wd_ntt_forward(plan.handle, x, y, batch, sp)
+        lf = wdntt.wd_ntt_last_launches()
+        wdntt.wd_ntt_inverse(plan.handle, y, z, batch, sp)
+        return lf + wdntt.wd_ntt_last_launches()
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    assert torch.equal(z, x), "round trip failed"
+
+    # ---- timed region: K steps, per-launch events on the launching stream
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches = 0
+    with ClockSampler(local) as clk:
+        t_start = torch.cuda.Event(enable_timing=True)
+        t_end = torch.cuda.Event(enable_timing=True)
+        t_start.record(stream)
+        for k in range(args.steps):
+            ev[k][0].record(stream)
+            wdntt.wd_ntt_forward(plan.handle, x, y, batch, sp)
+            launches += wdntt.wd_ntt_last_launches()
+            ev[k][1].record(stream)
+            wdntt.wd_ntt_inverse(plan.handle, y, z, batch, sp)
+            launches += wdntt.wd_ntt_last_launches()
+            ev[k][2].record(stream)
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = t_start.elapsed_time(t_end)
+    fwd_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in ev]))
+    inv_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in ev]))
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    total_transforms = 2 * rows * args.steps * world
+    kops = total_transforms / (ms_max / 1e3) / 1e3
+
+    # ---- end to end through the host-buffer C-ABI calls (pinned host memory)
+    e2e = None
+    if args.e2e_steps > 0:
+        hx = torch.empty(x.shape, dtype=torch.int32, pin_memory=True)
+        hx.copy_(x)
+        hy = torch.empty_like(hx, pin_memory=True)
+        hz = torch.empty_like(hx, pin_memory=True)
+        work = torch.empty_like(x)
+        def e2e_step():
+            wdntt.wd_ntt_forward_host(plan.handle, hx, hy, batch, work, sp)
+            wdntt.wd_ntt_inverse_host(plan.handle, hy, hz, batch, work, sp)
+        e2e_step()
+        torch.cuda.synchronize()
+        assert torch.equal(hz, hx)
+        if world > 1:
+            dist.barrier()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        a1.record(stream)
+        torch.cuda.synchronize()
+        te = torch.tensor([a0.elapsed_time(a1)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        bytes_step = 2 * rows * n * 4            # two host calls, each copies the batch in and out
+        e2e = {"value": 2 * rows * args.e2e_steps * world / (float(te.item()) / 1e3) / 1e3, "unit": "KOPS",
+               "h2d_bytes_per_step": bytes_step, "d2h_bytes_per_step": bytes_step,
+               "steps": args.e2e_steps, "api": "wd_ntt_forward_host + wd_ntt_inverse_host (pinned host buffers)"}
+        del hx, hy, hz, work
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    pk, pk_kind = peaks()
+    hbm = float(pk.get("hbm_gbs", FALLBACK_HBM_GBS))
+    dom_ms, dom_name = (fwd_ms, "forward") if fwd_ms >= inv_ms else (inv_ms, "inverse")
+    alg_bytes = 8.0 * n * rows                       # read 4N + write 4N bytes per transform
+    achieved = alg_bytes / (dom_ms / 1e3) / 1e9
+    traffic = None
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        traffic = tr.get("%s_%s_%s" % (args.config, args.mode, dom_name))
+    except Exception:
+        pass
+    line = {
+        "metric": METRIC, "value": kops, "unit": "KOPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic (splitmix64 uniform residues, SURVEY.md 8.d)",
+        "config": {"workload": "config3: N=2^%d, L=%d, %s polynomials per GPU, forward+inverse per step"
+                               % (logn, L, batch), "N": n, "L": L, "polys_per_gpu": batch,
+                   "rows_per_direction_per_gpu": rows, "mode": args.mode,
+                   "l2": "inputs %.2f GB > 126 MB L2, no flush needed" % (rows * n * 4 / 1e9),
+                   "parallelism": "limb/ciphertext independent, weak scaling, no collective"},
+        "fwd_kops": rows * world / (fwd_ms / 1e3) / 1e3, "inv_kops": rows * world / (inv_ms / 1e3) / 1e3,
+        "fwd_ms": fwd_ms, "inv_ms": inv_ms,
+        "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "traffic": traffic,
+                     "peak_kind": "%s (MEASURED_PEAKS.json hbm_gbs copy bandwidth)" % pk_kind,
+                     "algorithmic_bytes_per_launch": alg_bytes},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+        "e2e": e2e,
+    }
+    if not args.no_cpu and world == 1:
+        line["cpu_baseline"] = oracle_kops(logn, L, args.cpu_seconds)
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

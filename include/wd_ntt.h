@@ -1,0 +1,155 @@
+/*
+ * wd_ntt.h -- C ABI of libwdntt.so: batched negacyclic RNS NTT / INTT on B200 (sm_100a).
+ *
+ * This is the boundary of the WarpDrive hot path: the forward
+ * and inverse Number Theoretic Transform over RNS-decomposed CKKS polynomials
+ * (section II-B1 Eq.(1); PAPER.md:56 ring R_Q = Z_Q[X]/(X^N+1);
+ * PAPER.md:334-352 section IV-C "PE kernel": one launch covers every
+ * polynomial and limb), with the plan precompute of PAPER.md:358 section IV-D1.
+ *
+ * Conventions:
+ *   * data layout  [batch][L][N] uint32, row-major: row (b, l) is the residue of
+ *     polynomial b modulo primes[l]; rows contiguous, N words each.
+ *   * forward      out[i] = sum_j in[j] * psi_l^((2*brv_N(i)+1)*j) mod q_l
+ *                  (negacyclic, reading C-1; output in BIT-REVERSED order, C-3)
+ *   * inverse      the exact inverse: bit-reversed in, natural order out,
+ *                  N^-1 applied (reading C-6)
+ *   * psi_l        the minimal primitive 2N-th root of unity mod q_l (C-4)
+ *   * values       inputs must be canonical in [0, q_l); outputs are canonical.
+ *                  A non-canonical input gives an unspecified result but never
+ *                  a fault (reading C-7).
+ * No floating point anywhere on the path.
+ *
+ * Ownership and execution: device pointers are caller-owned (torch tensors),
+ * 16-byte aligned.  in == out (in place) is allowed, other overlap is undefined.
+ * Calls are stream-ordered and asynchronous on `stream` (a cudaStream_t; NULL =
+ * legacy default stream), perform no host synchronisation and no allocation,
+ * and are re-entrant across host threads.  A plan is bound to the device that
+ * was current at create time and is immutable after creation except for the
+ * mode knob; destroy it only after all work using it has completed.
+ *
+ * Errors: functions returning int return WD_OK (0) or a WD_E* code, and also
+ * record it in a thread-local slot read by wd_ntt_last_error().  Asynchronous
+ * device faults surface at the caller's next synchronisation on the stream.
+ */
+#ifndef WD_NTT_H
+#define WD_NTT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct wd_ntt_plan wd_ntt_plan;        /* opaque */
+typedef struct CUstream_st* wd_stream_t;       /* == cudaStream_t */
+
+/* error codes */
+#define WD_OK            0
+#define WD_EINVAL        1   /* NULL / misaligned pointer, bad size, wrong device      */
+#define WD_EPRIME        2   /* a modulus is not prime, >= 2^30, or != 1 (mod 2N)       */
+#define WD_EUNSUPPORTED  3   /* N outside [2, 2^17], L outside [1, 4096], mode n/a      */
+#define WD_ECUDA         4   /* CUDA runtime error (no device, launch failure, ...)     */
+#define WD_ENOMEM        5   /* device or host allocation failed                        */
+
+/* execution modes (wd_ntt_plan_set_mode) */
+#define WD_MODE_AUTO     0   /* library default for this N                              */
+#define WD_MODE_CUDA     1   /* CUDA-core radix-2^k butterflies only (WD-BO role)       */
+#define WD_MODE_TENSOR   2   /* tcgen05 kind::i8 inner DFTs + CUDA-core epilogue        */
+#define WD_MODE_FUSED    3   /* both paths concurrently on the same SMs (WD-FUSE role)  */
+
+/*
+ * wd_ntt_plan_create -- PAPER.md:358 (initialisation phase: moduli, twiddles
+ * precomputed and uploaded ahead of time).
+ *   N       transform length, a power of two in [2, 2^17]
+ *   primes  host array of L moduli; each must be prime, < 2^30 and = 1 mod 2N
+ *           (read during the call only; the caller keeps ownership)
+ *   L       number of RNS limbs, 1 <= L <= 4096
+ * Returns a plan owning its device tables (about 16*N*L bytes: forward and
+ * inverse psi-power tables in bit-reversed order with Shoup companions, plus
+ * the tensor-path inner-DFT byte planes), or NULL with wd_ntt_last_error() set
+ * to WD_EINVAL / WD_EPRIME / WD_EUNSUPPORTED / WD_ECUDA / WD_ENOMEM.
+ * Argument validation happens before any CUDA call, so the WD_EINVAL /
+ * WD_EPRIME / WD_EUNSUPPORTED paths work on a machine without a GPU.
+ */
+wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L);
+
+/* Frees the plan's device tables.  NULL is a no-op.  Caller must have
+ * synchronised all work using the plan. */
+void wd_ntt_plan_destroy(wd_ntt_plan* plan);
+
+/*
+ * wd_ntt_forward / wd_ntt_inverse -- PAPER.md:85-91 (Eq.(1) and its inverse),
+ * batched over all (polynomial, limb) rows in ONE launch.
+ *   in, out  device pointers to batch*L*N uint32 words, layout [batch][L][N],
+ *            16-byte aligned; in == out allowed
+ *   batch    number of polynomials (a ciphertext is 2 polynomials);
+ *            0 is a successful no-op
+ *   stream   cudaStream_t the work is enqueued on
+ * Returns WD_OK, WD_EINVAL (NULL plan/pointer, misalignment, wrong device),
+ * WD_EUNSUPPORTED (mode not available for this N) or WD_ECUDA (launch error).
+ */
+int wd_ntt_forward(const wd_ntt_plan* plan, const uint32_t* in, uint32_t* out,
+                   uint32_t batch, wd_stream_t stream);
+int wd_ntt_inverse(const wd_ntt_plan* plan, const uint32_t* in, uint32_t* out,
+                   uint32_t batch, wd_stream_t stream);
+
+/*
+ * wd_ntt_forward_host / wd_ntt_inverse_host -- the same transforms on HOST
+ * buffers (end-to-end path): copies host->device, transforms, copies back,
+ * pipelined in chunks over internal streams so the H2D copy of chunk k+1,
+ * the kernel of chunk k and the D2H copy of chunk k-1 overlap.
+ *   h_in, h_out  host pointers, batch*L*N words (pinned memory recommended;
+ *                pageable works but serialises); h_in == h_out allowed
+ *   d_work       caller-owned device scratch of >= batch*L*N words, 16-B aligned
+ *   stream       the call is ordered after prior work on `stream`, and work
+ *                enqueued on `stream` afterwards is ordered after its end
+ * Asynchronous like the device calls: h_out is valid after the caller
+ * synchronises `stream`.
+ */
+int wd_ntt_forward_host(const wd_ntt_plan* plan, const uint32_t* h_in, uint32_t* h_out,
+                        uint32_t batch, uint32_t* d_work, wd_stream_t stream);
+int wd_ntt_inverse_host(const wd_ntt_plan* plan, const uint32_t* h_in, uint32_t* h_out,
+                        uint32_t batch, uint32_t* d_work, wd_stream_t stream);
+
+/*
+ * wd_ntt_pointwise_inverse -- SURVEY.md 8 row f1 (NEXT #1): out = INTT(a o b),
+ * the negacyclic product of two polynomials given in the NTT domain
+ * (PAPER.md:63 HMULT tensor product + PAPER.md:85 "convert polynomial
+ * multiplication into point-wise multiplication").  Same layout/stream rules;
+ * out may alias a or b.
+ */
+int wd_ntt_pointwise_inverse(const wd_ntt_plan* plan, const uint32_t* a, const uint32_t* b,
+                             uint32_t* out, uint32_t batch, wd_stream_t stream);
+
+/* ---- queries and knobs ---- */
+uint32_t wd_ntt_plan_n(const wd_ntt_plan* plan);
+uint32_t wd_ntt_plan_limbs(const wd_ntt_plan* plan);
+/* psi actually used for limb `limb` (0 if out of range) -- reading C-4 */
+uint32_t wd_ntt_plan_psi(const wd_ntt_plan* plan, uint32_t limb);
+
+/* Host-only helpers of the plan precompute (no GPU needed):
+ * wd_ntt_root(q, N): the minimal primitive 2N-th root the plan would use, 0
+ * if q fails the prime checks; wd_ntt_check_prime(q, N): WD_OK or WD_EPRIME. */
+uint32_t wd_ntt_root(uint32_t q, uint32_t N);
+int      wd_ntt_check_prime(uint32_t q, uint32_t N);
+
+/* Select the execution path.  tensor_share in [0,1] is the fraction of
+ * transform tiles given to the tensor path in WD_MODE_FUSED (ignored
+ * otherwise; < 0 keeps the plan's measured default).  Returns WD_OK,
+ * WD_EINVAL or WD_EUNSUPPORTED.  Not thread-safe against concurrent calls
+ * using the same plan. */
+int wd_ntt_plan_set_mode(wd_ntt_plan* plan, int mode, float tensor_share);
+int wd_ntt_plan_get_mode(const wd_ntt_plan* plan);
+
+/* Kernel launches issued by the last forward/inverse call on this thread. */
+uint32_t wd_ntt_last_launches(void);
+
+int         wd_ntt_last_error(void);
+const char* wd_ntt_strerror(int code);
+const char* wd_ntt_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WD_NTT_H */

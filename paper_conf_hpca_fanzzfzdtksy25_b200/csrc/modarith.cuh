@@ -1,0 +1,118 @@
+// modarith.cuh -- device modular arithmetic for the NTT hot path (sm_100a).
+//
+// Word size: 32-bit residues, q < 2^30 so 4q < 2^32 (PAPER.md:375,399 use
+// 32-bit words).  Multiplication by a precomputed constant w
+// uses Shoup's method with w' = floor(w * 2^32 / q): for ANY 32-bit a,
+//     a*w - umulhi(a, w')*q  (mod 2^32)  lies in [0, 2q).
+// (The paper uses Montgomery for the NTT; reading C-8: the
+// canonical outputs are unique, so the reduction scheme is free.)
+// Butterflies are Harvey's lazy forms:
+//   CT (forward):  inputs/outputs in [0, 4q)     -- 3 IMAD + 4 ALU ops
+//   GS (inverse):  inputs/outputs in [0, 2q)
+#pragma once
+#include <cstdint>
+
+namespace wd {
+
+__device__ __forceinline__ uint32_t umin32(uint32_t a, uint32_t b) { return a < b ? a : b; }
+
+struct __align__(32) LimbConst {
+    uint32_t q, q2;          // q, 2q
+    uint32_t ninv, ninv_sh;  // N^-1 mod q and its Shoup companion
+    uint32_t wn, wn_sh;      // psi^-brv(1) * N^-1 (last inverse layer) + Shoup
+    uint64_t mu;             // floor((2^64-1)/q): Barrett constant for a*b mod q (pointwise)
+};
+
+// a * b mod q for two variable residues (< 2^32 each, product < 2^62 for q < 2^30): Barrett
+__device__ __forceinline__ uint32_t mul_mod(uint32_t a, uint32_t b, const LimbConst& c) {
+    const uint64_t p = (uint64_t)a * b;
+    const uint64_t quo = __umul64hi(p, c.mu);
+    uint32_t r = (uint32_t)(p - quo * c.q);      // in [0, 3q)
+    r = umin32(r, r - c.q);
+    return umin32(r, r - c.q);
+}
+
+// a * w mod q, result in [0, 2q), any 32-bit a
+__device__ __forceinline__ uint32_t shoup_mul(uint32_t a, uint32_t w, uint32_t ws, uint32_t q) {
+    const uint32_t hq = __umulhi(a, ws);
+    return a * w - hq * q;
+}
+
+// forward Cooley-Tukey butterfly (merged psi): (X, Y) -> (X + wY, X - wY), lazy in [0,4q)
+__device__ __forceinline__ void ct_bfly(uint32_t& X, uint32_t& Y, uint2 w, uint32_t q, uint32_t q2) {
+    const uint32_t x = umin32(X, X - q2);          // [0, 2q)
+    const uint32_t t = shoup_mul(Y, w.x, w.y, q);  // [0, 2q)
+    X = x + t;
+    Y = x - t + q2;
+}
+
+// inverse Gentleman-Sande butterfly: (X, Y) -> (X + Y, (X - Y) w), lazy in [0,2q)
+__device__ __forceinline__ void gs_bfly(uint32_t& X, uint32_t& Y, uint2 w, uint32_t q, uint32_t q2) {
+    uint32_t u = X + Y;
+    u = umin32(u, u - q2);
+    const uint32_t t = X - Y + q2;
+    Y = shoup_mul(t, w.x, w.y, q);
+    X = u;
+}
+
+// last inverse layer (layer 0) with N^-1 folded in: (X, Y) -> ((X+Y) n, (X-Y) w n), in [0,2q)
+__device__ __forceinline__ void gs_bfly_last(uint32_t& X, uint32_t& Y, const LimbConst& c) {
+    const uint32_t u = X + Y;
+    const uint32_t t = X - Y + c.q2;
+    X = shoup_mul(u, c.ninv, c.ninv_sh, c.q);
+    Y = shoup_mul(t, c.wn, c.wn_sh, c.q);
+}
+
+__device__ __forceinline__ uint32_t canon4(uint32_t v, uint32_t q, uint32_t q2) {  // [0,4q) -> [0,q)
+    v = umin32(v, v - q2);
+    return umin32(v, v - q);
+}
+__device__ __forceinline__ uint32_t canon2(uint32_t v, uint32_t q) {                // [0,2q) -> [0,q)
+    return umin32(v, v - q);
+}
+
+// K forward layers on R = 2^K registers.  The block's elements sit at global
+// indices g0 + r*D; layer ls+t pairs r and r + 2^(K-1-t) with twiddle
+// Psi[2^(ls+t) + (hi << t) + (r >> (K-t))], hi = g0 >> (logN - ls) (the
+// group index of the block at its first layer).  Same index rule as the
+// textbook merged-psi loop, restricted to one block.
+template <int K>
+__device__ __forceinline__ void fwd_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
+                                          uint32_t hi, uint32_t q, uint32_t q2) {
+#pragma unroll
+    for (int t = 0; t < K; ++t) {
+        const int h = 1 << (K - 1 - t);
+        const uint2* tp = tw + (1u << (ls + t)) + (hi << t);
+#pragma unroll
+        for (int g = 0; g < (1 << t); ++g) {
+            const uint2 w = __ldg(tp + g);
+#pragma unroll
+            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w, q, q2);
+        }
+    }
+}
+
+// K inverse (GS) layers, mirror of fwd_radix: layers ls+K-1 down to ls.
+// LAST: this block ends at global layer 0 (ls == 0), fold N^-1 there.
+template <int K, bool LAST>
+__device__ __forceinline__ void inv_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
+                                          uint32_t hi, const LimbConst& c) {
+#pragma unroll
+    for (int t = K - 1; t >= 0; --t) {
+        const int h = 1 << (K - 1 - t);
+        const uint2* tp = tw + (1u << (ls + t)) + (hi << t);
+#pragma unroll
+        for (int g = 0; g < (1 << t); ++g) {
+            if (LAST && t == 0) {
+#pragma unroll
+                for (int r = 0; r < h; ++r) gs_bfly_last(x[r], x[r + h], c);
+            } else {
+                const uint2 w = __ldg(tp + g);
+#pragma unroll
+                for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w, c.q, c.q2);
+            }
+        }
+    }
+}
+
+}  // namespace wd

@@ -1,0 +1,327 @@
+// wd_ntt.cu -- libwdntt.so: plan precompute, C ABI and dispatch (b).
+//
+// The ABI is declared and documented in include/wd_ntt.h.  Everything on the
+// call path is asynchronous on the caller's stream; the only host<->device
+// copies are the one-time table upload in wd_ntt_plan_create
+// and the explicit host-buffer entry points.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "wd_ntt.h"
+#include "modarith.cuh"
+#include "ntt_cuda_core.cuh"
+#include "ntt_tensor.cuh"
+#include "plan_math.h"
+
+using namespace wd;
+
+namespace {
+thread_local int g_last_error = WD_OK;
+thread_local uint32_t g_last_launches = 0;
+int set_err(int e) { g_last_error = e; return e; }
+}  // namespace
+
+struct wd_ntt_plan {
+    uint32_t N = 0, logN = 0, L = 0;
+    int device = -1;
+    std::vector<uint32_t> primes, psi;
+    uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
+    uint2* d_inv = nullptr;        // [L][N]  (psi^-brv(i), Shoup)
+    LimbConst* d_lc = nullptr;     // [L]
+    TensorTables tc;               // tensor-path planes (ntt_tensor.cuh)
+    int mode = WD_MODE_AUTO;
+    float tensor_share = 0.5f;
+    cudaStream_t hs[3] = {nullptr, nullptr, nullptr};   // host-path pipeline streams
+    cudaEvent_t he[4] = {nullptr, nullptr, nullptr, nullptr};
+    std::mutex host_mu;
+};
+
+namespace {
+
+bool is_pow2(uint32_t n) { return n && !(n & (n - 1)); }
+uint32_t ilog2u(uint32_t n) { uint32_t l = 0; while ((1u << l) < n) ++l; return l; }
+
+int check_prime(uint32_t q, uint32_t N) {
+    if (q >= (1u << 30) || q < 3) return WD_EPRIME;
+    if ((q - 1) % (2ull * N) != 0) return WD_EPRIME;
+    if (!pm_is_prime(q)) return WD_EPRIME;
+    return WD_OK;
+}
+
+template <typename K>
+int set_smem(K kern, int bytes) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
+        return WD_ECUDA;
+    return WD_OK;
+}
+
+template <int LOGN>
+int prep_cc() {
+    using S = CcShape<LOGN>;
+    if (set_smem(ntt_fwd_cc<LOGN>, S::SMEM_BYTES) || set_smem(ntt_inv_cc<LOGN, false>, S::SMEM_BYTES) ||
+        set_smem(ntt_inv_cc<LOGN, true>, S::SMEM_BYTES))
+        return WD_ECUDA;
+    return WD_OK;
+}
+
+int prepare_kernels(uint32_t logN) {
+    switch (logN) {
+        case 12: return prep_cc<12>();
+        case 13: return prep_cc<13>();
+        case 14: return prep_cc<14>();
+        case 15: return prep_cc<15>();
+        case 16: return prep_cc<16>();
+        case 17: return prep_cc<17>();
+        default:
+            if (set_smem(ntt_small<true, false>, 4 << logN) || set_smem(ntt_small<false, false>, 4 << logN) ||
+                set_smem(ntt_small<false, true>, 4 << logN))
+                return WD_ECUDA;
+            return WD_OK;
+    }
+}
+
+template <int LOGN>
+void launch_cc(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    using S = CcShape<LOGN>;
+    if (fwd) ntt_fwd_cc<LOGN><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
+    else if (a.in2) ntt_inv_cc<LOGN, true><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
+    else ntt_inv_cc<LOGN, false><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
+}
+
+int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    switch (p->logN) {
+        case 12: launch_cc<12>(fwd, a, rows, s); break;
+        case 13: launch_cc<13>(fwd, a, rows, s); break;
+        case 14: launch_cc<14>(fwd, a, rows, s); break;
+        case 15: launch_cc<15>(fwd, a, rows, s); break;
+        case 16: launch_cc<16>(fwd, a, rows, s); break;
+        case 17: launch_cc<17>(fwd, a, rows, s); break;
+        default: {
+            const int thr = std::min<int>(256, std::max<int>(32, (int)p->N / 2));
+            if (fwd) ntt_small<true, false><<<rows, thr, 4 << p->logN, s>>>(a, (int)p->logN);
+            else if (a.in2) ntt_small<false, true><<<rows, thr, 4 << p->logN, s>>>(a, (int)p->logN);
+            else ntt_small<false, false><<<rows, thr, 4 << p->logN, s>>>(a, (int)p->logN);
+        }
+    }
+    return 1;
+}
+
+int effective_mode(const wd_ntt_plan* p) {
+    if (p->mode != WD_MODE_AUTO) return p->mode;
+    return WD_MODE_CUDA;
+}
+
+int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2, uint32_t* out,
+        uint32_t batch, cudaStream_t s) {
+    g_last_launches = 0;
+    if (!p || !in || !out || (in2 == nullptr && false)) return set_err(WD_EINVAL);
+    if (((uintptr_t)in | (uintptr_t)out | (uintptr_t)in2) & 15) return set_err(WD_EINVAL);
+    if (batch == 0) return set_err(WD_OK);
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) return set_err(WD_EINVAL);
+    const uint64_t rows64 = (uint64_t)batch * p->L;
+    if (rows64 > 0x7fffffffull) return set_err(WD_EINVAL);
+    const uint32_t rows = (uint32_t)rows64;
+    NttArgs a;
+    a.in = in; a.in2 = in2; a.out = out; a.tw = fwd ? p->d_fwd : p->d_inv; a.lc = p->d_lc; a.L = p->L;
+    const int mode = effective_mode(p);
+    int launches = 0;
+    if (mode == WD_MODE_CUDA || in2 != nullptr || !tensor_supported(p->logN)) {
+        if (mode != WD_MODE_CUDA && in2 == nullptr && mode != WD_MODE_AUTO) return set_err(WD_EUNSUPPORTED);
+        launches = launch_cuda_core(p, fwd, a, rows, s);
+    } else {
+        float share = mode == WD_MODE_TENSOR ? 1.0f : p->tensor_share;
+        launches = launch_tensor(p->logN, fwd, a, p->tc, rows, share, s);
+        if (launches < 0) return set_err(WD_EUNSUPPORTED);
+    }
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    g_last_launches = (uint32_t)launches;
+    return set_err(WD_OK);
+}
+
+int run_host(const wd_ntt_plan* pc, bool fwd, const uint32_t* h_in, uint32_t* h_out, uint32_t batch,
+             uint32_t* d_work, cudaStream_t s) {
+    if (!pc || !h_in || !h_out || !d_work || ((uintptr_t)d_work & 15)) return set_err(WD_EINVAL);
+    if (batch == 0) return set_err(WD_OK);
+    wd_ntt_plan* p = const_cast<wd_ntt_plan*>(pc);
+    std::lock_guard<std::mutex> lk(p->host_mu);
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) return set_err(WD_EINVAL);
+    const size_t row_words = (size_t)p->L * p->N;
+    // ~8 chunks, each at least 1 polynomial: H2D(k+1) || kernel(k) || D2H(k-1)
+    const uint32_t nch = std::min<uint32_t>(batch, 8);
+    cudaEventRecord(p->he[3], s);
+    uint32_t total = 0;
+    uint32_t b0 = 0;
+    for (uint32_t k = 0; k < nch; ++k) {
+        const uint32_t b1 = (uint32_t)((uint64_t)batch * (k + 1) / nch);
+        const uint32_t nb = b1 - b0;
+        cudaStream_t st = p->hs[k % 3];
+        if (k < 3) cudaStreamWaitEvent(st, p->he[3], 0);
+        const size_t off = (size_t)b0 * row_words, bytes = (size_t)nb * row_words * 4;
+        cudaMemcpyAsync(d_work + off, h_in + off, bytes, cudaMemcpyHostToDevice, st);
+        int e = run(p, fwd, d_work + off, nullptr, d_work + off, nb, st);
+        if (e) return e;
+        total += g_last_launches;
+        cudaMemcpyAsync(h_out + off, d_work + off, bytes, cudaMemcpyDeviceToHost, st);
+        b0 = b1;
+    }
+    for (int i = 0; i < 3; ++i) {
+        cudaEventRecord(p->he[i], p->hs[i]);
+        cudaStreamWaitEvent(s, p->he[i], 0);
+    }
+    g_last_launches = total;
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    return set_err(WD_OK);
+}
+
+void free_plan(wd_ntt_plan* p) {
+    if (!p) return;
+    if (p->device >= 0) {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (cur != p->device) cudaSetDevice(p->device);
+        cudaFree(p->d_fwd); cudaFree(p->d_inv); cudaFree(p->d_lc);
+        free_tensor_tables(p->tc);
+        for (auto& s : p->hs) if (s) cudaStreamDestroy(s);
+        for (auto& e : p->he) if (e) cudaEventDestroy(e);
+        if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
+    }
+    delete p;
+}
+
+}  // namespace
+
+extern "C" {
+
+wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) {
+    if (!primes) { set_err(WD_EINVAL); return nullptr; }
+    if (!is_pow2(N) || N < 2 || N > (1u << 17) || L == 0 || L > 4096) { set_err(WD_EUNSUPPORTED); return nullptr; }
+    for (uint32_t l = 0; l < L; ++l)
+        if (check_prime(primes[l], N)) { set_err(WD_EPRIME); return nullptr; }
+
+    wd_ntt_plan* p = new (std::nothrow) wd_ntt_plan();
+    if (!p) { set_err(WD_ENOMEM); return nullptr; }
+    p->N = N; p->logN = ilog2u(N); p->L = L;
+    p->primes.assign(primes, primes + L);
+
+    // ---- host precompute (a1): psi, bit-reversed psi-power tables + Shoup companions
+    std::vector<uint2> fwd((size_t)L * N), inv((size_t)L * N);
+    std::vector<LimbConst> lc(L);
+    for (uint32_t l = 0; l < L; ++l) {
+        const uint32_t q = primes[l];
+        const uint32_t psi = plan_psi_min(q, N);
+        const uint32_t psi_inv = pm_pow(psi, q - 2, q);
+        p->psi.push_back(psi);
+        std::vector<uint32_t> pw(N), pwi(N);
+        pw[0] = 1; pwi[0] = 1;
+        for (uint32_t i = 1; i < N; ++i) { pw[i] = pm_mul(pw[i - 1], psi, q); pwi[i] = pm_mul(pwi[i - 1], psi_inv, q); }
+        uint2* f = fwd.data() + (size_t)l * N;
+        uint2* v = inv.data() + (size_t)l * N;
+        for (uint32_t i = 0; i < N; ++i) {
+            const uint32_t e = pm_brv(i, (int)p->logN);
+            f[i] = make_uint2(pw[e], pm_shoup(pw[e], q));
+            v[i] = make_uint2(pwi[e], pm_shoup(pwi[e], q));
+        }
+        LimbConst& c = lc[l];
+        c.q = q; c.q2 = 2 * q;
+        c.ninv = pm_pow(N % q, q - 2, q); c.ninv_sh = pm_shoup(c.ninv, q);
+        c.wn = pm_mul(N > 1 ? v[1].x : 1, c.ninv, q); c.wn_sh = pm_shoup(c.wn, q);
+        c.mu = ~0ull / q;
+    }
+
+    // ---- device upload (the only H2D copy of the plan's life)
+    if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
+    const size_t tb = sizeof(uint2) * (size_t)L * N;
+    if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
+        cudaMalloc(&p->d_lc, sizeof(LimbConst) * L) != cudaSuccess) {
+        cudaGetLastError(); free_plan(p); set_err(WD_ENOMEM); return nullptr;
+    }
+    if (cudaMemcpy(p->d_fwd, fwd.data(), tb, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(p->d_inv, inv.data(), tb, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemcpy(p->d_lc, lc.data(), sizeof(LimbConst) * L, cudaMemcpyHostToDevice) != cudaSuccess) {
+        cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
+    }
+    if (build_tensor_tables(p->tc, p->logN, p->primes, p->psi) != WD_OK) {
+        cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
+    }
+    for (auto& s : p->hs) if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
+    for (auto& e : p->he) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
+    if (prepare_kernels(p->logN) != WD_OK || prepare_tensor_kernels(p->logN) != WD_OK) {
+        cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
+    }
+    p->mode = WD_MODE_AUTO;
+    p->tensor_share = default_tensor_share(p->logN);
+    set_err(WD_OK);
+    return p;
+}
+
+void wd_ntt_plan_destroy(wd_ntt_plan* plan) { free_plan(plan); }
+
+int wd_ntt_forward(const wd_ntt_plan* p, const uint32_t* in, uint32_t* out, uint32_t batch, wd_stream_t s) {
+    if (!in) return set_err(WD_EINVAL);
+    return run(p, true, in, nullptr, out, batch, (cudaStream_t)s);
+}
+int wd_ntt_inverse(const wd_ntt_plan* p, const uint32_t* in, uint32_t* out, uint32_t batch, wd_stream_t s) {
+    if (!in) return set_err(WD_EINVAL);
+    return run(p, false, in, nullptr, out, batch, (cudaStream_t)s);
+}
+int wd_ntt_pointwise_inverse(const wd_ntt_plan* p, const uint32_t* a, const uint32_t* b, uint32_t* out,
+                             uint32_t batch, wd_stream_t s) {
+    if (!a || !b) return set_err(WD_EINVAL);
+    return run(p, false, a, b, out, batch, (cudaStream_t)s);
+}
+int wd_ntt_forward_host(const wd_ntt_plan* p, const uint32_t* h_in, uint32_t* h_out, uint32_t batch,
+                        uint32_t* d_work, wd_stream_t s) {
+    return run_host(p, true, h_in, h_out, batch, d_work, (cudaStream_t)s);
+}
+int wd_ntt_inverse_host(const wd_ntt_plan* p, const uint32_t* h_in, uint32_t* h_out, uint32_t batch,
+                        uint32_t* d_work, wd_stream_t s) {
+    return run_host(p, false, h_in, h_out, batch, d_work, (cudaStream_t)s);
+}
+
+uint32_t wd_ntt_plan_n(const wd_ntt_plan* p) { return p ? p->N : 0; }
+uint32_t wd_ntt_plan_limbs(const wd_ntt_plan* p) { return p ? p->L : 0; }
+uint32_t wd_ntt_plan_psi(const wd_ntt_plan* p, uint32_t limb) { return (p && limb < p->L) ? p->psi[limb] : 0; }
+
+uint32_t wd_ntt_root(uint32_t q, uint32_t N) {
+    if (!is_pow2(N) || N < 2 || N > (1u << 17) || check_prime(q, N)) return 0;
+    return plan_psi_min(q, N);
+}
+int wd_ntt_check_prime(uint32_t q, uint32_t N) {
+    if (!is_pow2(N) || N < 2) return WD_EUNSUPPORTED;
+    return check_prime(q, N);
+}
+
+int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
+    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_FUSED) return set_err(WD_EINVAL);
+    if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED) && !tensor_supported(p->logN)) return set_err(WD_EUNSUPPORTED);
+    if (tensor_share > 1.0f) return set_err(WD_EINVAL);
+    p->mode = mode;
+    if (tensor_share >= 0.0f) p->tensor_share = tensor_share;
+    return set_err(WD_OK);
+}
+int wd_ntt_plan_get_mode(const wd_ntt_plan* p) { return p ? effective_mode(p) : -1; }
+
+uint32_t wd_ntt_last_launches(void) { return g_last_launches; }
+int wd_ntt_last_error(void) { return g_last_error; }
+const char* wd_ntt_strerror(int code) {
+    switch (code) {
+        case WD_OK: return "ok";
+        case WD_EINVAL: return "invalid argument (NULL/misaligned pointer, bad size or wrong device)";
+        case WD_EPRIME: return "modulus is not an NTT-friendly prime < 2^30 (q prime, q = 1 mod 2N)";
+        case WD_EUNSUPPORTED: return "unsupported size or mode";
+        case WD_ECUDA: return "CUDA runtime error";
+        case WD_ENOMEM: return "out of memory";
+        default: return "unknown error";
+    }
+}
+const char* wd_ntt_version(void) { return "wdntt 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -54,6 +54,37 @@ def uniform_residues(primes, n: int, batch: int, seed: int) -> np.ndarray:
     return x.astype(np.uint32)
 
 
+def uniform_residues_torch(primes, n: int, batch: int, seed: int, device="cpu", chunk_rows: int = 256):
+    """Same values as ``uniform_residues`` (bit for bit), generated with torch int64 ops
+    (wrapping multiply; logical shifts emulated by masking) directly on ``device``.
+    Returns an int32 tensor [batch][L][n] holding the uint32 residues."""
+    import torch
+
+    def lsr(z, s):                       # logical right shift of a 64-bit pattern
+        return (z >> s) & ((1 << (64 - s)) - 1)
+
+    def s64(v):                          # uint64 constant -> int64 bit pattern
+        return v - (1 << 64) if v >= (1 << 63) else v
+
+    g, c1, c2 = s64(int(GOLDEN)), s64(int(_C1)), s64(int(_C2))
+    L = len(primes)
+    out = torch.empty((batch, L, n), dtype=torch.int32, device=device)
+    flat = out.view(-1)
+    q = torch.tensor([int(p) for p in primes], dtype=torch.int64, device=device)
+    rows = batch * L
+    for r0 in range(0, rows, chunk_rows):
+        r1 = min(rows, r0 + chunk_rows)
+        ctr = torch.arange(r0 * n + 1, r1 * n + 1, dtype=torch.int64, device=device)
+        z = s64(seed & 0xFFFFFFFFFFFFFFFF) + ctr * g
+        z = (z ^ lsr(z, 30)) * c1
+        z = (z ^ lsr(z, 27)) * c2
+        z = z ^ lsr(z, 31)
+        ql = q[(torch.arange(r0, r1, device=device) % L)].repeat_interleave(n)
+        x = (lsr(z, 32) * ql) >> 32
+        flat[r0 * n:r1 * n] = (x - ((x >> 31) << 32)).to(torch.int32)   # uint32 bits in int32
+    return out
+
+
 def structured(kind: str, primes, n: int, seed: int = 1) -> np.ndarray:
     """[1][L][n] structured inputs for parity edge cases."""
     primes = np.asarray(primes, dtype=np.int64)

@@ -1,0 +1,196 @@
+"""GPU parity: libwdntt.so (through the C ABI) vs the CPU oracle, bit for bit.
+
+Integer transforms have exactly one correct canonical answer,
+so every comparison is exact equality.  Small cases compare every row; the
+BASELINE.json full-size configs compare sampled rows against the oracle and
+check properties that hold at any size (round trip, sum rule) on every row.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs  # noqa: E402
+
+P = inputs.bench_primes(60)
+
+
+@pytest.fixture(scope="module")
+def wd():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import wdntt
+    return wdntt
+
+
+def to_dev(x: np.ndarray):
+    return torch.from_numpy(np.ascontiguousarray(x).view(np.int32)).cuda()
+
+
+def to_host(t) -> np.ndarray:
+    return t.cpu().numpy().view(np.uint32)
+
+
+def gpu_fwd(wd, plan, x, mode=None):
+    d = to_dev(x)
+    o = torch.empty_like(d)
+    if mode is not None:
+        plan.set_mode(mode)
+    plan.forward(d, o)
+    torch.cuda.synchronize()
+    return to_host(o)
+
+
+def gpu_inv(wd, plan, y):
+    d = to_dev(y)
+    o = torch.empty_like(d)
+    plan.inverse(d, o)
+    torch.cuda.synchronize()
+    return to_host(o)
+
+
+# -------------------------------------------------------------- config 1 (BASELINE configs[0])
+def test_config1_n4096_l4(wd):
+    primes = P[:4]
+    x = inputs.uniform_residues(primes, 1 << 12, 1, inputs.SEED_BASE + 0)
+    plan = wd.Plan(1 << 12, primes)
+    for l, q in enumerate(primes):
+        assert plan.psi(l) == oracle.psi_min(q, 1 << 12)
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes))
+    z = gpu_inv(wd, plan, y)
+    assert np.array_equal(z, x)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes))
+
+
+# -------------------------------------------------------------- every supported N, full rows
+@pytest.mark.parametrize("logn", list(range(1, 18)))
+def test_all_sizes_vs_oracle(wd, logn):
+    n = 1 << logn
+    primes = [P[0], P[11], P[37]]
+    batch = 3 if logn <= 15 else 2
+    x = inputs.uniform_residues(primes, n, batch, 1000 + logn)
+    plan = wd.Plan(n, primes)
+    y = gpu_fwd(wd, plan, x)
+    ref = oracle.ntt_forward(x, primes)
+    assert np.array_equal(y, ref)
+    assert np.array_equal(gpu_inv(wd, plan, y), x)
+    yi = gpu_inv(wd, plan, x)
+    assert np.array_equal(yi, oracle.ntt_inverse(x, primes))
+
+
+@pytest.mark.parametrize("logn", [12, 14, 16, 17])
+@pytest.mark.parametrize("kind", ["zeros", "qm1", "alt", "delta", "mono1", "mono4095", "ternary", "gauss"])
+def test_edge_inputs(wd, logn, kind):
+    n = 1 << logn
+    primes = [P[0], P[59]]
+    x = inputs.structured(kind, primes, n, seed=logn)
+    plan = wd.Plan(n, primes)
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes))
+    # all-(q-1) in the evaluation domain stresses the inverse's lazy bounds too
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes))
+
+
+@pytest.mark.parametrize("logn", [12, 16])
+def test_in_place_equals_out_of_place(wd, logn):
+    n = 1 << logn
+    primes = P[:5]
+    x = inputs.uniform_residues(primes, n, 2, 7)
+    plan = wd.Plan(n, primes)
+    d = to_dev(x)
+    o = torch.empty_like(d)
+    plan.forward(d, o)
+    plan.forward(d, d)
+    torch.cuda.synchronize()
+    assert torch.equal(d, o)
+    plan.inverse(d, d)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(d), x)
+
+
+def test_batch_zero_and_errors(wd):
+    plan = wd.Plan(1 << 12, P[:2])
+    d = torch.zeros(2 * 4096 + 4, dtype=torch.int32, device="cuda")
+    assert wd.wd_ntt_forward(plan.handle, d, d, 0) == 0
+    with pytest.raises(wd.WdNttError) as e:
+        wd.wd_ntt_forward(plan.handle, d.data_ptr() + 4, d.data_ptr() + 4, 1)
+    assert e.value.code == wd.WD_EINVAL
+
+
+def test_pointwise_inverse_is_negacyclic_product(wd):
+    # f1: INTT(NTT(a) o NTT(b)) = a * b mod (X^N + 1, q)
+    from oracle import brute
+    for logn in (6, 12):
+        n = 1 << logn
+        primes = P[:3]
+        a = inputs.uniform_residues(primes, n, 2, 11)
+        b = inputs.uniform_residues(primes, n, 2, 12)
+        plan = wd.Plan(n, primes)
+        A, B = to_dev(gpu_fwd(wd, plan, a)), to_dev(gpu_fwd(wd, plan, b))
+        o = torch.empty_like(A)
+        plan.pointwise_inverse(A, B, o)
+        torch.cuda.synchronize()
+        got = to_host(o)
+        fa, fb = oracle.ntt_forward(a, primes), oracle.ntt_forward(b, primes)
+        prod = (fa.astype(np.uint64) * fb.astype(np.uint64)) % np.array(primes, np.uint64)[None, :, None]
+        assert np.array_equal(got, oracle.ntt_inverse(prod.astype(np.uint32), primes))
+        if logn == 6:
+            for bi in range(2):
+                for l, q in enumerate(primes):
+                    assert got[bi, l].tolist() == brute.negacyclic_mul(a[bi, l].tolist(), b[bi, l].tolist(), q)
+
+
+# -------------------------------------------------------------- BASELINE configs at full size
+def _full_size_check(wd, n, L, batch, seed, nsample=12):
+    primes = P[:L]
+    x = inputs.uniform_residues(primes, n, batch, seed)
+    plan = wd.Plan(n, primes)
+    d = to_dev(x)
+    y = torch.empty_like(d)
+    plan.forward(d, y)
+    torch.cuda.synchronize()
+    # sampled rows vs oracle (same launch configuration as bench.py)
+    rng = np.random.default_rng(seed)
+    rows = rng.choice(batch * L, size=nsample, replace=False)
+    yh = to_host(y.view(batch * L, n)[torch.as_tensor(rows, device="cuda")])
+    for k, r in enumerate(rows):
+        b, l = divmod(int(r), L)
+        assert np.array_equal(yh[k], oracle.ntt_forward_row(x[b, l], primes[l])), (b, l)
+    # every row: sum rule  sum_i out[i] = N * x[0]  (mod q)
+    q = torch.tensor(primes, dtype=torch.int64, device="cuda").view(1, L)
+    s = y.view(batch, L, n).to(torch.int64).sum(-1) % q
+    x0 = d.view(batch, L, n)[:, :, 0].to(torch.int64)
+    assert torch.equal(s, (x0 * n) % q)
+    # every row: canonical range and exact round trip
+    assert bool((y.view(batch, L, n).to(torch.int64) < q.view(1, L, 1)).all())
+    z = torch.empty_like(y)
+    plan.inverse(y, z)
+    torch.cuda.synchronize()
+    assert torch.equal(z, d)
+    del d, y, z
+    torch.cuda.empty_cache()
+
+
+def test_config2_one_ciphertext(wd):
+    _full_size_check(wd, 1 << 16, 36, 2, inputs.SEED_BASE + 1, nsample=8)
+
+
+def test_config3_headline_64_ciphertexts(wd):
+    _full_size_check(wd, 1 << 16, 36, 128, inputs.SEED_BASE + 2)
+
+
+def test_config4_n131072_l48(wd):
+    _full_size_check(wd, 1 << 17, 48, 64, inputs.SEED_BASE + 3, nsample=8)
+
+
+@pytest.mark.parametrize("logn,L", [(12, 1), (13, 60), (14, 17), (15, 9), (16, 60), (17, 2)])
+def test_config5_sweep_batch1(wd, logn, L):
+    n = 1 << logn
+    primes = P[:L]
+    x = inputs.uniform_residues(primes, n, 2, 5000 + logn)   # batch 1 ciphertext
+    plan = wd.Plan(n, primes)
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes))
