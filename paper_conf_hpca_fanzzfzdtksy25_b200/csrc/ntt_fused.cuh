@@ -1,0 +1,175 @@
+// ntt_fused.cuh -- concurrent tensor-core + CUDA-core NTT/INTT for N = 2^16.
+//
+// WD-FUSE role of the paper (section IV-B, Fig. 3: tensor-core
+// warps and CUDA-core warps in the SAME block so that every SM sub-partition
+// holds both kinds of work; section IV-D3: the split follows the
+// units' relative throughput; Fig. 6: WD-FUSE beats either unit).
+// B200 design: one persistent CTA per SM with two warp groups --
+//   warps  0..15 (512 threads): CUDA-core chunk worker (radix-16 butterflies,
+//                                cp.async double-buffered chunks, ntt_persist.cuh)
+//   warps 16..19 (128 threads): tcgen05 worker (ntt_tensor.cuh); warp 16 owns
+//                                TMEM (its warp index is 0 mod 4, so warp 16+w
+//                                reads TMEM lanes 32w..32w+31)
+// Each group takes whole rows from the CTA's row list through a shared-memory
+// counter, so the split between the units is decided at run time by their
+// measured speed (a dynamic version of the paper's ratio knob).  If
+// tensor_share is given (0..1), rows are instead assigned statically:
+// row index i of the CTA goes to the tensor group iff frac(i*share) < share.
+#pragma once
+#include "ntt_tensor.cuh"
+
+namespace wd {
+
+constexpr int FU_CC = 512, FU_TC = 128, FU_T = FU_CC + FU_TC;
+constexpr int FU_CC_BAR = 2;
+constexpr int FU_SMEM = PGeo<16>::SMEM_BYTES + TC_SMEM + 64;
+
+template <int BAR, int NT>
+__device__ __forceinline__ void gbar() {
+    if constexpr (BAR == 0) __syncthreads();
+    else named_bar(BAR, NT);
+}
+
+// one whole row on the CUDA-core group (chunk pipeline of ntt_persist.cuh, named barrier BAR)
+template <bool FWD, bool PW, int BAR>
+__device__ __forceinline__ void cc_row(const NttArgs& a, uint32_t* smem, uint32_t row_id) {
+    using G = PGeo<16>;
+    constexpr int CA = FWD ? G::C1 : G::C2;
+    constexpr int CH = G::C1 + G::C2;
+    const uint32_t* in = a.in + ((size_t)row_id << 16);
+    uint32_t* out = a.out + ((size_t)row_id << 16);
+    const uint32_t limb = row_id % a.L;
+    const LimbConst lc = a.lc[limb];
+    const uint2* __restrict__ tw = a.tw + ((size_t)limb << 16);
+    auto issue = [&](int kk, uint32_t* S) {
+        if (FWD) {
+            if (kk < G::C1) load_p1<16>(S, in, kk * G::W1);
+            else load_p2<16>(S, out, (kk - G::C1) * G::W2);
+        } else {
+            if (kk < G::C2) load_p2<16>(S, in, kk * G::W2);
+            else load_p1<16>(S, out, (kk - G::C2) * G::W1);
+        }
+        cp_async_commit();
+    };
+    issue(0, smem);
+#pragma unroll 1
+    for (int kk = 0; kk < CH; ++kk) {
+        uint32_t* S = smem + (kk & 1) * G::BUF_WORDS;
+        const bool dep = (kk + 1 == CA);
+        if (kk + 1 < CH && !dep) {
+            issue(kk + 1, smem + ((kk + 1) & 1) * G::BUF_WORDS);
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
+        gbar<BAR, FU_CC>();
+        if (FWD) {
+            if (kk < G::C1) fwd_p1_chunk<16, BAR>(S, out, kk * G::W1, tw, lc.q, lc.q2);
+            else fwd_p2_chunk<16, BAR>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
+        } else {
+            const uint32_t* in2 = a.in2 + ((size_t)row_id << 16);
+            if (kk < G::C2) inv_p2_chunk<16, PW, BAR>(S, out, in2, kk * G::W2, tw, lc);
+            else inv_p1_chunk<16, BAR>(S, out, (kk - G::C2) * G::W1, tw, lc);
+        }
+        __threadfence_block();
+        gbar<BAR, FU_CC>();
+        if (dep) issue(kk + 1, smem + ((kk + 1) & 1) * G::BUF_WORDS);
+    }
+}
+
+template <bool FWD, bool PW>
+__global__ void __launch_bounds__(FU_T, 1) ntt_fused16(TcArgs ta, uint32_t rows, float share) {
+    extern __shared__ __align__(1024) uint8_t fsm[];
+    uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
+    uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
+    int* ctl = reinterpret_cast<int*>(tcb + TC_SMEM);           // [0] counter, [1] cc slot, [2] tc slot
+    TcShared sh;
+    sh.Ain = tcb;
+    sh.Amid = tcb + 4 * TC_TILE;
+    sh.B = tcb + 8 * TC_TILE;
+    sh.stg = reinterpret_cast<uint32_t*>(tcb + 8 * TC_TILE + 8192);
+    sh.bar = reinterpret_cast<uint64_t*>(tcb + 8 * TC_TILE + 8192 + 32 * 257 * 4);
+    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        ctl[0] = 0;
+        mbar_init(&sh.bar[0], 1);
+        mbar_init(&sh.bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (tid >= FU_CC && tid < FU_CC + 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(sh.tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t nmine = rows > blockIdx.x ? (rows - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    const bool is_tc = tid >= FU_CC;
+    const int gtid = is_tc ? tid - FU_CC : tid;
+    // static split helper: does CTA-local row index i belong to the tensor group?
+    auto tc_owns = [&](uint32_t i) { return floorf((float)(i + 1) * share) > floorf((float)i * share); };
+    uint32_t sidx = 0;                                           // static-mode cursor
+    if (is_tc) {
+        const uint32_t tmem = *sh.tslot;
+        uint32_t ph[2] = {0, 0};
+        for (;;) {
+            uint32_t i;
+            if (share >= 0.0f) {
+                while (sidx < nmine && !tc_owns(sidx)) ++sidx;
+                i = sidx++;
+            } else {
+                if (gtid == 0) ctl[2] = atomicAdd(&ctl[0], 1);
+                named_bar(TC_BAR_ID, FU_TC);
+                i = (uint32_t)ctl[2];
+                named_bar(TC_BAR_ID, FU_TC);
+            }
+            if (i >= nmine) break;
+            tc_transform<FWD>(ta, sh, tmem, ph, blockIdx.x + i * gridDim.x);
+        }
+        tc_fence_before();
+        named_bar(TC_BAR_ID, FU_TC);
+        if (gtid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
+    } else {
+        for (;;) {
+            uint32_t i;
+            if (share >= 0.0f) {
+                while (sidx < nmine && tc_owns(sidx)) ++sidx;
+                i = sidx++;
+            } else {
+                if (gtid == 0) ctl[1] = atomicAdd(&ctl[0], 1);
+                named_bar(FU_CC_BAR, FU_CC);
+                i = (uint32_t)ctl[1];
+                named_bar(FU_CC_BAR, FU_CC);
+            }
+            if (i >= nmine) break;
+            cc_row<FWD, PW, FU_CC_BAR>(ta.a, ccbuf, blockIdx.x + i * gridDim.x);
+        }
+    }
+}
+
+inline int prepare_fused_kernels(uint32_t logN) {
+    if (logN != 16) return 0;
+    if (cudaFuncSetAttribute(ntt_fused16<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess ||
+        cudaFuncSetAttribute(ntt_fused16<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess)
+        return 4;
+    return 0;
+}
+
+inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows,
+                        int sm_count, float share, cudaStream_t s) {
+    if (logN != 16 || !tc.ok || a.in2) return -1;
+    TcArgs ta;
+    ta.a = a;
+    ta.B = tc.d_B;
+    ta.t1 = fwd ? tc.d_tw1 : tc.d_sg1;
+    ta.t2 = fwd ? tc.d_tw2 : tc.d_sg2;
+    ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
+    ta.c16 = tc.d_c16;
+    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
+    if (fwd) ntt_fused16<true, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);
+    else ntt_fused16<false, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);
+    return 1;
+}
+
+}  // namespace wd

@@ -1,0 +1,312 @@
+// ntt_persist.cuh -- persistent, cp.async-pipelined CUDA-core NTT/INTT for N = 2^15..2^17
+// (the large-N "dual kernel" case of PAPER.md:366).
+//
+// One CTA per SM loops over its share of the batch*L rows (PE-kernel idea,
+// PAPER.md:334-352).  A row is N = N1 x 256: phase 1 = the first log2(N1)
+// merged-CT layers on 256 columns (stride 256), phase 2 = the last 8 layers on
+// N1 contiguous 256-word rows (the paper's 4-step / 7-step decomposition,
+// PAPER.md:93-100, 272-282, without the transpose -> bit-reversed output).
+// Each phase is cut into CHUNKS of ~8192 words.  A chunk is copied global ->
+// shared with 16-byte cp.async (LDGSTS) one chunk ahead of its use (double
+// buffer), then two register stages run on it IN PLACE in shared memory
+// (radix 2^A0 then 2^A1 on columns, radix 16 x 16 on rows), so the
+// inter-stage exchange needs no extra buffer.  Phase-1 results go to the
+// row's own output slot (L2-resident), phase 2 reads them back.
+#pragma once
+#include <cstdint>
+#include "modarith.cuh"
+#include "ntt_cuda_core.cuh"
+
+namespace wd {
+
+__device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc) {
+    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
+
+// barrier among the 512 CUDA-core threads: __syncthreads when they are the whole CTA,
+// a named barrier when they share the CTA with the tensor group (ntt_fused.cuh)
+template <int BAR>
+__device__ __forceinline__ void pbar() {
+    if constexpr (BAR == 0) __syncthreads();
+    else asm volatile("bar.sync %0, 512;" :: "n"(BAR) : "memory");
+}
+
+template <int LOGN> struct PCfg;
+template <> struct PCfg<15> { static constexpr int A0 = 4, A1 = 3; };
+template <> struct PCfg<16> { static constexpr int A0 = 4, A1 = 4; };
+template <> struct PCfg<17> { static constexpr int A0 = 5, A1 = 4; };
+
+template <int LOGN>
+struct PGeo {
+    static constexpr int T = 512;
+    static constexpr int A0 = PCfg<LOGN>::A0, A1 = PCfg<LOGN>::A1;
+    static constexpr int B1 = LOGN - 8, N1 = 1 << B1;
+    static constexpr int R0 = 1 << A0, R1 = 1 << A1;
+    static constexpr int E1 = R0 > R1 ? R0 : R1;
+    static constexpr int G1 = N1 / E1;               // threads per column
+    static constexpr int W1 = T / G1;                // columns per phase-1 chunk
+    static constexpr int C1 = 256 / W1;              // phase-1 chunks per row
+    static constexpr int INST0 = E1 / R0, INST1 = E1 / R1;
+    static constexpr int W2 = T / 16;                // rows per phase-2 chunk
+    static constexpr int C2 = N1 / W2;               // phase-2 chunks per row
+    static constexpr int P1_WORDS = N1 * W1;
+    static constexpr int P2_WORDS = W2 * RS;
+    static constexpr int BUF_WORDS = P1_WORDS > P2_WORDS ? P1_WORDS : P2_WORDS;
+    static constexpr int SMEM_BYTES = 2 * 4 * BUF_WORDS;
+    static_assert(W1 % 4 == 0 && W1 >= 16 && 256 % W1 == 0, "phase-1 chunk");
+    static_assert(N1 % W2 == 0, "phase-2 chunk");
+};
+
+// ---- chunk loads (all T threads) --------------------------------------------------------
+// phase-1 chunk: columns [c0, c0+W1) of every one of the N1 256-word rows -> S[p*W1 + w]
+template <int LOGN>
+__device__ __forceinline__ void load_p1(uint32_t* S, const uint32_t* src, int c0) {
+    using G = PGeo<LOGN>;
+    constexpr int SEG = G::W1 / 4, NSEG = G::N1 * SEG;
+#pragma unroll
+    for (int i = threadIdx.x; i < NSEG; i += G::T) {
+        const int p = i / SEG, s = i % SEG;
+        cp_async16(S + p * G::W1 + 4 * s, src + p * 256 + c0 + 4 * s);
+    }
+}
+// phase-2 chunk: rows [r0, r0+W2), 256 words each -> swizzled ywords() layout
+template <int LOGN>
+__device__ __forceinline__ void load_p2(uint32_t* S, const uint32_t* src, int r0) {
+    using G = PGeo<LOGN>;
+    constexpr int NSEG = G::W2 * 64;
+#pragma unroll
+    for (int i = threadIdx.x; i < NSEG; i += G::T) {
+        const int w = i >> 6, v4 = i & 63, chi = v4 >> 2, v = v4 & 3;
+        cp_async16(S + w * RS + chi * 16 + (((v ^ (chi >> 1)) & 3) << 2), src + (r0 + w) * 256 + 4 * v4);
+    }
+}
+
+// ---- forward chunk compute ------------------------------------------------------------
+template <int LOGN, int BAR = 0>
+__device__ __forceinline__ void fwd_p1_chunk(uint32_t* S, uint32_t* out, int c0, const uint2* __restrict__ tw,
+                                             uint32_t q, uint32_t q2) {
+    using G = PGeo<LOGN>;
+    const int w = threadIdx.x % G::W1, j = threadIdx.x / G::W1;
+    uint32_t x[G::E1];
+#pragma unroll
+    for (int u = 0; u < G::INST0; ++u) {
+        const int i0 = j * G::INST0 + u;
+#pragma unroll
+        for (int r = 0; r < G::R0; ++r) x[u * G::R0 + r] = S[(i0 + (r << G::A1)) * G::W1 + w];
+        fwd_radix<G::A0>(x + u * G::R0, tw, 0, 0, q, q2);
+#pragma unroll
+        for (int r = 0; r < G::R0; ++r) S[(i0 + (r << G::A1)) * G::W1 + w] = x[u * G::R0 + r];
+    }
+    pbar<BAR>();
+    const int c = c0 + w;
+#pragma unroll
+    for (int u = 0; u < G::INST1; ++u) {
+        const int i1 = j * G::INST1 + u;
+#pragma unroll
+        for (int r = 0; r < G::R1; ++r) x[r] = S[((i1 << G::A1) + r) * G::W1 + w];
+        fwd_radix<G::A1>(x, tw, G::A0, i1, q, q2);
+#pragma unroll
+        for (int r = 0; r < G::R1; ++r) out[((i1 << G::A1) + r) * 256 + c] = x[r];
+    }
+}
+
+// stage-3 twiddles of one 16-point block: Psi[4096+g], Psi[8192+2g..], Psi[16384+4g..], Psi[32768+8g..]
+// (generic: layer ls..ls+3 with group hi) fetched as 16-byte vectors.
+__device__ __forceinline__ void load_tw16(uint2* w, const uint2* __restrict__ tw, int ls, uint32_t hi) {
+    w[0] = __ldg(tw + (1u << ls) + hi);
+    const uint4 a = __ldg(reinterpret_cast<const uint4*>(tw + (2u << ls) + 2 * hi));
+    w[1] = make_uint2(a.x, a.y); w[2] = make_uint2(a.z, a.w);
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const uint4 b = __ldg(reinterpret_cast<const uint4*>(tw + (4u << ls) + 4 * hi) + k);
+        w[3 + 2 * k] = make_uint2(b.x, b.y); w[4 + 2 * k] = make_uint2(b.z, b.w);
+    }
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const uint4 b = __ldg(reinterpret_cast<const uint4*>(tw + (8u << ls) + 8 * hi) + k);
+        w[7 + 2 * k] = make_uint2(b.x, b.y); w[8 + 2 * k] = make_uint2(b.z, b.w);
+    }
+}
+// radix-16 forward block with explicit twiddles w[0..14] (layer t group g -> w[(1<<t)-1+g])
+__device__ __forceinline__ void fwd16_tw(uint32_t* x, const uint2* w, uint32_t q, uint32_t q2) {
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+        const int h = 8 >> t;
+#pragma unroll
+        for (int g = 0; g < (1 << t); ++g)
+#pragma unroll
+            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w[(1 << t) - 1 + g], q, q2);
+    }
+}
+__device__ __forceinline__ void inv16_tw(uint32_t* x, const uint2* w, uint32_t q, uint32_t q2) {
+#pragma unroll
+    for (int t = 3; t >= 0; --t) {
+        const int h = 8 >> t;
+#pragma unroll
+        for (int g = 0; g < (1 << t); ++g)
+#pragma unroll
+            for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w[(1 << t) - 1 + g], q, q2);
+    }
+}
+
+template <int LOGN, int BAR = 0>
+__device__ __forceinline__ void fwd_p2_chunk(uint32_t* S, uint32_t* out, int r0, const uint2* __restrict__ tw,
+                                             uint32_t q, uint32_t q2) {
+    using G = PGeo<LOGN>;
+    const int c = threadIdx.x & 15, w = threadIdx.x >> 4;
+    const int row = r0 + w;
+    uint32_t x[16];
+    uint2 w3[15];
+    load_tw16(w3, tw, G::B1 + 4, (uint32_t)row * 16 + c);      // in flight during stage 2
+#pragma unroll
+    for (int r = 0; r < 16; ++r) x[r] = S[ywords(w, r, c)];
+    fwd_radix<4>(x, tw, G::B1, row, q, q2);
+#pragma unroll
+    for (int r = 0; r < 16; ++r) S[ywords(w, r, c)] = x[r];
+    pbar<BAR>();
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+        const uint4 t = *reinterpret_cast<const uint4*>(S + w * RS + c * 16 + (((v ^ (c >> 1)) & 3) << 2));
+        x[4 * v] = t.x; x[4 * v + 1] = t.y; x[4 * v + 2] = t.z; x[4 * v + 3] = t.w;
+    }
+    fwd16_tw(x, w3, q, q2);
+    uint4* o = reinterpret_cast<uint4*>(out + row * 256 + c * 16);
+#pragma unroll
+    for (int v = 0; v < 4; ++v)
+        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
+                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+}
+
+// ---- inverse chunk compute (phase 2' then phase 1') ---------------------------------------
+template <int LOGN, bool PW, int BAR = 0>
+__device__ __forceinline__ void inv_p2_chunk(uint32_t* S, uint32_t* out, const uint32_t* in2, int r0,
+                                             const uint2* __restrict__ tw, const LimbConst& lc) {
+    using G = PGeo<LOGN>;
+    const int c = threadIdx.x & 15, w = threadIdx.x >> 4;
+    const int row = r0 + w;
+    uint32_t x[16];
+    uint2 w3[15];
+    load_tw16(w3, tw, G::B1 + 4, (uint32_t)row * 16 + c);
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+        const uint4 t = *reinterpret_cast<const uint4*>(S + w * RS + c * 16 + (((v ^ (c >> 1)) & 3) << 2));
+        x[4 * v] = t.x; x[4 * v + 1] = t.y; x[4 * v + 2] = t.z; x[4 * v + 3] = t.w;
+    }
+    if constexpr (PW) {
+        const uint4* ip2 = reinterpret_cast<const uint4*>(in2 + row * 256 + c * 16);
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const uint4 t = __ldcs(ip2 + v);
+            x[4 * v] = mul_mod(x[4 * v], t.x, lc); x[4 * v + 1] = mul_mod(x[4 * v + 1], t.y, lc);
+            x[4 * v + 2] = mul_mod(x[4 * v + 2], t.z, lc); x[4 * v + 3] = mul_mod(x[4 * v + 3], t.w, lc);
+        }
+    }
+    inv16_tw(x, w3, lc.q, lc.q2);
+#pragma unroll
+    for (int v = 0; v < 4; ++v)
+        *reinterpret_cast<uint4*>(S + w * RS + c * 16 + (((v ^ (c >> 1)) & 3) << 2)) =
+            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+    pbar<BAR>();
+#pragma unroll
+    for (int r = 0; r < 16; ++r) x[r] = S[ywords(w, r, c)];
+    inv_radix<4, false>(x, tw, G::B1, row, lc);
+#pragma unroll
+    for (int r = 0; r < 16; ++r) out[row * 256 + c + 16 * r] = x[r];
+}
+
+template <int LOGN, int BAR = 0>
+__device__ __forceinline__ void inv_p1_chunk(uint32_t* S, uint32_t* out, int c0, const uint2* __restrict__ tw,
+                                             const LimbConst& lc) {
+    using G = PGeo<LOGN>;
+    const int w = threadIdx.x % G::W1, j = threadIdx.x / G::W1;
+    uint32_t x[G::E1];
+#pragma unroll
+    for (int u = 0; u < G::INST1; ++u) {
+        const int i1 = j * G::INST1 + u;
+#pragma unroll
+        for (int r = 0; r < G::R1; ++r) x[r] = S[((i1 << G::A1) + r) * G::W1 + w];
+        inv_radix<G::A1, false>(x, tw, G::A0, i1, lc);
+#pragma unroll
+        for (int r = 0; r < G::R1; ++r) S[((i1 << G::A1) + r) * G::W1 + w] = x[r];
+    }
+    pbar<BAR>();
+    const int c = c0 + w;
+#pragma unroll
+    for (int u = 0; u < G::INST0; ++u) {
+        const int i0 = j * G::INST0 + u;
+#pragma unroll
+        for (int r = 0; r < G::R0; ++r) x[u * G::R0 + r] = S[(i0 + (r << G::A1)) * G::W1 + w];
+        inv_radix<G::A0, true>(x + u * G::R0, tw, 0, 0, lc);
+#pragma unroll
+        for (int r = 0; r < G::R0; ++r)
+            __stcs(out + (i0 + (r << G::A1)) * 256 + c, canon2(x[u * G::R0 + r], lc.q));
+    }
+}
+
+// ---- the persistent kernel ---------------------------------------------------------------
+// chunk k of a row: forward  k <  C1 -> phase-1 chunk k (src = in),  else phase-2 chunk k-C1 (src = out)
+//                   inverse  k <  C2 -> phase-2' chunk k (src = in), else phase-1' chunk k-C2 (src = out)
+template <int LOGN, bool FWD, bool PW>
+__global__ void __launch_bounds__(512, 2) ntt_persist_cc(NttArgs a, uint32_t rows) {
+    using G = PGeo<LOGN>;
+    constexpr int CA = FWD ? G::C1 : G::C2;          // chunks of the first phase
+    constexpr int CH = G::C1 + G::C2;
+    extern __shared__ __align__(16) uint32_t smem[];
+
+    const uint32_t nmine = rows > blockIdx.x ? (rows - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    const uint32_t total = nmine * CH;
+    if (total == 0) return;
+
+    auto issue = [&](uint32_t k, uint32_t* S) {
+        const uint32_t row_id = blockIdx.x + (k / CH) * gridDim.x;
+        const int kk = k % CH;
+        const uint32_t* in = a.in + ((size_t)row_id << LOGN);
+        const uint32_t* mid = a.out + ((size_t)row_id << LOGN);
+        if (FWD) {
+            if (kk < G::C1) load_p1<LOGN>(S, in, kk * G::W1);
+            else load_p2<LOGN>(S, mid, (kk - G::C1) * G::W2);
+        } else {
+            if (kk < G::C2) load_p2<LOGN>(S, in, kk * G::W2);
+            else load_p1<LOGN>(S, mid, (kk - G::C2) * G::W1);
+        }
+        cp_async_commit();
+    };
+
+    issue(0, smem);
+    for (uint32_t k = 0; k < total; ++k) {
+        uint32_t* S = smem + (k & 1) * G::BUF_WORDS;
+        const int kk = k % CH;
+        // chunk k+1 may be the first chunk of phase B of this row: it reads what this chunk writes
+        const bool dep = (k + 1 < total) && ((k + 1) % CH == (uint32_t)CA);
+        if (k + 1 < total && !dep) {
+            issue(k + 1, smem + ((k + 1) & 1) * G::BUF_WORDS);
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
+        __syncthreads();
+
+        const uint32_t row_id = blockIdx.x + (k / CH) * gridDim.x;
+        const uint32_t limb = row_id % a.L;
+        const LimbConst lc = a.lc[limb];
+        const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+        uint32_t* out = a.out + ((size_t)row_id << LOGN);
+        if (FWD) {
+            if (kk < G::C1) fwd_p1_chunk<LOGN>(S, out, kk * G::W1, tw, lc.q, lc.q2);
+            else fwd_p2_chunk<LOGN>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
+        } else {
+            const uint32_t* in2 = a.in2 + ((size_t)row_id << LOGN);
+            if (kk < G::C2) inv_p2_chunk<LOGN, PW>(S, out, in2, kk * G::W2, tw, lc);
+            else inv_p1_chunk<LOGN>(S, out, (kk - G::C2) * G::W1, tw, lc);
+        }
+        __threadfence_block();
+        __syncthreads();
+        if (dep) issue(k + 1, smem + ((k + 1) & 1) * G::BUF_WORDS);
+    }
+}
+
+}  // namespace wd

@@ -1,20 +1,467 @@
-// ntt_tensor.cuh -- tcgen05 int8 tensor-core path.  [stub: filled in next]
+// ntt_tensor.cuh -- tcgen05 int8 tensor-core NTT/INTT for N = 2^16.
+//
+// WD-Tensor role of the paper (Alg.2 "OneStageNTTKernel";
+// 4-step decomposition PAPER.md:93-100, 272-290 with inner dimension 16),
+// re-derived for sm_100a:
+//   * N = 2^16 = 256 columns x 256 rows; phase 1 = two radix-16 stages on
+//     32-column chunks, phase 2 = two radix-16 stages on 32-row chunks
+//     (intermediate through the row's own output slot, L2-resident).
+//   * a radix-16 stage over 512 instances = 4 MMA tiles of M = 128 rows; one
+//     row = one 16-point inner NTT whose 16 u32 inputs are 64 bytes along K
+//     (the u8 view of the words, SURVEY H-3: no bit-splitting pass);
+//     B = 64 x 64 byte planes of the stage matrix (tensor_tables.h);
+//     D = 128 x 64 s32 in TMEM: 4 byte-plane partial sums per output.
+//   * tcgen05.mma.cta_group::1.kind::i8 (u8 x u8 -> s32) issued by one thread,
+//     operands in shared memory (K-major, no swizzle), accumulators in TMEM,
+//     completion via tcgen05.commit -> mbarrier; two TMEM regions ping-pong so
+//     the MMA of tile t+2 overlaps the epilogue of tile t.
+//   * CUDA-core epilogue (tcgen05.ld 32x32b): Y = D0 + 2^8 D1 + 2^16 (D2 + 2^8 D3)
+//     mod q (one Shoup multiply by 2^16), then the per-group twist of the next
+//     stage (forward) / of this stage (inverse), then a conflict-free scalar
+//     st.shared into the next stage's operand tile, or global stores.
+//   * stage 0 (forward) / stage 0' (inverse, with N^-1) have a single group,
+//     so their twist is folded into the matrix; the other stages use the fixed
+//     DFT16 F (F') and a CUDA-core twist -- the paper's Hadamard step
+//     (steps 2/4/6 of Fig. 2).
 #pragma once
+#include <cuda_runtime.h>
 #include <cstdint>
 #include <vector>
+#include "modarith.cuh"
 #include "ntt_cuda_core.cuh"
+#include "ntt_persist.cuh"
+#include "tensor_tables.h"
 
 namespace wd {
 
 struct TensorTables {
-    void* d_planes = nullptr;
+    uint8_t* d_B = nullptr;        // [L][4][4096]: fwd M0, fwd F, inv MI0 (with N^-1), inv F'
+    uint2* d_tw1 = nullptr;        // [L][16][16]    fwd twist tau, stage 1   (group, j)
+    uint2* d_tw2 = nullptr;        // [L][256][16]   fwd twist tau, stage 2
+    uint2* d_tw3 = nullptr;        // [L][4096][16]  fwd twist tau, stage 3
+    uint2* d_sg1 = nullptr;        // [L][16][16]    inv twist sigma, stage 1' (group, k)
+    uint2* d_sg2 = nullptr;        // [L][256][16]
+    uint2* d_sg3 = nullptr;        // [L][4096][16]
+    uint2* d_c16 = nullptr;        // [L] Shoup companions of 2^16 and of 1
+    bool ok = false;
 };
 
-inline bool tensor_supported(uint32_t) { return false; }
-inline float default_tensor_share(uint32_t) { return 0.0f; }
-inline int build_tensor_tables(TensorTables&, uint32_t, const std::vector<uint32_t>&, const std::vector<uint32_t>&) { return 0; }
-inline void free_tensor_tables(TensorTables& t) { if (t.d_planes) cudaFree(t.d_planes); t.d_planes = nullptr; }
-inline int prepare_tensor_kernels(uint32_t) { return 0; }
-inline int launch_tensor(uint32_t, bool, const NttArgs&, const TensorTables&, uint32_t, float, cudaStream_t) { return -1; }
+struct TcArgs {
+    NttArgs a;
+    const uint8_t* B;
+    const uint2 *t1, *t2, *t3;
+    const uint2* c16;
+};
+
+inline bool tensor_supported(uint32_t logN) { return logN == 16; }
+inline float default_tensor_share(uint32_t) { return -1.0f; }   // < 0: dynamic split in FUSED mode
+
+// ------------------------------------------------------------------ device helpers
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {       // K-major, SWIZZLE_NONE, LBO 128, SBO 512
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)(128 >> 4) << 16) | ((uint64_t)(512 >> 4) << 32) |
+           ((uint64_t)1 << 46);
+}
+constexpr uint32_t IDESC_I8_128x64 = (2u << 4) | ((uint32_t)(64 >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+
+__device__ __forceinline__ void tc_mma(uint32_t d, uint64_t a, uint64_t b, uint32_t acc) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
+                 :: "r"(d), "l"(a), "l"(b), "r"(IDESC_I8_128x64), "r"(acc));
+}
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                 :: "r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t n) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_addr(bar)), "r"(n));
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t ph) {
+    asm volatile("{\n\t.reg .pred P1;\n\tTCW_%=:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+                 "@!P1 bra TCW_%=;\n\t}\n" :: "r"(smem_addr(bar)), "r"(ph) : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(n) : "memory"); }
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+        "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+__device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(smem_addr(smem_dst)), "l"(gsrc) : "memory");
+}
+
+// byte offset of (row m, coefficient j) inside one 128 x 64-byte operand tile
+__device__ __forceinline__ uint32_t aoff_w(int m, int j) {
+    return (uint32_t)((m & 7) * 16 + (m >> 3) * 512 + (j >> 2) * 128 + (j & 3) * 4);
+}
+
+// Y = sum_b 2^(8b) D_b mod-ish: result < 2^32, congruent mod q
+__device__ __forceinline__ uint32_t combine(const uint32_t* d, uint32_t q, uint32_t c16s) {
+    const uint32_t lo = d[0] + (d[1] << 8);
+    const uint32_t hi = d[2] + (d[3] << 8);
+    return lo + shoup_mul(hi, 65536u, c16s, q);
+}
+
+// ------------------------------------------------------------------ the kernel
+constexpr int TC_T = 128;                 // threads (4 warps; warp w owns TMEM lanes 32w..32w+31)
+constexpr int TC_TILE = 128 * 64;         // bytes per operand tile
+constexpr int TC_SMEM = 2 * 4 * TC_TILE   // A_in, A_mid (4 tiles each)
+                        + 2 * 4096        // B images of the two stages of this phase
+                        + 32 * 257 * 4    // inverse stage-2' staging (row stride 257 words)
+                        + 64;             // mbarriers + TMEM address
+constexpr int TC_BAR_ID = 1;              // named barrier used by the tensor group
+
+struct TcShared {
+    uint8_t* Ain; uint8_t* Amid; uint8_t* B; uint32_t* stg; uint64_t* bar; uint32_t* tslot;
+};
+
+// one radix-16 stage over the 4 tiles of Abuf with B image Bimg; epi(t, d[64]) consumes tile t
+template <typename Epi>
+__device__ __forceinline__ void tc_stage(const TcShared& sh, uint32_t tmem, const uint8_t* Abuf, const uint8_t* Bimg,
+                                         uint32_t* ph, Epi&& epi) {
+    const int tid = threadIdx.x % TC_T, w = tid >> 5;
+    const uint32_t a0 = smem_addr(Abuf), b0 = smem_addr(Bimg);
+    auto issue = [&](int t) {
+        const uint32_t d = tmem + (t & 1) * 64;
+        tc_fence_after();
+        tc_mma(d, umma_desc(a0 + t * TC_TILE), umma_desc(b0), 0);
+        tc_mma(d, umma_desc(a0 + t * TC_TILE + 256), umma_desc(b0 + 256), 1);
+        tc_commit(&sh.bar[t & 1]);
+    };
+    if (tid == 0) { issue(0); issue(1); }
+#pragma unroll 1
+    for (int t = 0; t < 4; ++t) {
+        const int r = t & 1;
+        mbar_wait(&sh.bar[r], ph[r]);
+        ph[r] ^= 1;
+        tc_fence_after();
+        uint32_t d[64];
+        const uint32_t ta = tmem + ((uint32_t)(32 * w) << 16) + r * 64;
+        tmem_ld32(ta, d);
+        tmem_ld32(ta + 32, d + 32);
+        tmem_wait_ld();
+        tc_fence_before();
+        named_bar(TC_BAR_ID, TC_T);
+        if (tid == 0 && t + 2 < 4) issue(t + 2);
+        epi(t, d);
+    }
+}
+
+template <bool FWD>
+__device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& sh, uint32_t tmem, uint32_t* ph,
+                                             uint32_t row_id) {
+    const NttArgs& a = ta.a;
+    const int tid = threadIdx.x % TC_T, w = tid >> 5, lane = tid & 31;
+    const uint32_t limb = row_id % a.L;
+    const LimbConst lc = a.lc[limb];
+    const uint32_t q = lc.q, q2 = lc.q2;
+    const uint2 cc = ta.c16[limb];
+    const uint32_t c16s = cc.x, one_s = cc.y;
+    const uint32_t* in = a.in + ((size_t)row_id << 16);
+    uint32_t* out = a.out + ((size_t)row_id << 16);
+    const uint8_t* Bl = ta.B + (size_t)limb * 4 * 4096 + (FWD ? 0 : 2 * 4096);
+    const uint2* T1 = ta.t1 + (size_t)limb * 256;
+    const uint2* T2 = ta.t2 + (size_t)limb * 4096;
+    const uint2* T3 = ta.t3 + (size_t)limb * 65536;
+
+    // B images: [0] = folded single-group matrix (M0 or MI0), [1] = fixed DFT16 (F or F')
+    for (int i = tid; i < 2 * 4096 / 16; i += TC_T)
+        cp_async16(sh.B + 16 * i, Bl + 16 * i);
+    cp_async_commit();
+
+    for (int ch = 0; ch < 16; ++ch) {
+        const bool phase1 = FWD ? (ch < 8) : (ch >= 8);
+        const int k8 = ch & 7;
+        const int c0 = 32 * k8, r0 = 32 * k8;
+        // ---------------- load the chunk into the first stage's operand tiles
+        if (FWD && phase1) {                       // F-S0: (c, i0), coeff r, p = i0 + 16 r
+#pragma unroll 4
+            for (int e = tid; e < 8192; e += TC_T) {
+                const int p = e >> 5, c = e & 31, i0 = p & 15, r = p >> 4;
+                const int t = i0 >> 2, m = (c & 7) + 8 * (i0 & 3) + 32 * (c >> 3);
+                cp_async4(sh.Ain + t * TC_TILE + aoff_w(m, r), in + p * 256 + c0 + c);
+            }
+        } else if (FWD) {                          // F-S2: (rho, clo), coeff chi, col = clo + 16 chi
+#pragma unroll 4
+            for (int e = tid; e < 8192; e += TC_T) {
+                const int rho = e >> 8, col = e & 255, clo = col & 15, chi = col >> 4;
+                const int t = clo >> 2, m = (rho & 7) + 8 * (clo & 3) + 32 * (rho >> 3);
+                cp_async4(sh.Ain + t * TC_TILE + aoff_w(m, chi), out + (r0 + rho) * 256 + col);
+            }
+        } else if (!phase1) {                      // I-S3: (rho, chi), coeff clo (16-byte runs)
+#pragma unroll 4
+            for (int s = tid; s < 2048; s += TC_T) {
+                const int rho = s >> 6, chi = (s >> 2) & 15, v = s & 3;
+                const int t = chi >> 2, m = (rho & 7) + 8 * (chi & 3) + 32 * (rho >> 3);
+                cp_async16(sh.Ain + t * TC_TILE + aoff_w(m, 4 * v), in + (r0 + rho) * 256 + 16 * chi + 4 * v);
+            }
+        } else {                                   // I-S1: (c, i1), coeff j, p = 16 i1 + j
+#pragma unroll 4
+            for (int e = tid; e < 8192; e += TC_T) {
+                const int p = e >> 5, c = e & 31, i1 = p >> 4, j = p & 15;
+                const int t = i1 >> 2, m = (c & 7) + 8 * (i1 & 3) + 32 * (c >> 3);
+                cp_async4(sh.Ain + t * TC_TILE + aoff_w(m, j), out + p * 256 + c0 + c);
+            }
+        }
+        cp_async_commit();
+        cp_async_wait<0>();
+        fence_async_smem();
+        named_bar(TC_BAR_ID, TC_T);
+
+        if (FWD && phase1) {
+            // stage 0 (folded M0) -> twist tau1 -> A_mid (F-S1 layout)
+            tc_stage(sh, tmem, sh.Ain, sh.B, ph, [&](int t, const uint32_t* d) {
+                const int c = (lane & 7) + 8 * w, i0 = 4 * t + (lane >> 3);
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const uint2 tw = __ldg(T1 + k * 16 + i0);
+                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), tw.x, tw.y, q);
+                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + c, i0)) = z;
+                }
+            });
+            fence_async_smem();
+            named_bar(TC_BAR_ID, TC_T);
+            // stage 1 (F) -> twist tau2 -> intermediate (coalesced over c)
+            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+                const int i1 = 4 * t + w, c = lane;
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const int p = 16 * i1 + k;
+                    const uint2 tw = __ldg(T2 + p * 16 + ((c0 + c) >> 4));
+                    out[p * 256 + c0 + c] = shoup_mul(combine(d + 4 * k, q, c16s), tw.x, tw.y, q);
+                }
+            });
+        } else if (FWD) {
+            // stage 2 (F) -> twist tau3 -> A_mid (F-S3 layout)
+            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+                const int rho = (lane & 7) + 8 * w, clo = 4 * t + (lane >> 3);
+                const uint2* t3 = T3 + (size_t)(r0 + rho) * 256 + clo;        // group (row*16 + k), j = clo
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const uint2 tw = __ldg(t3 + 16 * k);
+                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), tw.x, tw.y, q);
+                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + rho, clo)) = z;
+                }
+            });
+            fence_async_smem();
+            named_bar(TC_BAR_ID, TC_T);
+            // stage 3 (F) -> canonical -> final rows
+            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+                const int chi = 4 * t + w, rho = lane;
+                uint4* o = reinterpret_cast<uint4*>(out + (r0 + rho) * 256 + 16 * chi);
+#pragma unroll
+                for (int v = 0; v < 4; ++v) {
+                    uint32_t y[4];
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) {
+                        const uint32_t yy = shoup_mul(combine(d + 4 * (4 * v + e), q, c16s), 1u, one_s, q);
+                        y[e] = umin32(yy, yy - q);
+                    }
+                    __stcs(o + v, make_uint4(y[0], y[1], y[2], y[3]));
+                }
+            });
+        } else if (!phase1) {
+            // stage 3' (F') -> sigma3 -> A_mid (I-S2 layout)
+            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+                const int rho = (lane & 7) + 8 * w, chi = 4 * t + (lane >> 3);
+                const uint2* s3 = T3 + ((size_t)(r0 + rho) * 16 + chi) * 16;
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const uint2 sg = __ldg(s3 + k);
+                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), sg.x, sg.y, q);
+                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + rho, chi)) = z;
+                }
+            });
+            fence_async_smem();
+            named_bar(TC_BAR_ID, TC_T);
+            // stage 2' (F') -> sigma2 -> staging rows -> coalesced intermediate
+            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+                const int clo = 4 * t + w, rho = lane;
+                const uint2* s2 = T2 + (size_t)(r0 + rho) * 16;
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const uint2 sg = __ldg(s2 + k);
+                    sh.stg[rho * 257 + clo + 16 * k] = shoup_mul(combine(d + 4 * k, q, c16s), sg.x, sg.y, q);
+                }
+            });
+            named_bar(TC_BAR_ID, TC_T);
+#pragma unroll 4
+            for (int e = tid; e < 8192; e += TC_T) {
+                const int rho = e >> 8, col = e & 255;
+                out[(r0 + rho) * 256 + col] = sh.stg[rho * 257 + col];
+            }
+        } else {
+            // stage 1' (F') -> sigma1 -> A_mid (I-S0 layout)
+            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+                const int c = (lane & 7) + 8 * w, i1 = 4 * t + (lane >> 3);
+                const uint2* s1 = T1 + i1 * 16;
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    const uint2 sg = __ldg(s1 + k);
+                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), sg.x, sg.y, q);
+                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + c, i1)) = z;
+                }
+            });
+            fence_async_smem();
+            named_bar(TC_BAR_ID, TC_T);
+            // stage 0' (folded MI0 incl. N^-1) -> canonical -> final columns
+            tc_stage(sh, tmem, sh.Amid, sh.B, ph, [&](int t, const uint32_t* d) {
+                const int i0 = 4 * t + w, c = lane;
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    uint32_t y = shoup_mul(combine(d + 4 * k, q, c16s), 1u, one_s, q);
+                    y = umin32(y, y - q);
+                    __stcs(out + (i0 + 16 * k) * 256 + c0 + c, y);
+                }
+            });
+        }
+        // chunk boundary: global intermediate visible to this group's later loads; buffers free
+        __threadfence_block();
+        named_bar(TC_BAR_ID, TC_T);
+    }
+}
+
+// Standalone tensor-core kernel: persistent CTAs of 128 threads (TENSOR mode).
+template <bool FWD>
+__global__ void __launch_bounds__(TC_T, 1) ntt_tc16(TcArgs ta, uint32_t rows) {
+    extern __shared__ __align__(1024) uint8_t tsm[];
+    TcShared sh;
+    sh.Ain = tsm;
+    sh.Amid = tsm + 4 * TC_TILE;
+    sh.B = tsm + 8 * TC_TILE;
+    sh.stg = reinterpret_cast<uint32_t*>(tsm + 8 * TC_TILE + 8192);
+    sh.bar = reinterpret_cast<uint64_t*>(tsm + 8 * TC_TILE + 8192 + 32 * 257 * 4);
+    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        mbar_init(&sh.bar[0], 1);
+        mbar_init(&sh.bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (tid < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(sh.tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *sh.tslot;
+    uint32_t ph[2] = {0, 0};
+    for (uint32_t row = blockIdx.x; row < rows; row += gridDim.x) tc_transform<FWD>(ta, sh, tmem, ph, row);
+    tc_fence_before();
+    __syncthreads();
+    if (tid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
+}
+
+// ------------------------------------------------------------------ host side
+inline void free_tensor_tables(TensorTables& t) {
+    cudaFree(t.d_B); cudaFree(t.d_tw1); cudaFree(t.d_tw2); cudaFree(t.d_tw3);
+    cudaFree(t.d_sg1); cudaFree(t.d_sg2); cudaFree(t.d_sg3); cudaFree(t.d_c16);
+    t = TensorTables();
+}
+
+// Builds and verifies the factorised block tables for every limb (logN == 16 only).
+inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vector<uint32_t>& primes,
+                               const std::vector<uint32_t>& psis) {
+    if (logN != 16) return 0;
+    const uint32_t N = 1u << 16, L = (uint32_t)primes.size();
+    std::vector<uint8_t> B((size_t)L * 4 * 4096);
+    std::vector<uint2> t1((size_t)L * 256), t2((size_t)L * 4096), t3((size_t)L * 65536);
+    std::vector<uint2> s1((size_t)L * 256), s2((size_t)L * 4096), s3((size_t)L * 65536);
+    std::vector<uint2> c16(L);
+    for (uint32_t l = 0; l < L; ++l) {
+        const uint32_t q = primes[l], psi = psis[l], psi_inv = pm_pow(psi, q - 2, q);
+        std::vector<uint32_t> pw(N), pwi(N), fb(N), ib(N);
+        pw[0] = pwi[0] = 1;
+        for (uint32_t i = 1; i < N; ++i) { pw[i] = pm_mul(pw[i - 1], psi, q); pwi[i] = pm_mul(pwi[i - 1], psi_inv, q); }
+        for (uint32_t i = 0; i < N; ++i) { fb[i] = pw[pm_brv(i, 16)]; ib[i] = pwi[pm_brv(i, 16)]; }
+        const uint32_t ninv = pm_pow(N % q, q - 2, q);
+        uint32_t M[16][16], F[16][16], Fi[16][16];
+        block_fwd(M, fb, 0, 0, q);
+        byte_planes(&B[((size_t)l * 4 + 0) * 4096], M, q);
+        block_inv(M, ib, 0, 0, q, ninv);
+        byte_planes(&B[((size_t)l * 4 + 2) * 4096], M, q);
+        // fixed DFTs from one group, then every group of stages 1..3 must factor through them
+        bool have_f = false;
+        struct S { int ls; uint32_t groups; uint2* tw; uint2* sg; };
+        S st[3] = {{4, 16, &t1[(size_t)l * 256], &s1[(size_t)l * 256]},
+                   {8, 256, &t2[(size_t)l * 4096], &s2[(size_t)l * 4096]},
+                   {12, 4096, &t3[(size_t)l * 65536], &s3[(size_t)l * 65536]}};
+        for (auto& s : st) {
+            for (uint32_t g = 0; g < s.groups; ++g) {
+                uint32_t Mf[16][16], Mi[16][16];
+                block_fwd(Mf, fb, s.ls, g, q);
+                block_inv(Mi, ib, s.ls, g, q, 0);
+                for (int j = 0; j < 16; ++j) {
+                    const uint32_t tau = Mf[0][j], taui = pm_pow(tau, q - 2, q);
+                    const uint32_t sig = Mi[j][0], sigi = pm_pow(sig, q - 2, q);
+                    s.tw[g * 16 + j] = make_uint2(tau, pm_shoup(tau, q));
+                    s.sg[g * 16 + j] = make_uint2(sig, pm_shoup(sig, q));
+                    for (int k = 0; k < 16; ++k) {
+                        const uint32_t f = pm_mul(Mf[k][j], taui, q);       // F[k][j]
+                        const uint32_t fi = pm_mul(Mi[j][k], sigi, q);      // F'[j][k]
+                        if (!have_f) { F[k][j] = f; Fi[j][k] = fi; }
+                        else if (F[k][j] != f || Fi[j][k] != fi) return 4;  // factorisation failed
+                    }
+                }
+                have_f = true;
+            }
+        }
+        byte_planes(&B[((size_t)l * 4 + 1) * 4096], F, q);
+        byte_planes(&B[((size_t)l * 4 + 3) * 4096], Fi, q);
+        c16[l] = make_uint2(pm_shoup(65536u % q, q), pm_shoup(1u, q));
+    }
+    auto up = [](void** d, const void* h, size_t n) {
+        if (cudaMalloc(d, n) != cudaSuccess) return false;
+        return cudaMemcpy(*d, h, n, cudaMemcpyHostToDevice) == cudaSuccess;
+    };
+    if (!up((void**)&tc.d_B, B.data(), B.size()) || !up((void**)&tc.d_tw1, t1.data(), t1.size() * 8) ||
+        !up((void**)&tc.d_tw2, t2.data(), t2.size() * 8) || !up((void**)&tc.d_tw3, t3.data(), t3.size() * 8) ||
+        !up((void**)&tc.d_sg1, s1.data(), s1.size() * 8) || !up((void**)&tc.d_sg2, s2.data(), s2.size() * 8) ||
+        !up((void**)&tc.d_sg3, s3.data(), s3.size() * 8) || !up((void**)&tc.d_c16, c16.data(), c16.size() * 8))
+        return 4;
+    tc.ok = true;
+    return 0;
+}
+
+inline int prepare_tensor_kernels(uint32_t logN) {
+    if (logN != 16) return 0;
+    if (cudaFuncSetAttribute(ntt_tc16<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess ||
+        cudaFuncSetAttribute(ntt_tc16<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess)
+        return 4;
+    return 0;
+}
+
+// TENSOR mode launch (FUSED lives in ntt_fused.cuh)
+inline int launch_tensor(uint32_t logN, bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows,
+                         int sm_count, cudaStream_t s) {
+    if (logN != 16 || !tc.ok) return -1;
+    TcArgs ta;
+    ta.a = a;
+    ta.B = tc.d_B;
+    ta.t1 = fwd ? tc.d_tw1 : tc.d_sg1;
+    ta.t2 = fwd ? tc.d_tw2 : tc.d_sg2;
+    ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
+    ta.c16 = tc.d_c16;
+    int occ = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_tc16<true>, TC_T, TC_SMEM);
+    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * (occ > 0 ? occ : 1)));
+    if (fwd) ntt_tc16<true><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
+    else ntt_tc16<false><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
+    return 1;
+}
 
 }  // namespace wd

@@ -8,6 +8,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -16,7 +17,10 @@
 #include "wd_ntt.h"
 #include "modarith.cuh"
 #include "ntt_cuda_core.cuh"
+#include "ntt_persist.cuh"
+#include "ntt_smem.cuh"
 #include "ntt_tensor.cuh"
+#include "ntt_fused.cuh"
 #include "plan_math.h"
 
 using namespace wd;
@@ -30,6 +34,8 @@ int set_err(int e) { g_last_error = e; return e; }
 struct wd_ntt_plan {
     uint32_t N = 0, logN = 0, L = 0;
     int device = -1;
+    int sm_count = 148;
+    int kernel_ver = 2;            // WD_NTT_KERNEL=v1|v2|v3 selects the CUDA-core kernel generation (A/B runs)
     std::vector<uint32_t> primes, psi;
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
     uint2* d_inv = nullptr;        // [L][N]  (psi^-brv(i), Shoup)
@@ -67,6 +73,18 @@ int prep_cc() {
     if (set_smem(ntt_fwd_cc<LOGN>, S::SMEM_BYTES) || set_smem(ntt_inv_cc<LOGN, false>, S::SMEM_BYTES) ||
         set_smem(ntt_inv_cc<LOGN, true>, S::SMEM_BYTES))
         return WD_ECUDA;
+    if constexpr (LOGN == 15 || LOGN == 16) {
+        if (set_smem(ntt_fwd_smem<LOGN>, SM_BYTES) || set_smem(ntt_inv_smem<LOGN, false>, SM_BYTES) ||
+            set_smem(ntt_inv_smem<LOGN, true>, SM_BYTES))
+            return WD_ECUDA;
+    }
+    if constexpr (LOGN >= 15) {
+        using G = PGeo<LOGN>;
+        if (set_smem(ntt_persist_cc<LOGN, true, false>, G::SMEM_BYTES) ||
+            set_smem(ntt_persist_cc<LOGN, false, false>, G::SMEM_BYTES) ||
+            set_smem(ntt_persist_cc<LOGN, false, true>, G::SMEM_BYTES))
+            return WD_ECUDA;
+    }
     return WD_OK;
 }
 
@@ -87,8 +105,37 @@ int prepare_kernels(uint32_t logN) {
 }
 
 template <int LOGN>
-void launch_cc(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     using S = CcShape<LOGN>;
+    if constexpr (LOGN == 15 || LOGN == 16) {
+        if (p->kernel_ver == 3) {
+            constexpr int PAIR = LOGN == 16 ? 2 : 1;
+            const uint32_t units = std::min<uint32_t>(rows, (uint32_t)(p->sm_count / PAIR));
+            const uint32_t grid = units * PAIR;
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(grid); cfg.blockDim = dim3(SM_T); cfg.dynamicSmemBytes = SM_BYTES; cfg.stream = s;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = PAIR; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+            cfg.attrs = at; cfg.numAttrs = 1;
+            if (fwd) cudaLaunchKernelEx(&cfg, ntt_fwd_smem<LOGN>, a, rows);
+            else if (a.in2) cudaLaunchKernelEx(&cfg, ntt_inv_smem<LOGN, true>, a, rows);
+            else cudaLaunchKernelEx(&cfg, ntt_inv_smem<LOGN, false>, a, rows);
+            return;
+        }
+    }
+    if constexpr (LOGN >= 15) {
+        if (p->kernel_ver == 2) {
+            using G = PGeo<LOGN>;
+            int occ = 1;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_persist_cc<LOGN, true, false>, G::T, G::SMEM_BYTES);
+            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * std::max(occ, 1)));
+            if (fwd) ntt_persist_cc<LOGN, true, false><<<grid, G::T, G::SMEM_BYTES, s>>>(a, rows);
+            else if (a.in2) ntt_persist_cc<LOGN, false, true><<<grid, G::T, G::SMEM_BYTES, s>>>(a, rows);
+            else ntt_persist_cc<LOGN, false, false><<<grid, G::T, G::SMEM_BYTES, s>>>(a, rows);
+            return;
+        }
+    }
     if (fwd) ntt_fwd_cc<LOGN><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
     else if (a.in2) ntt_inv_cc<LOGN, true><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
     else ntt_inv_cc<LOGN, false><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
@@ -96,12 +143,12 @@ void launch_cc(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
 
 int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     switch (p->logN) {
-        case 12: launch_cc<12>(fwd, a, rows, s); break;
-        case 13: launch_cc<13>(fwd, a, rows, s); break;
-        case 14: launch_cc<14>(fwd, a, rows, s); break;
-        case 15: launch_cc<15>(fwd, a, rows, s); break;
-        case 16: launch_cc<16>(fwd, a, rows, s); break;
-        case 17: launch_cc<17>(fwd, a, rows, s); break;
+        case 12: launch_cc<12>(p, fwd, a, rows, s); break;
+        case 13: launch_cc<13>(p, fwd, a, rows, s); break;
+        case 14: launch_cc<14>(p, fwd, a, rows, s); break;
+        case 15: launch_cc<15>(p, fwd, a, rows, s); break;
+        case 16: launch_cc<16>(p, fwd, a, rows, s); break;
+        case 17: launch_cc<17>(p, fwd, a, rows, s); break;
         default: {
             const int thr = std::min<int>(256, std::max<int>(32, (int)p->N / 2));
             if (fwd) ntt_small<true, false><<<rows, thr, 4 << p->logN, s>>>(a, (int)p->logN);
@@ -136,8 +183,8 @@ int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2,
         if (mode != WD_MODE_CUDA && in2 == nullptr && mode != WD_MODE_AUTO) return set_err(WD_EUNSUPPORTED);
         launches = launch_cuda_core(p, fwd, a, rows, s);
     } else {
-        float share = mode == WD_MODE_TENSOR ? 1.0f : p->tensor_share;
-        launches = launch_tensor(p->logN, fwd, a, p->tc, rows, share, s);
+        if (mode == WD_MODE_TENSOR) launches = launch_tensor(p->logN, fwd, a, p->tc, rows, p->sm_count, s);
+        else launches = launch_fused(p->logN, fwd, a, p->tc, rows, p->sm_count, p->tensor_share, s);
         if (launches < 0) return set_err(WD_EUNSUPPORTED);
     }
     if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
@@ -238,6 +285,8 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
 
     // ---- device upload (the only H2D copy of the plan's life)
     if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
+    cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
+    if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : 2;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
         cudaMalloc(&p->d_lc, sizeof(LimbConst) * L) != cudaSuccess) {
@@ -253,7 +302,8 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     }
     for (auto& s : p->hs) if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->he) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
-    if (prepare_kernels(p->logN) != WD_OK || prepare_tensor_kernels(p->logN) != WD_OK) {
+    if (prepare_kernels(p->logN) != WD_OK || prepare_tensor_kernels(p->logN) != WD_OK ||
+        prepare_fused_kernels(p->logN) != WD_OK) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
     p->mode = WD_MODE_AUTO;

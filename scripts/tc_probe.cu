@@ -33,6 +33,14 @@ DEVI void mma_i8(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint
         "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}\n"
         :: "r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(acc));
 }
+DEVI void mma_i8_mask(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc,
+                      uint32_t m0, uint32_t m1, uint32_t m2, uint32_t m3) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, {%5, %6, %7, %8}, p;\n\t}\n"
+        :: "r"(tmem_d), "l"(da), "l"(db), "r"(idesc), "r"(acc), "r"(m0), "r"(m1), "r"(m2), "r"(m3));
+}
 DEVI void mma_commit(uint64_t* bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
                  :: "r"(smem_u32(bar)) : "memory");
@@ -101,6 +109,50 @@ extern "C" __global__ void k_probe_mma(const uint8_t* A, const uint8_t* B, int32
         const uint32_t id = idesc_i8(128, 64);
         mma_i8(tmem, make_desc(a0, LBO, SBO), make_desc(b0, LBO, SBO), id, 0);
         mma_i8(tmem, make_desc(a0 + 2 * LBO, LBO, SBO), make_desc(b0 + 2 * LBO, LBO, SBO), id, 1);
+        mma_commit(&bar);
+    }
+    mbar_wait(&bar, 0);
+    fence_after();
+    uint32_t r[32];
+    const int warp = t >> 5;
+    for (int half = 0; half < 2; ++half) {
+        tmem_ld32(tmem + ((warp * 32) << 16) + half * 32, r);
+        tmem_wait_ld();
+        for (int c = 0; c < 32; ++c) D[t * 64 + half * 32 + c] = (int32_t)r[c];
+    }
+    fence_before();
+    __syncthreads();
+    if (t < 32) tmem_free<64>(tmem);
+}
+
+// masked: 4 B matrices (64x64 each, [g][n][k]); MMA g writes only lanes 32g..32g+31 (mask bit 1 = disabled?)
+extern "C" __global__ void k_probe_mask(const uint8_t* A, const uint8_t* B4, int32_t* D) {
+    __shared__ __align__(1024) uint8_t sA[128 * 64];
+    __shared__ __align__(1024) uint8_t sB[4][64 * 64];
+    __shared__ __align__(8) uint64_t bar;
+    __shared__ uint32_t taddr_s;
+    const int t = threadIdx.x;
+    for (int i = t; i < 128 * 64; i += blockDim.x) sA[aoff(i / 64, i % 64)] = A[i];
+    for (int g = 0; g < 4; ++g)
+        for (int i = t; i < 64 * 64; i += blockDim.x) sB[g][aoff(i / 64, i % 64)] = B4[g * 4096 + i];
+    if (t == 0) { mbar_init(&bar, 1); asm volatile("fence.mbarrier_init.release.cluster;"); }
+    if (t < 32) tmem_alloc<64>(&taddr_s);
+    fence_proxy_async();
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tmem = taddr_s;
+    if (t == 0) {
+        const uint32_t a0 = smem_u32(sA);
+        const uint32_t id = idesc_i8(128, 64);
+        for (int g = 0; g < 4; ++g) {
+            const uint32_t b0 = smem_u32(sB[g]);
+            uint32_t m[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
+            m[g] = 0;
+            mma_i8_mask(tmem, make_desc(a0, LBO, SBO), make_desc(b0, LBO, SBO), id, 0, m[0], m[1], m[2], m[3]);
+            mma_i8_mask(tmem, make_desc(a0 + 2 * LBO, LBO, SBO), make_desc(b0 + 2 * LBO, LBO, SBO), id, 1,
+                        m[0], m[1], m[2], m[3]);
+        }
         mma_commit(&bar);
     }
     mbar_wait(&bar, 0);
@@ -204,6 +256,18 @@ extern "C" int probe_mma(const uint8_t* hA, const uint8_t* hB, int32_t* hD) {
     cudaMemcpy(dA, hA, 128 * 64, cudaMemcpyHostToDevice);
     cudaMemcpy(dB, hB, 64 * 64, cudaMemcpyHostToDevice);
     k_probe_mma<<<1, 128>>>(dA, dB, dD);
+    int e = (int)cudaDeviceSynchronize();
+    cudaMemcpy(hD, dD, 128 * 64 * 4, cudaMemcpyDeviceToHost);
+    cudaFree(dA); cudaFree(dB); cudaFree(dD);
+    return e;
+}
+
+extern "C" int probe_mask(const uint8_t* hA, const uint8_t* hB4, int32_t* hD) {
+    uint8_t *dA, *dB; int32_t* dD;
+    cudaMalloc(&dA, 128 * 64); cudaMalloc(&dB, 4 * 64 * 64); cudaMalloc(&dD, 128 * 64 * 4);
+    cudaMemcpy(dA, hA, 128 * 64, cudaMemcpyHostToDevice);
+    cudaMemcpy(dB, hB4, 4 * 64 * 64, cudaMemcpyHostToDevice);
+    k_probe_mask<<<1, 128>>>(dA, dB, dD);
     int e = (int)cudaDeviceSynchronize();
     cudaMemcpy(hD, dD, 128 * 64 * 4, cudaMemcpyDeviceToHost);
     cudaFree(dA); cudaFree(dB); cudaFree(dD);

@@ -36,6 +36,18 @@ if not ok:
     res["eq_T"] = bool(np.array_equal(D.astype(np.int64), (A.astype(np.int64) @ B.astype(np.int64))))
 print(json.dumps(res), flush=True)
 
+B4 = rng.integers(0, 256, size=(4, 64, 64), dtype=np.uint8)
+D4 = np.zeros((128, 64), dtype=np.int32)
+e = lib.probe_mask(A.ctypes.data, B4.ctypes.data, D4.ctypes.data)
+res = {"probe": "mma_mask", "err": e}
+for g in range(4):
+    refg = A[32 * g:32 * g + 32].astype(np.int64) @ B4[g].astype(np.int64).T
+    res["group%d_exact" % g] = bool(np.array_equal(D4[32 * g:32 * g + 32], refg))
+    res["group%d_matches_B3" % g] = bool(np.array_equal(D4[32 * g:32 * g + 32], A[32*g:32*g+32].astype(np.int64) @ B4[3].astype(np.int64).T))
+print(json.dumps(res), flush=True)
+import sys
+if "--mask-only" in sys.argv:
+    sys.exit(0)
 SM = 148
 for blocks_per_sm in (1, 2, 4):
     blocks = SM * blocks_per_sm

@@ -194,3 +194,52 @@ def test_config5_sweep_batch1(wd, logn, L):
     plan = wd.Plan(n, primes)
     y = gpu_fwd(wd, plan, x)
     assert np.array_equal(y, oracle.ntt_forward(x, primes))
+
+
+# -------------------------------------------------------------- execution modes (rows a4 / a5 / a9)
+def _modes(wd):
+    return ["cuda", "tensor", "fused"]
+
+
+@pytest.mark.parametrize("mode", ["cuda", "tensor", "fused"])
+def test_modes_vs_oracle_n65536(wd, mode):
+    n = 1 << 16
+    primes = [P[0], P[13], P[59]]
+    x = inputs.uniform_residues(primes, n, 3, 77)
+    plan = wd.Plan(n, primes)
+    try:
+        plan.set_mode(mode)
+    except wd.WdNttError as e:
+        pytest.fail("mode %s unavailable: %s" % (mode, e))
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), mode
+    assert np.array_equal(gpu_inv(wd, plan, y), x), mode
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), mode
+    q = inputs.structured("qm1", primes, n)
+    assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes)), mode
+    assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes)), mode
+
+
+@pytest.mark.parametrize("mode", ["tensor", "fused"])
+def test_modes_headline_config(wd, mode):
+    n, L, batch = 1 << 16, 36, 128
+    primes = P[:L]
+    x = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 2, device="cuda")
+    plan = wd.Plan(n, primes)
+    ref_plan = wd.Plan(n, primes, mode="cuda")
+    plan.set_mode(mode)
+    y = torch.empty_like(x)
+    yr = torch.empty_like(x)
+    plan.forward(x, y)
+    ref_plan.forward(x, yr)
+    torch.cuda.synchronize()
+    assert torch.equal(y, yr)                  # bit-identical across paths, every row
+    rows = [0, 1, 35, 36 * 64 + 7, batch * L - 1]
+    yh = to_host(y.view(batch * L, n)[torch.as_tensor(rows, device="cuda")])
+    xh = to_host(x.view(batch * L, n)[torch.as_tensor(rows, device="cuda")])
+    for k, r in enumerate(rows):
+        assert np.array_equal(yh[k], oracle.ntt_forward_row(xh[k], primes[r % L]))
+    z = torch.empty_like(x)
+    plan.inverse(y, z)
+    torch.cuda.synchronize()
+    assert torch.equal(z, x)
