@@ -321,6 +321,9 @@ def main():
                      "peak_kind": "%s (MEASURED_PEAKS.json hbm_gbs copy bandwidth)" % pk_kind,
                      "algorithmic_bytes_per_launch": alg_bytes},
         "gpu_launches": launches,
+        "occupancy_ctas_per_sm": {"cuda": wdntt.wd_ntt_occupancy(plan.handle, "cuda"),
+                                  "tensor_fwd": wdntt.wd_ntt_occupancy(plan.handle, "tensor", True),
+                                  "tensor_inv": wdntt.wd_ntt_occupancy(plan.handle, "tensor", False)},
         "clocks": clk.summary(),
         "e2e": e2e,
     }

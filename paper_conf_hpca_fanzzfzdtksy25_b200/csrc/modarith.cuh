@@ -79,15 +79,23 @@ __device__ __forceinline__ uint32_t canon2(uint32_t v, uint32_t q) {            
 template <int K>
 __device__ __forceinline__ void fwd_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
                                           uint32_t hi, uint32_t q, uint32_t q2) {
+    {   // layer ls: one twiddle
+        const uint2 w = __ldg(tw + (1u << ls) + hi);
 #pragma unroll
-    for (int t = 0; t < K; ++t) {
+        for (int r = 0; r < (1 << (K - 1)); ++r) ct_bfly(x[r], x[r + (1 << (K - 1))], w, q, q2);
+    }
+#pragma unroll
+    for (int t = 1; t < K; ++t) {            // layers ls+1..: twiddle pairs are adjacent -> 16-byte loads
         const int h = 1 << (K - 1 - t);
-        const uint2* tp = tw + (1u << (ls + t)) + (hi << t);
+        const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
 #pragma unroll
-        for (int g = 0; g < (1 << t); ++g) {
-            const uint2 w = __ldg(tp + g);
+        for (int g = 0; g < (1 << t); g += 2) {
+            const uint4 v = __ldg(tp + g / 2);
+            const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
 #pragma unroll
-            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w, q, q2);
+            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], wa, q, q2);
+#pragma unroll
+            for (int r = 0; r < h; ++r) ct_bfly(x[2 * (g + 1) * h + r], x[2 * (g + 1) * h + r + h], wb, q, q2);
         }
     }
 }
@@ -98,20 +106,26 @@ template <int K, bool LAST>
 __device__ __forceinline__ void inv_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
                                           uint32_t hi, const LimbConst& c) {
 #pragma unroll
-    for (int t = K - 1; t >= 0; --t) {
+    for (int t = K - 1; t >= 1; --t) {
         const int h = 1 << (K - 1 - t);
-        const uint2* tp = tw + (1u << (ls + t)) + (hi << t);
+        const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
 #pragma unroll
-        for (int g = 0; g < (1 << t); ++g) {
-            if (LAST && t == 0) {
+        for (int g = 0; g < (1 << t); g += 2) {
+            const uint4 v = __ldg(tp + g / 2);
+            const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
 #pragma unroll
-                for (int r = 0; r < h; ++r) gs_bfly_last(x[r], x[r + h], c);
-            } else {
-                const uint2 w = __ldg(tp + g);
+            for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], wa, c.q, c.q2);
 #pragma unroll
-                for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w, c.q, c.q2);
-            }
+            for (int r = 0; r < h; ++r) gs_bfly(x[2 * (g + 1) * h + r], x[2 * (g + 1) * h + r + h], wb, c.q, c.q2);
         }
+    }
+    if (LAST) {
+#pragma unroll
+        for (int r = 0; r < (1 << (K - 1)); ++r) gs_bfly_last(x[r], x[r + (1 << (K - 1))], c);
+    } else {
+        const uint2 w = __ldg(tw + (1u << ls) + hi);
+#pragma unroll
+        for (int r = 0; r < (1 << (K - 1)); ++r) gs_bfly(x[r], x[r + (1 << (K - 1))], w, c.q, c.q2);
     }
 }
 

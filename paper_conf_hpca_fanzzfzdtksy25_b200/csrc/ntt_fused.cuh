@@ -87,8 +87,7 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16(TcArgs ta, uint32_t rows,
     sh.Ain = tcb;
     sh.Amid = tcb + 4 * TC_TILE;
     sh.B = tcb + 8 * TC_TILE;
-    sh.stg = reinterpret_cast<uint32_t*>(tcb + 8 * TC_TILE + 8192);
-    sh.bar = reinterpret_cast<uint64_t*>(tcb + 8 * TC_TILE + 8192 + 32 * 257 * 4);
+    sh.bar = reinterpret_cast<uint64_t*>(tcb + 8 * TC_TILE + 8192);
     sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
     const int tid = threadIdx.x;
     if (tid == 0) {
@@ -148,11 +147,113 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16(TcArgs ta, uint32_t rows,
     }
 }
 
+// ---- phase-split pipeline: the tensor warps run the COLUMN phase (phase 1) of each row, the
+// CUDA-core warps run the ROW phase (phase 2); the two groups walk the CTA's row list in
+// step, handing each row over through its L2-resident output slot and a shared-memory
+// counter.  Forward: tensor leads (P1 of row i+1 overlaps P2 of row i).  Inverse: the
+// CUDA-core group leads (P2' first), the tensor group finishes each row with P1'.
+// The leader stays at most FU_LEAD rows ahead, bounding the in-flight intermediates.
+constexpr int FU_LEAD = 2;
+
+__device__ __forceinline__ int ld_volatile(const int* p) { return *reinterpret_cast<const volatile int*>(p); }
+
+// CUDA-core group: only phase 2 (forward) / phase 2' (inverse) of one row
+template <bool FWD, int BAR>
+__device__ __forceinline__ void cc_row_phase2(const NttArgs& a, uint32_t* smem, uint32_t row_id) {
+    using G = PGeo<16>;
+    const uint32_t* in = a.in + ((size_t)row_id << 16);
+    uint32_t* out = a.out + ((size_t)row_id << 16);
+    const uint32_t limb = row_id % a.L;
+    const LimbConst lc = a.lc[limb];
+    const uint2* __restrict__ tw = a.tw + ((size_t)limb << 16);
+    const uint32_t* src = FWD ? out : in;
+    load_p2<16>(smem, src, 0);
+    cp_async_commit();
+#pragma unroll 1
+    for (int kk = 0; kk < G::C2; ++kk) {
+        uint32_t* S = smem + (kk & 1) * G::BUF_WORDS;
+        if (kk + 1 < G::C2) {
+            load_p2<16>(smem + ((kk + 1) & 1) * G::BUF_WORDS, src, (kk + 1) * G::W2);
+            cp_async_commit();
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
+        gbar<BAR, FU_CC>();
+        if (FWD) fwd_p2_chunk<16, BAR>(S, out, kk * G::W2, tw, lc.q, lc.q2);
+        else inv_p2_chunk<16, false, BAR>(S, out, nullptr, kk * G::W2, tw, lc);
+        gbar<BAR, FU_CC>();
+    }
+}
+
+template <bool FWD>
+__global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, uint32_t rows) {
+    extern __shared__ __align__(1024) uint8_t fsm[];
+    uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
+    uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
+    int* ctl = reinterpret_cast<int*>(tcb + TC_SMEM);           // [0] rows done by the leader, [1] by the follower
+    TcShared sh;
+    sh.Ain = tcb;
+    sh.Amid = tcb + 4 * TC_TILE;
+    sh.B = tcb + 8 * TC_TILE;
+    sh.bar = reinterpret_cast<uint64_t*>(tcb + 8 * TC_TILE + 8192);
+    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        ctl[0] = 0; ctl[1] = 0;
+        mbar_init(&sh.bar[0], 1);
+        mbar_init(&sh.bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (tid >= FU_CC && tid < FU_CC + 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(sh.tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const int nmine = rows > blockIdx.x ? (int)((rows - blockIdx.x + gridDim.x - 1) / gridDim.x) : 0;
+    const bool is_tc = tid >= FU_CC;
+    const bool leader = FWD ? is_tc : !is_tc;                    // who runs the first phase of a row
+    const int gtid = is_tc ? tid - FU_CC : tid;
+    const int nthr = is_tc ? FU_TC : FU_CC;
+    const int bar = is_tc ? TC_BAR_ID : FU_CC_BAR;
+    int* mine = &ctl[leader ? 0 : 1];
+    const int* other = &ctl[leader ? 1 : 0];
+    const uint32_t tmem = *sh.tslot;
+    uint32_t ph[2] = {0, 0};
+    for (int i = 0; i < nmine; ++i) {
+        // leader: stay <= FU_LEAD rows ahead; follower: wait until the leader finished row i
+        if (gtid == 0) {
+            if (leader) { while (i - ld_volatile(other) >= FU_LEAD) __nanosleep(256); }
+            else { while (ld_volatile(other) <= i) __nanosleep(128); }
+        }
+        named_bar(bar, nthr);
+        __threadfence_block();
+        const uint32_t row = blockIdx.x + (uint32_t)i * gridDim.x;
+        if (is_tc) tc_transform<FWD, 1, true>(ta, sh, tmem, ph, row);           // column phase, either direction
+        else cc_row_phase2<FWD, FU_CC_BAR>(ta.a, ccbuf, row);
+        __threadfence_block();
+        named_bar(bar, nthr);
+        if (gtid == 0) atomicExch(mine, i + 1);
+    }
+    if (is_tc) {
+        tc_fence_before();
+        named_bar(TC_BAR_ID, FU_TC);
+        if (gtid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
+    }
+}
+
 inline int prepare_fused_kernels(uint32_t logN) {
     if (logN != 16) return 0;
-    if (cudaFuncSetAttribute(ntt_fused16<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess ||
-        cudaFuncSetAttribute(ntt_fused16<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess)
-        return 4;
+    for (auto k : {ntt_fused16_pipe<true>, ntt_fused16_pipe<false>})
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess ||
+            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+            return 4;
+    for (auto k : {ntt_fused16<true, false>, ntt_fused16<false, false>})
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess ||
+            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+            return 4;
     return 0;
 }
 
@@ -167,6 +268,11 @@ inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorT
     ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
     ta.c16 = tc.d_c16;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
+    if (share > 1.5f) {            // tensor_share = 2: phase-split pipeline (tensor: columns, CUDA: rows)
+        if (fwd) ntt_fused16_pipe<true><<<grid, FU_T, FU_SMEM, s>>>(ta, rows);
+        else ntt_fused16_pipe<false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows);
+        return 1;
+    }
     if (fwd) ntt_fused16<true, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);
     else ntt_fused16<false, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);
     return 1;

@@ -67,8 +67,10 @@ template <int LOGN>
 __device__ __forceinline__ void load_p1(uint32_t* S, const uint32_t* src, int c0) {
     using G = PGeo<LOGN>;
     constexpr int SEG = G::W1 / 4, NSEG = G::N1 * SEG;
+    static_assert(NSEG % G::T == 0, "whole segments per thread");
 #pragma unroll
-    for (int i = threadIdx.x; i < NSEG; i += G::T) {
+    for (int k = 0; k < NSEG / G::T; ++k) {
+        const int i = threadIdx.x % G::T + k * G::T;
         const int p = i / SEG, s = i % SEG;
         cp_async16(S + p * G::W1 + 4 * s, src + p * 256 + c0 + 4 * s);
     }
@@ -78,8 +80,10 @@ template <int LOGN>
 __device__ __forceinline__ void load_p2(uint32_t* S, const uint32_t* src, int r0) {
     using G = PGeo<LOGN>;
     constexpr int NSEG = G::W2 * 64;
+    static_assert(NSEG % G::T == 0, "whole segments per thread");
 #pragma unroll
-    for (int i = threadIdx.x; i < NSEG; i += G::T) {
+    for (int k = 0; k < NSEG / G::T; ++k) {
+        const int i = threadIdx.x % G::T + k * G::T;
         const int w = i >> 6, v4 = i & 63, chi = v4 >> 2, v = v4 & 3;
         cp_async16(S + w * RS + chi * 16 + (((v ^ (chi >> 1)) & 3) << 2), src + (r0 + w) * 256 + 4 * v4);
     }

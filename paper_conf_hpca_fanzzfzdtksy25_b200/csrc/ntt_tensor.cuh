@@ -118,17 +118,18 @@ __device__ __forceinline__ uint32_t combine(const uint32_t* d, uint32_t q, uint3
 // ------------------------------------------------------------------ the kernel
 constexpr int TC_T = 128;                 // threads (4 warps; warp w owns TMEM lanes 32w..32w+31)
 constexpr int TC_TILE = 128 * 64;         // bytes per operand tile
-constexpr int TC_SMEM = 2 * 4 * TC_TILE   // A_in, A_mid (4 tiles each)
-                        + 2 * 4096        // B images of the two stages of this phase
-                        + 32 * 257 * 4    // inverse stage-2' staging (row stride 257 words)
+constexpr int TC_SMEM = 2 * 4 * TC_TILE   // A_in (also the inverse stage-2' staging), A_mid
+                        + 2 * 4096        // B images of the current limb (folded stage, fixed DFT16)
                         + 64;             // mbarriers + TMEM address
 constexpr int TC_BAR_ID = 1;              // named barrier used by the tensor group
+constexpr int TC_CTAS_PER_SM = 3;         // 3 x 73 KB smem, 3 x 128 TMEM columns, 3 x 128 threads per SM
 
 struct TcShared {
-    uint8_t* Ain; uint8_t* Amid; uint8_t* B; uint32_t* stg; uint64_t* bar; uint32_t* tslot;
+    uint8_t* Ain; uint8_t* Amid; uint8_t* B; uint64_t* bar; uint32_t* tslot;
 };
 
-// one radix-16 stage over the 4 tiles of Abuf with B image Bimg; epi(t, d[64]) consumes tile t
+// One radix-16 stage over the 4 tiles of Abuf with B image Bimg.  epi(t, half, d[32]) consumes
+// outputs k = 8*half .. 8*half+7 of tile t (TMEM columns 32*half .. 32*half+31).
 template <typename Epi>
 __device__ __forceinline__ void tc_stage(const TcShared& sh, uint32_t tmem, const uint8_t* Abuf, const uint8_t* Bimg,
                                          uint32_t* ph, Epi&& epi) {
@@ -148,26 +149,32 @@ __device__ __forceinline__ void tc_stage(const TcShared& sh, uint32_t tmem, cons
         mbar_wait(&sh.bar[r], ph[r]);
         ph[r] ^= 1;
         tc_fence_after();
-        uint32_t d[64];
         const uint32_t ta = tmem + ((uint32_t)(32 * w) << 16) + r * 64;
+        uint32_t d[32];
         tmem_ld32(ta, d);
-        tmem_ld32(ta + 32, d + 32);
+        tmem_wait_ld();
+        epi(t, 0, d);
+        tmem_ld32(ta + 32, d);
         tmem_wait_ld();
         tc_fence_before();
         named_bar(TC_BAR_ID, TC_T);
         if (tid == 0 && t + 2 < 4) issue(t + 2);
-        epi(t, d);
+        epi(t, 1, d);
     }
 }
 
-template <bool FWD>
+// PH = 0: the whole row; PH = 1: only the column phase (chunks of phase 1);
+// PH = 2: only the row phase.  (The fused kernel splits a row's phases between the units.)
+// PLAIN_MID (forward, PH = 1): store the plain merged-CT intermediate instead of pre-twisting
+// it by tau2 for the tensor stage 2, so the CUDA-core butterflies can take phase 2 over.
+template <bool FWD, int PH = 0, bool PLAIN_MID = false>
 __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& sh, uint32_t tmem, uint32_t* ph,
                                              uint32_t row_id) {
     const NttArgs& a = ta.a;
     const int tid = threadIdx.x % TC_T, w = tid >> 5, lane = tid & 31;
     const uint32_t limb = row_id % a.L;
     const LimbConst lc = a.lc[limb];
-    const uint32_t q = lc.q, q2 = lc.q2;
+    const uint32_t q = lc.q;
     const uint2 cc = ta.c16[limb];
     const uint32_t c16s = cc.x, one_s = cc.y;
     const uint32_t* in = a.in + ((size_t)row_id << 16);
@@ -176,45 +183,54 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
     const uint2* T1 = ta.t1 + (size_t)limb * 256;
     const uint2* T2 = ta.t2 + (size_t)limb * 4096;
     const uint2* T3 = ta.t3 + (size_t)limb * 65536;
+    uint32_t* stg = reinterpret_cast<uint32_t*>(sh.Ain);      // inverse stage-2' staging (32 x 256, XOR-swizzled)
 
     // B images: [0] = folded single-group matrix (M0 or MI0), [1] = fixed DFT16 (F or F')
-    for (int i = tid; i < 2 * 4096 / 16; i += TC_T)
-        cp_async16(sh.B + 16 * i, Bl + 16 * i);
+    for (int i = tid; i < 2 * 4096 / 16; i += TC_T) cp_async16(sh.B + 16 * i, Bl + 16 * i);
     cp_async_commit();
 
+#pragma unroll 1
     for (int ch = 0; ch < 16; ++ch) {
         const bool phase1 = FWD ? (ch < 8) : (ch >= 8);
-        const int k8 = ch & 7;
-        const int c0 = 32 * k8, r0 = 32 * k8;
-        // ---------------- load the chunk into the first stage's operand tiles
+        if ((PH == 1 && !phase1) || (PH == 2 && phase1)) continue;
+        const int c0 = 32 * (ch & 7), r0 = 32 * (ch & 7);
+        // ---------------- chunk -> operand tiles of the first stage.  Lane maps put 8 distinct
+        // (row & 7) x 4 distinct (coefficient & 3) in a warp: conflict-free 4-byte smem writes
+        // and 32-byte global sectors.
         if (FWD && phase1) {                       // F-S0: (c, i0), coeff r, p = i0 + 16 r
-#pragma unroll 4
-            for (int e = tid; e < 8192; e += TC_T) {
-                const int p = e >> 5, c = e & 31, i0 = p & 15, r = p >> 4;
-                const int t = i0 >> 2, m = (c & 7) + 8 * (i0 & 3) + 32 * (c >> 3);
-                cp_async4(sh.Ain + t * TC_TILE + aoff_w(m, r), in + p * 256 + c0 + c);
-            }
+            const int c = (lane & 7) + 8 * w, r3 = lane >> 3;
+            const uint32_t* src = in + (16 * r3) * 256 + c0 + c;
+            uint8_t* dst = sh.Ain + (lane & 7) * 16 + (4 * w) * 512 + r3 * 4;
+#pragma unroll
+            for (int i0 = 0; i0 < 16; ++i0)
+#pragma unroll
+                for (int rh = 0; rh < 4; ++rh)
+                    cp_async4(dst + (i0 >> 2) * TC_TILE + (i0 & 3) * 512 + rh * 128, src + (i0 + 64 * rh) * 256);
         } else if (FWD) {                          // F-S2: (rho, clo), coeff chi, col = clo + 16 chi
-#pragma unroll 4
-            for (int e = tid; e < 8192; e += TC_T) {
-                const int rho = e >> 8, col = e & 255, clo = col & 15, chi = col >> 4;
-                const int t = clo >> 2, m = (rho & 7) + 8 * (clo & 3) + 32 * (rho >> 3);
-                cp_async4(sh.Ain + t * TC_TILE + aoff_w(m, chi), out + (r0 + rho) * 256 + col);
-            }
+            const int rho = (lane >> 2) + 8 * w, cl3 = lane & 3;
+            const uint32_t* src = out + (r0 + rho) * 256 + cl3;
+            uint8_t* dst = sh.Ain + (rho & 7) * 16 + (cl3 + 4 * w) * 512;
+#pragma unroll
+            for (int ch2 = 0; ch2 < 4; ++ch2)
+#pragma unroll
+                for (int chi = 0; chi < 16; ++chi)
+                    cp_async4(dst + ch2 * TC_TILE + (chi >> 2) * 128 + (chi & 3) * 4, src + 4 * ch2 + 16 * chi);
         } else if (!phase1) {                      // I-S3: (rho, chi), coeff clo (16-byte runs)
-#pragma unroll 4
-            for (int s = tid; s < 2048; s += TC_T) {
-                const int rho = s >> 6, chi = (s >> 2) & 15, v = s & 3;
-                const int t = chi >> 2, m = (rho & 7) + 8 * (chi & 3) + 32 * (rho >> 3);
-                cp_async16(sh.Ain + t * TC_TILE + aoff_w(m, 4 * v), in + (r0 + rho) * 256 + 16 * chi + 4 * v);
-            }
+            const int rho = (lane & 7) + 8 * w, v = lane >> 3;
+            const uint32_t* src = in + (r0 + rho) * 256 + 4 * v;
+            uint8_t* dst = sh.Ain + (lane & 7) * 16 + (4 * w) * 512 + v * 128;
+#pragma unroll
+            for (int chi = 0; chi < 16; ++chi)
+                cp_async16(dst + (chi >> 2) * TC_TILE + (chi & 3) * 512, src + 16 * chi);
         } else {                                   // I-S1: (c, i1), coeff j, p = 16 i1 + j
-#pragma unroll 4
-            for (int e = tid; e < 8192; e += TC_T) {
-                const int p = e >> 5, c = e & 31, i1 = p >> 4, j = p & 15;
-                const int t = i1 >> 2, m = (c & 7) + 8 * (i1 & 3) + 32 * (c >> 3);
-                cp_async4(sh.Ain + t * TC_TILE + aoff_w(m, j), out + p * 256 + c0 + c);
-            }
+            const int c = (lane & 7) + 8 * w, j3 = lane >> 3;
+            const uint32_t* src = out + j3 * 256 + c0 + c;
+            uint8_t* dst = sh.Ain + (lane & 7) * 16 + (4 * w) * 512 + j3 * 4;
+#pragma unroll
+            for (int i1 = 0; i1 < 16; ++i1)
+#pragma unroll
+                for (int jh = 0; jh < 4; ++jh)
+                    cp_async4(dst + (i1 >> 2) * TC_TILE + (i1 & 3) * 512 + jh * 128, src + (16 * i1 + 4 * jh) * 256);
         }
         cp_async_commit();
         cp_async_wait<0>();
@@ -222,48 +238,58 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
         named_bar(TC_BAR_ID, TC_T);
 
         if (FWD && phase1) {
-            // stage 0 (folded M0) -> twist tau1 -> A_mid (F-S1 layout)
-            tc_stage(sh, tmem, sh.Ain, sh.B, ph, [&](int t, const uint32_t* d) {
+            // stage 0 (folded M0) -> twist tau1 -> A_mid (F-S1 layout: m = 32 (k&3) + c, coeff i0)
+            tc_stage(sh, tmem, sh.Ain, sh.B, ph, [&](int t, int hf, const uint32_t* d) {
                 const int c = (lane & 7) + 8 * w, i0 = 4 * t + (lane >> 3);
+                uint8_t* dst = sh.Amid + (c & 7) * 16 + (c >> 3) * 512 + (i0 >> 2) * 128 + (i0 & 3) * 4;
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
+                for (int kk = 0; kk < 8; ++kk) {
+                    const int k = 8 * hf + kk;
                     const uint2 tw = __ldg(T1 + k * 16 + i0);
-                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), tw.x, tw.y, q);
-                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + c, i0)) = z;
+                    const uint32_t z = shoup_mul(combine(d + 4 * kk, q, c16s), tw.x, tw.y, q);
+                    *reinterpret_cast<uint32_t*>(dst + (k >> 2) * TC_TILE + (k & 3) * 2048) = z;
                 }
             });
             fence_async_smem();
             named_bar(TC_BAR_ID, TC_T);
-            // stage 1 (F) -> twist tau2 -> intermediate (coalesced over c)
-            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+            // stage 1 (F) -> twist tau2 -> intermediate (lanes walk c: coalesced)
+            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, int hf, const uint32_t* d) {
                 const int i1 = 4 * t + w, c = lane;
+                const uint2* t2 = T2 + (16 * i1) * 16 + ((c0 + c) >> 4);
+                uint32_t* o = out + (16 * i1) * 256 + c0 + c;
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
-                    const int p = 16 * i1 + k;
-                    const uint2 tw = __ldg(T2 + p * 16 + ((c0 + c) >> 4));
-                    out[p * 256 + c0 + c] = shoup_mul(combine(d + 4 * k, q, c16s), tw.x, tw.y, q);
+                for (int kk = 0; kk < 8; ++kk) {
+                    const int k = 8 * hf + kk;
+                    if (PLAIN_MID) {
+                        o[k * 256] = shoup_mul(combine(d + 4 * kk, q, c16s), 1u, one_s, q);   // [0, 2q)
+                    } else {
+                        const uint2 tw = __ldg(t2 + 16 * k);
+                        o[k * 256] = shoup_mul(combine(d + 4 * kk, q, c16s), tw.x, tw.y, q);
+                    }
                 }
             });
         } else if (FWD) {
-            // stage 2 (F) -> twist tau3 -> A_mid (F-S3 layout)
-            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+            // stage 2 (F) -> twist tau3 -> A_mid (F-S3 layout: m = 32 (k&3) + rho, coeff clo)
+            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, int hf, const uint32_t* d) {
                 const int rho = (lane & 7) + 8 * w, clo = 4 * t + (lane >> 3);
                 const uint2* t3 = T3 + (size_t)(r0 + rho) * 256 + clo;        // group (row*16 + k), j = clo
+                uint8_t* dst = sh.Amid + (rho & 7) * 16 + (rho >> 3) * 512 + (clo >> 2) * 128 + (clo & 3) * 4;
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
+                for (int kk = 0; kk < 8; ++kk) {
+                    const int k = 8 * hf + kk;
                     const uint2 tw = __ldg(t3 + 16 * k);
-                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), tw.x, tw.y, q);
-                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + rho, clo)) = z;
+                    const uint32_t z = shoup_mul(combine(d + 4 * kk, q, c16s), tw.x, tw.y, q);
+                    *reinterpret_cast<uint32_t*>(dst + (k >> 2) * TC_TILE + (k & 3) * 2048) = z;
                 }
             });
             fence_async_smem();
             named_bar(TC_BAR_ID, TC_T);
-            // stage 3 (F) -> canonical -> final rows
-            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+            // stage 3 (F) -> canonical -> final rows (lane = row, 8 consecutive words per half)
+            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, int hf, const uint32_t* d) {
                 const int chi = 4 * t + w, rho = lane;
-                uint4* o = reinterpret_cast<uint4*>(out + (r0 + rho) * 256 + 16 * chi);
+                uint4* o = reinterpret_cast<uint4*>(out + (r0 + rho) * 256 + 16 * chi + 8 * hf);
 #pragma unroll
-                for (int v = 0; v < 4; ++v) {
+                for (int v = 0; v < 2; ++v) {
                     uint32_t y[4];
 #pragma unroll
                     for (int e = 0; e < 4; ++e) {
@@ -274,57 +300,74 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
                 }
             });
         } else if (!phase1) {
-            // stage 3' (F') -> sigma3 -> A_mid (I-S2 layout)
-            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+            // stage 3' (F') -> sigma3 -> A_mid (I-S2 layout: m = 32 (k&3) + rho, coeff chi)
+            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, int hf, const uint32_t* d) {
                 const int rho = (lane & 7) + 8 * w, chi = 4 * t + (lane >> 3);
-                const uint2* s3 = T3 + ((size_t)(r0 + rho) * 16 + chi) * 16;
+                const uint4* s3 = reinterpret_cast<const uint4*>(T3 + ((size_t)(r0 + rho) * 16 + chi) * 16 + 8 * hf);
+                uint8_t* dst = sh.Amid + (rho & 7) * 16 + (rho >> 3) * 512 + (chi >> 2) * 128 + (chi & 3) * 4;
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
-                    const uint2 sg = __ldg(s3 + k);
-                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), sg.x, sg.y, q);
-                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + rho, chi)) = z;
+                for (int k2 = 0; k2 < 4; ++k2) {
+                    const uint4 sg = __ldg(s3 + k2);
+#pragma unroll
+                    for (int e = 0; e < 2; ++e) {
+                        const int kk = 2 * k2 + e, k = 8 * hf + kk;
+                        const uint32_t z = shoup_mul(combine(d + 4 * kk, q, c16s), e ? sg.z : sg.x, e ? sg.w : sg.y, q);
+                        *reinterpret_cast<uint32_t*>(dst + (k >> 2) * TC_TILE + (k & 3) * 2048) = z;
+                    }
                 }
             });
             fence_async_smem();
             named_bar(TC_BAR_ID, TC_T);
-            // stage 2' (F') -> sigma2 -> staging rows -> coalesced intermediate
-            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+            // stage 2' (F') -> sigma2 -> staging (col XOR row swizzle) -> coalesced intermediate
+            tc_stage(sh, tmem, sh.Amid, sh.B + 4096, ph, [&](int t, int hf, const uint32_t* d) {
                 const int clo = 4 * t + w, rho = lane;
-                const uint2* s2 = T2 + (size_t)(r0 + rho) * 16;
+                const uint4* s2 = reinterpret_cast<const uint4*>(T2 + (size_t)(r0 + rho) * 16 + 8 * hf);
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
-                    const uint2 sg = __ldg(s2 + k);
-                    sh.stg[rho * 257 + clo + 16 * k] = shoup_mul(combine(d + 4 * k, q, c16s), sg.x, sg.y, q);
+                for (int k2 = 0; k2 < 4; ++k2) {
+                    const uint4 sg = __ldg(s2 + k2);
+#pragma unroll
+                    for (int e = 0; e < 2; ++e) {
+                        const int kk = 2 * k2 + e, k = 8 * hf + kk;
+                        const int col = clo + 16 * k;
+                        stg[rho * 256 + (col ^ rho)] = shoup_mul(combine(d + 4 * kk, q, c16s), e ? sg.z : sg.x,
+                                                                 e ? sg.w : sg.y, q);
+                    }
                 }
             });
             named_bar(TC_BAR_ID, TC_T);
 #pragma unroll 4
             for (int e = tid; e < 8192; e += TC_T) {
                 const int rho = e >> 8, col = e & 255;
-                out[(r0 + rho) * 256 + col] = sh.stg[rho * 257 + col];
+                out[(r0 + rho) * 256 + col] = stg[rho * 256 + (col ^ rho)];
             }
         } else {
-            // stage 1' (F') -> sigma1 -> A_mid (I-S0 layout)
-            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, const uint32_t* d) {
+            // stage 1' (F') -> sigma1 -> A_mid (I-S0 layout: m = 32 (k&3) + c, coeff i1)
+            tc_stage(sh, tmem, sh.Ain, sh.B + 4096, ph, [&](int t, int hf, const uint32_t* d) {
                 const int c = (lane & 7) + 8 * w, i1 = 4 * t + (lane >> 3);
-                const uint2* s1 = T1 + i1 * 16;
+                const uint4* s1 = reinterpret_cast<const uint4*>(T1 + i1 * 16 + 8 * hf);
+                uint8_t* dst = sh.Amid + (c & 7) * 16 + (c >> 3) * 512 + (i1 >> 2) * 128 + (i1 & 3) * 4;
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
-                    const uint2 sg = __ldg(s1 + k);
-                    const uint32_t z = shoup_mul(combine(d + 4 * k, q, c16s), sg.x, sg.y, q);
-                    *reinterpret_cast<uint32_t*>(sh.Amid + (k >> 2) * TC_TILE + aoff_w(32 * (k & 3) + c, i1)) = z;
+                for (int k2 = 0; k2 < 4; ++k2) {
+                    const uint4 sg = __ldg(s1 + k2);
+#pragma unroll
+                    for (int e = 0; e < 2; ++e) {
+                        const int kk = 2 * k2 + e, k = 8 * hf + kk;
+                        const uint32_t z = shoup_mul(combine(d + 4 * kk, q, c16s), e ? sg.z : sg.x, e ? sg.w : sg.y, q);
+                        *reinterpret_cast<uint32_t*>(dst + (k >> 2) * TC_TILE + (k & 3) * 2048) = z;
+                    }
                 }
             });
             fence_async_smem();
             named_bar(TC_BAR_ID, TC_T);
-            // stage 0' (folded MI0 incl. N^-1) -> canonical -> final columns
-            tc_stage(sh, tmem, sh.Amid, sh.B, ph, [&](int t, const uint32_t* d) {
+            // stage 0' (folded MI0 incl. N^-1) -> canonical -> final columns (lanes walk c)
+            tc_stage(sh, tmem, sh.Amid, sh.B, ph, [&](int t, int hf, const uint32_t* d) {
                 const int i0 = 4 * t + w, c = lane;
+                uint32_t* o = out + i0 * 256 + c0 + c;
 #pragma unroll
-                for (int k = 0; k < 16; ++k) {
-                    uint32_t y = shoup_mul(combine(d + 4 * k, q, c16s), 1u, one_s, q);
-                    y = umin32(y, y - q);
-                    __stcs(out + (i0 + 16 * k) * 256 + c0 + c, y);
+                for (int kk = 0; kk < 8; ++kk) {
+                    const int k = 8 * hf + kk;
+                    uint32_t y = shoup_mul(combine(d + 4 * kk, q, c16s), 1u, one_s, q);
+                    __stcs(o + 16 * k * 256, umin32(y, y - q));
                 }
             });
         }
@@ -336,14 +379,13 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
 
 // Standalone tensor-core kernel: persistent CTAs of 128 threads (TENSOR mode).
 template <bool FWD>
-__global__ void __launch_bounds__(TC_T, 1) ntt_tc16(TcArgs ta, uint32_t rows) {
+__global__ void __launch_bounds__(TC_T, TC_CTAS_PER_SM) ntt_tc16(TcArgs ta, uint32_t rows) {
     extern __shared__ __align__(1024) uint8_t tsm[];
     TcShared sh;
     sh.Ain = tsm;
     sh.Amid = tsm + 4 * TC_TILE;
     sh.B = tsm + 8 * TC_TILE;
-    sh.stg = reinterpret_cast<uint32_t*>(tsm + 8 * TC_TILE + 8192);
-    sh.bar = reinterpret_cast<uint64_t*>(tsm + 8 * TC_TILE + 8192 + 32 * 257 * 4);
+    sh.bar = reinterpret_cast<uint64_t*>(tsm + 8 * TC_TILE + 8192);
     sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
     const int tid = threadIdx.x;
     if (tid == 0) {
@@ -439,9 +481,10 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
 
 inline int prepare_tensor_kernels(uint32_t logN) {
     if (logN != 16) return 0;
-    if (cudaFuncSetAttribute(ntt_tc16<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess ||
-        cudaFuncSetAttribute(ntt_tc16<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess)
-        return 4;
+    for (auto k : {ntt_tc16<true>, ntt_tc16<false>})
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess ||
+            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+            return 4;
     return 0;
 }
 
@@ -456,9 +499,7 @@ inline int launch_tensor(uint32_t logN, bool fwd, const NttArgs& a, const Tensor
     ta.t2 = fwd ? tc.d_tw2 : tc.d_sg2;
     ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
     ta.c16 = tc.d_c16;
-    int occ = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_tc16<true>, TC_T, TC_SMEM);
-    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * (occ > 0 ? occ : 1)));
+    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * TC_CTAS_PER_SM));
     if (fwd) ntt_tc16<true><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
     else ntt_tc16<false><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
     return 1;

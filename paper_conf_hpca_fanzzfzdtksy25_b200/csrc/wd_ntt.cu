@@ -64,6 +64,9 @@ template <typename K>
 int set_smem(K kern, int bytes) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
         return WD_ECUDA;
+    // ask for the maximum shared-memory carveout so occupancy is limited by our own budget
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+        return WD_ECUDA;
     return WD_OK;
 }
 
@@ -352,7 +355,7 @@ int wd_ntt_check_prime(uint32_t q, uint32_t N) {
 int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
     if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_FUSED) return set_err(WD_EINVAL);
     if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED) && !tensor_supported(p->logN)) return set_err(WD_EUNSUPPORTED);
-    if (tensor_share > 1.0f) return set_err(WD_EINVAL);
+    if (tensor_share > 2.0f) return set_err(WD_EINVAL);
     p->mode = mode;
     if (tensor_share >= 0.0f) p->tensor_share = tensor_share;
     return set_err(WD_OK);
@@ -360,6 +363,19 @@ int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
 int wd_ntt_plan_get_mode(const wd_ntt_plan* p) { return p ? effective_mode(p) : -1; }
 
 uint32_t wd_ntt_last_launches(void) { return g_last_launches; }
+
+int wd_ntt_occupancy(const wd_ntt_plan* p, int mode, int fwd) {
+    if (!p) return -1;
+    int occ = -1;
+    cudaError_t e = cudaErrorInvalidValue;
+    if (p->logN == 16 && mode == WD_MODE_TENSOR)
+        e = fwd ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_tc16<true>, TC_T, TC_SMEM)
+                : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_tc16<false>, TC_T, TC_SMEM);
+    else if (p->logN == 16 && mode == WD_MODE_CUDA)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_persist_cc<16, true, false>, 512, PGeo<16>::SMEM_BYTES);
+    if (e != cudaSuccess) { cudaGetLastError(); return -(int)e; }
+    return occ;
+}
 int wd_ntt_last_error(void) { return g_last_error; }
 const char* wd_ntt_strerror(int code) {
     switch (code) {

@@ -54,6 +54,7 @@ _SIGS = {
     "wd_ntt_plan_set_mode": (_i32, [_vp, _i32, _f32]),
     "wd_ntt_plan_get_mode": (_i32, [_vp]),
     "wd_ntt_last_launches": (_u32, []),
+    "wd_ntt_occupancy": (_i32, [_vp, _i32, _i32]),
     "wd_ntt_last_error": (_i32, []),
     "wd_ntt_strerror": (ctypes.c_char_p, [_i32]),
     "wd_ntt_version": (ctypes.c_char_p, []),
@@ -163,6 +164,11 @@ def wd_ntt_plan_get_mode(plan: int) -> int:
 
 def wd_ntt_last_launches() -> int:
     return _lib.wd_ntt_last_launches()
+
+
+def wd_ntt_occupancy(plan: int, mode, fwd: bool = True) -> int:
+    mode = MODES[mode] if isinstance(mode, str) else int(mode)
+    return _lib.wd_ntt_occupancy(plan, mode, 1 if fwd else 0)
 
 
 def wd_ntt_last_error() -> int:

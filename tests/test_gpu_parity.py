@@ -201,14 +201,17 @@ def _modes(wd):
     return ["cuda", "tensor", "fused"]
 
 
-@pytest.mark.parametrize("mode", ["cuda", "tensor", "fused"])
-def test_modes_vs_oracle_n65536(wd, mode):
+MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.25), ("fused", 2.0)]
+
+
+@pytest.mark.parametrize("mode,share", MODES)
+def test_modes_vs_oracle_n65536(wd, mode, share):
     n = 1 << 16
     primes = [P[0], P[13], P[59]]
     x = inputs.uniform_residues(primes, n, 3, 77)
     plan = wd.Plan(n, primes)
     try:
-        plan.set_mode(mode)
+        plan.set_mode(mode, share)
     except wd.WdNttError as e:
         pytest.fail("mode %s unavailable: %s" % (mode, e))
     y = gpu_fwd(wd, plan, x)
@@ -220,14 +223,14 @@ def test_modes_vs_oracle_n65536(wd, mode):
     assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes)), mode
 
 
-@pytest.mark.parametrize("mode", ["tensor", "fused"])
-def test_modes_headline_config(wd, mode):
+@pytest.mark.parametrize("mode,share", MODES[1:])
+def test_modes_headline_config(wd, mode, share):
     n, L, batch = 1 << 16, 36, 128
     primes = P[:L]
     x = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 2, device="cuda")
     plan = wd.Plan(n, primes)
     ref_plan = wd.Plan(n, primes, mode="cuda")
-    plan.set_mode(mode)
+    plan.set_mode(mode, share)
     y = torch.empty_like(x)
     yr = torch.empty_like(x)
     plan.forward(x, y)
