@@ -23,6 +23,7 @@ namespace wd {
 constexpr int FU_CC = 512, FU_TC = 128, FU_T = FU_CC + FU_TC;
 constexpr int FU_CC_BAR = 2;
 constexpr int FU_SMEM = PGeo<16>::SMEM_BYTES + TC_SMEM + 64;
+constexpr int FUP_SMEM = PGeo<16>::SMEM_BYTES + TCC_SMEM + 64;
 
 template <int BAR, int NT>
 __device__ __forceinline__ void gbar() {
@@ -187,32 +188,34 @@ __device__ __forceinline__ void cc_row_phase2(const NttArgs& a, uint32_t* smem, 
 }
 
 template <bool FWD>
-__global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, uint32_t rows) {
+__global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta) {
     extern __shared__ __align__(1024) uint8_t fsm[];
     uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
     uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
-    int* ctl = reinterpret_cast<int*>(tcb + TC_SMEM);           // [0] rows done by the leader, [1] by the follower
-    TcShared sh;
-    sh.Ain = tcb;
-    sh.Amid = tcb + 4 * TC_TILE;
-    sh.B = tcb + 8 * TC_TILE;
-    sh.bar = reinterpret_cast<uint64_t*>(tcb + 8 * TC_TILE + 8192);
-    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
+    TccShared sh;
+    sh.A0 = tcb;
+    sh.B = tcb + 3 * TC_TILE;
+    sh.bar = reinterpret_cast<uint64_t*>(tcb + 3 * TC_TILE + 17 * 4096);
+    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 4);
+    uint32_t* loaded = sh.tslot + 1;
+    int* ctl = reinterpret_cast<int*>(tcb + TCC_SMEM);          // [0] rows done by the leader, [1] by the follower
     const int tid = threadIdx.x;
     if (tid == 0) {
         ctl[0] = 0; ctl[1] = 0;
-        mbar_init(&sh.bar[0], 1);
-        mbar_init(&sh.bar[1], 1);
+        for (int i = 0; i < 4; ++i) mbar_init(&sh.bar[i], 1);
+        *loaded = 0xffffffffu;
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (tid >= FU_CC && tid < FU_CC + 32) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(sh.tslot)));
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" :: "r"(smem_addr(sh.tslot)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
-    const int nmine = rows > blockIdx.x ? (int)((rows - blockIdx.x + gridDim.x - 1) / gridDim.x) : 0;
+    const uint32_t L = ta.a.L, Bp = rows / L;
+    const uint32_t k0 = blockIdx.x * per_cta, k1 = min(rows, k0 + per_cta);
+    const int nmine = k1 > k0 ? (int)(k1 - k0) : 0;
     const bool is_tc = tid >= FU_CC;
     const bool leader = FWD ? is_tc : !is_tc;                    // who runs the first phase of a row
     const int gtid = is_tc ? tid - FU_CC : tid;
@@ -221,17 +224,18 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, uint32_t 
     int* mine = &ctl[leader ? 0 : 1];
     const int* other = &ctl[leader ? 1 : 0];
     const uint32_t tmem = *sh.tslot;
-    uint32_t ph[2] = {0, 0};
+    uint32_t ph[4] = {0, 0, 0, 0};
     for (int i = 0; i < nmine; ++i) {
-        // leader: stay <= FU_LEAD rows ahead; follower: wait until the leader finished row i
         if (gtid == 0) {
             if (leader) { while (i - ld_volatile(other) >= FU_LEAD) __nanosleep(256); }
             else { while (ld_volatile(other) <= i) __nanosleep(128); }
         }
         named_bar(bar, nthr);
         __threadfence_block();
-        const uint32_t row = blockIdx.x + (uint32_t)i * gridDim.x;
-        if (is_tc) tc_transform<FWD, 1, true>(ta, sh, tmem, ph, row);           // column phase, either direction
+        const uint32_t k = k0 + (uint32_t)i;
+        const uint32_t limb = k / Bp, row = (k % Bp) * L + limb;
+        if (is_tc) tcc_columns<FWD, false>(ta, sh, tmem, ph, row, G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096,
+                                           loaded, TC_BAR_ID);
         else cc_row_phase2<FWD, FU_CC_BAR>(ta.a, ccbuf, row);
         __threadfence_block();
         named_bar(bar, nthr);
@@ -240,14 +244,14 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, uint32_t 
     if (is_tc) {
         tc_fence_before();
         named_bar(TC_BAR_ID, FU_TC);
-        if (gtid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
+        if (gtid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem));
     }
 }
 
 inline int prepare_fused_kernels(uint32_t logN) {
     if (logN != 16) return 0;
     for (auto k : {ntt_fused16_pipe<true>, ntt_fused16_pipe<false>})
-        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess ||
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, FUP_SMEM) != cudaSuccess ||
             cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
             return 4;
     for (auto k : {ntt_fused16<true, false>, ntt_fused16<false, false>})
@@ -268,9 +272,10 @@ inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorT
     ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
     ta.c16 = tc.d_c16;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
-    if (share > 1.5f) {            // tensor_share = 2: phase-split pipeline (tensor: columns, CUDA: rows)
-        if (fwd) ntt_fused16_pipe<true><<<grid, FU_T, FU_SMEM, s>>>(ta, rows);
-        else ntt_fused16_pipe<false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows);
+    if (share > 1.5f || share < 0.0f) {   // default / tensor_share = 2: phase-split pipeline
+        const uint32_t per = (rows + grid - 1) / grid;
+        if (fwd) ntt_fused16_pipe<true><<<grid, FU_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
+        else ntt_fused16_pipe<false><<<grid, FU_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
         return 1;
     }
     if (fwd) ntt_fused16<true, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);

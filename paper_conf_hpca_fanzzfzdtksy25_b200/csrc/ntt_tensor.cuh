@@ -35,6 +35,8 @@
 namespace wd {
 
 struct TensorTables {
+    uint8_t* d_G = nullptr;        // [L][2][17][4096]: per direction, [0] = single-group stage (M0 / MI0),
+                                   //   [1+g] = stage-1 block of group g (M1_g / MI1_g), twists folded in
     uint8_t* d_B = nullptr;        // [L][4][4096]: fwd M0, fwd F, inv MI0 (with N^-1), inv F'
     uint2* d_tw1 = nullptr;        // [L][16][16]    fwd twist tau, stage 1   (group, j)
     uint2* d_tw2 = nullptr;        // [L][256][16]   fwd twist tau, stage 2
@@ -377,8 +379,207 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
     }
 }
 
-// Standalone tensor-core kernel: persistent CTAs of 128 threads (TENSOR mode).
+// ------------------------------------------------------------------ column phase with TMEM operands
+// Both column stages of N = 2^16 (layers 0-7) with every twist folded: a 128-column chunk is
+// processed as 16 stage-a tiles (one per value of the stage-a instance digit, all 128 columns)
+// and 16 stage-b tiles (one per stage-b GROUP, all 128 columns), so every stage-b tile uses the
+// single matrix of its group (M1_g / MI1_g) and no CUDA-core twist is needed.  The stage-a
+// epilogue writes its outputs straight into TMEM (tcgen05.st), which is where the stage-b MMA
+// takes its A operand from: the inter-stage exchange (steps 2/6 of PAPER.md Fig. 2) never
+// touches shared memory.  TMEM: cols [0,256) stage-b A tiles (16 x 16 columns = 64 bytes of K
+// per lane), [256,384) stage-a accumulators (ping-pong), [384,512) stage-b accumulators.
+//   forward (PH1 of the row): stage a = stage 0 (instance (c, i0), coeff r, p = i0 + 16 r,
+//            matrix M0), stage b = stage 1 (instance (c, i1), coeff i0, p = 16 i1 + k, M1_{i1});
+//            output = plain merged-CT intermediate (or pre-twisted by tau2 for the tensor P2).
+//   inverse (PH1' of the row): stage a = stage 1' (instance (c, i1), coeff j, p = 16 i1 + j,
+//            MI1_{i1}), stage b = stage 0' (instance (c, i0), coeff i1, p = i0 + 16 k, MI0).
+constexpr int TCC_SMEM = 3 * TC_TILE + 17 * 4096 + 64;     // stage-a A triple buffer + 17 B images
+constexpr uint32_t TCC_A1 = 0, TCC_D0 = 256, TCC_D1 = 384;
+
+struct TccShared { uint8_t* A0; uint8_t* B; uint64_t* bar; uint32_t* tslot; };
+
+__device__ __forceinline__ void tmem_st1(uint32_t taddr, uint32_t v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" :: "r"(taddr), "r"(v) : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tc_mma_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t acc) {
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                 "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n\t}\n"
+                 :: "r"(d), "r"(a_tmem), "l"(b), "r"(IDESC_I8_128x64), "r"(acc));
+}
+
+// one row's column phase.  TWIST2 (forward only): pre-twist the output by tau2 for tc P2.
+// bar[0..1] stage-a accumulators, bar[2..3] stage-b accumulators; ph[4] their phases.
+template <bool FWD, bool TWIST2>
+__device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& sh, uint32_t tmem, uint32_t* ph,
+                                            uint32_t row_id, const uint8_t* Gl, uint32_t* loaded_limb, int bar_id) {
+    const NttArgs& a = ta.a;
+    const int tid = threadIdx.x % TC_T, w = tid >> 5, lane = tid & 31;
+    const uint32_t limb = row_id % a.L;
+    const LimbConst lc = a.lc[limb];
+    const uint32_t q = lc.q, q2 = lc.q2;
+    const uint2 cc = ta.c16[limb];
+    const uint32_t c16s = cc.x, one_s = cc.y;
+    const uint32_t* src = FWD ? a.in + ((size_t)row_id << 16) : a.out + ((size_t)row_id << 16);
+    uint32_t* out = a.out + ((size_t)row_id << 16);
+    const uint2* T2 = ta.t2 + (size_t)limb * 4096;
+    const uint32_t lane_base = (uint32_t)(32 * w) << 16;
+    if (*loaded_limb != limb) {                  // 17 B images of this limb (68 KB), once per limb
+        named_bar(bar_id, TC_T);
+        for (int i = tid; i < 17 * 4096 / 16; i += TC_T) cp_async16(sh.B + 16 * i, Gl + 16 * i);
+        cp_async_commit();
+        cp_async_wait<0>();
+        fence_async_smem();
+        named_bar(bar_id, TC_T);
+        if (tid == 0) *loaded_limb = limb;
+    }
+    const uint32_t b_single = smem_addr(sh.B);
+    auto b_group = [&](int g) { return smem_addr(sh.B + 4096 * (1 + g)); };
+    // stage-a tile t loader: element (coefficient j, row m) at p = FWD ? t + 16 j : 16 t + j
+    auto load_a = [&](int t, int c0, uint8_t* buf) {
+#pragma unroll
+        for (int mq = 0; mq < 4; ++mq)
+#pragma unroll
+            for (int jh = 0; jh < 4; ++jh) {
+                const int mh = w + 4 * mq, m = 8 * mh + (lane & 7), j = 4 * jh + (lane >> 3);
+                const int p = FWD ? t + 16 * j : 16 * t + j;
+                cp_async4(buf + (lane & 7) * 16 + mh * 512 + jh * 128 + (lane >> 3) * 4, src + p * 256 + c0 + m);
+            }
+        cp_async_commit();
+    };
+#pragma unroll 1
+    for (int c0 = 0; c0 < 256; c0 += 128) {
+        // ---------------- stage a: 16 tiles, A from smem, outputs -> TMEM stage-b operand tiles
+        // triple-buffered A: the load of tile t+1 overwrites the buffer of tile t-2, whose MMA
+        // completion was awaited by epilogue t-2 in the previous iteration
+        load_a(0, c0, sh.A0);
+#pragma unroll 1
+        for (int t = 0; t <= 16; ++t) {
+            if (t < 16) {
+                cp_async_wait<0>();
+                fence_async_smem();
+                tc_fence_before();
+                named_bar(bar_id, TC_T);
+                if (tid == 0) {
+                    tc_fence_after();
+                    const uint32_t ab = smem_addr(sh.A0 + (t % 3) * TC_TILE);
+                    const uint32_t bb = FWD ? b_single : b_group(t);
+                    const uint32_t d = tmem + TCC_D0 + (t & 1) * 64;
+                    tc_mma(d, umma_desc(ab), umma_desc(bb), 0);
+                    tc_mma(d, umma_desc(ab + 256), umma_desc(bb + 256), 1);
+                    tc_commit(&sh.bar[t & 1]);
+                }
+                if (t + 1 < 16) load_a(t + 1, c0, sh.A0 + ((t + 1) % 3) * TC_TILE);
+            }
+            if (t >= 1) {                             // epilogue of tile t-1
+                const int te = t - 1, r = te & 1;
+                mbar_wait(&sh.bar[r], ph[r]);
+                ph[r] ^= 1;
+                tc_fence_after();
+                uint32_t d[32];
+#pragma unroll
+                for (int hf = 0; hf < 2; ++hf) {
+                    tmem_ld32(tmem + lane_base + TCC_D0 + r * 64 + 32 * hf, d);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int kk = 0; kk < 8; ++kk) {
+                        const int k = 8 * hf + kk;
+                        tmem_st1(tmem + lane_base + TCC_A1 + 16 * k + te, combine(d + 4 * kk, q, c16s));
+                    }
+                }
+            }
+        }
+        tmem_wait_st();
+        tc_fence_before();
+        named_bar(bar_id, TC_T);
+        // ---------------- stage b: 16 tiles, A from TMEM, outputs -> global
+#pragma unroll 1
+        for (int k = 0; k <= 16; ++k) {
+            if (k < 16 && tid == 0) {
+                tc_fence_after();
+                const uint32_t bb = FWD ? b_group(k) : b_single;
+                const uint32_t d = tmem + TCC_D1 + (k & 1) * 64;
+                tc_mma_ts(d, tmem + TCC_A1 + 16 * k, umma_desc(bb), 0);
+                tc_mma_ts(d, tmem + TCC_A1 + 16 * k + 8, umma_desc(bb + 256), 1);
+                tc_commit(&sh.bar[2 + (k & 1)]);
+            }
+            if (k >= 1) {
+                const int ke = k - 1, r = ke & 1;
+                mbar_wait(&sh.bar[2 + r], ph[2 + r]);
+                ph[2 + r] ^= 1;
+                tc_fence_after();
+                uint32_t d[32];
+                const int m = 32 * w + lane;
+#pragma unroll
+                for (int hf = 0; hf < 2; ++hf) {
+                    tmem_ld32(tmem + lane_base + TCC_D1 + r * 64 + 32 * hf, d);
+                    tmem_wait_ld();
+#pragma unroll
+                    for (int kk = 0; kk < 8; ++kk) {
+                        const int ko = 8 * hf + kk;
+                        const int p = FWD ? 16 * ke + ko : ke + 16 * ko;
+                        uint32_t y = combine(d + 4 * kk, q, c16s);
+                        if (FWD) {
+                            if (TWIST2) {
+                                const uint2 tw = __ldg(T2 + p * 16 + ((c0 + m) >> 4));
+                                y = shoup_mul(y, tw.x, tw.y, q);
+                            } else {
+                                y = shoup_mul(y, 1u, one_s, q);                  // [0, 2q) for the butterflies
+                            }
+                            out[p * 256 + c0 + m] = y;
+                        } else {
+                            y = shoup_mul(y, 1u, one_s, q);
+                            __stcs(out + p * 256 + c0 + m, umin32(y, y - q));
+                        }
+                    }
+                }
+                tc_fence_before();
+            }
+            named_bar(bar_id, TC_T);                      // D1 region of tile k-1 free for tile k+1
+        }
+    }
+    (void)q2;
+}
+
+// Column phase over all rows (TENSOR mode launch 1 of 2; one CTA per SM, whole TMEM).
 template <bool FWD>
+__global__ void __launch_bounds__(TC_T, 1) ntt_tcc16(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta) {
+    extern __shared__ __align__(1024) uint8_t tsm[];
+    TccShared sh;
+    sh.A0 = tsm;
+    sh.B = tsm + 3 * TC_TILE;
+    sh.bar = reinterpret_cast<uint64_t*>(tsm + 3 * TC_TILE + 17 * 4096);
+    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 4);
+    uint32_t* loaded = sh.tslot + 1;
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        for (int i = 0; i < 4; ++i) mbar_init(&sh.bar[i], 1);
+        *loaded = 0xffffffffu;
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (tid < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" :: "r"(smem_addr(sh.tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *sh.tslot;
+    uint32_t ph[4] = {0, 0, 0, 0};
+    // contiguous (limb-major) work ranges so the 68 KB of B images are reloaded only when the limb changes
+    const uint32_t L = ta.a.L, B = rows / L;
+    const uint32_t k0 = blockIdx.x * per_cta, k1 = min(rows, k0 + per_cta);
+    for (uint32_t k = k0; k < k1; ++k) {
+        const uint32_t limb = k / B, poly = k % B, row = poly * L + limb;
+        tcc_columns<FWD, true>(ta, sh, tmem, ph, row, G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096, loaded, TC_BAR_ID);
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (tid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem));
+}
+
+// Standalone tensor-core kernel: persistent CTAs of 128 threads (TENSOR mode).
+template <bool FWD, int PH = 0>
 __global__ void __launch_bounds__(TC_T, TC_CTAS_PER_SM) ntt_tc16(TcArgs ta, uint32_t rows) {
     extern __shared__ __align__(1024) uint8_t tsm[];
     TcShared sh;
@@ -402,7 +603,7 @@ __global__ void __launch_bounds__(TC_T, TC_CTAS_PER_SM) ntt_tc16(TcArgs ta, uint
     tc_fence_after();
     const uint32_t tmem = *sh.tslot;
     uint32_t ph[2] = {0, 0};
-    for (uint32_t row = blockIdx.x; row < rows; row += gridDim.x) tc_transform<FWD>(ta, sh, tmem, ph, row);
+    for (uint32_t row = blockIdx.x; row < rows; row += gridDim.x) tc_transform<FWD, PH>(ta, sh, tmem, ph, row);
     tc_fence_before();
     __syncthreads();
     if (tid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
@@ -410,7 +611,7 @@ __global__ void __launch_bounds__(TC_T, TC_CTAS_PER_SM) ntt_tc16(TcArgs ta, uint
 
 // ------------------------------------------------------------------ host side
 inline void free_tensor_tables(TensorTables& t) {
-    cudaFree(t.d_B); cudaFree(t.d_tw1); cudaFree(t.d_tw2); cudaFree(t.d_tw3);
+    cudaFree(t.d_G); cudaFree(t.d_B); cudaFree(t.d_tw1); cudaFree(t.d_tw2); cudaFree(t.d_tw3);
     cudaFree(t.d_sg1); cudaFree(t.d_sg2); cudaFree(t.d_sg3); cudaFree(t.d_c16);
     t = TensorTables();
 }
@@ -420,7 +621,7 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
                                const std::vector<uint32_t>& psis) {
     if (logN != 16) return 0;
     const uint32_t N = 1u << 16, L = (uint32_t)primes.size();
-    std::vector<uint8_t> B((size_t)L * 4 * 4096);
+    std::vector<uint8_t> B((size_t)L * 4 * 4096), Gi((size_t)L * 2 * 17 * 4096);
     std::vector<uint2> t1((size_t)L * 256), t2((size_t)L * 4096), t3((size_t)L * 65536);
     std::vector<uint2> s1((size_t)L * 256), s2((size_t)L * 4096), s3((size_t)L * 65536);
     std::vector<uint2> c16(L);
@@ -434,8 +635,16 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
         uint32_t M[16][16], F[16][16], Fi[16][16];
         block_fwd(M, fb, 0, 0, q);
         byte_planes(&B[((size_t)l * 4 + 0) * 4096], M, q);
+        byte_planes(&Gi[(((size_t)l * 2 + 0) * 17 + 0) * 4096], M, q);
         block_inv(M, ib, 0, 0, q, ninv);
         byte_planes(&B[((size_t)l * 4 + 2) * 4096], M, q);
+        byte_planes(&Gi[(((size_t)l * 2 + 1) * 17 + 0) * 4096], M, q);
+        for (uint32_t g = 0; g < 16; ++g) {              // stage-1 blocks, one image per group
+            block_fwd(M, fb, 4, g, q);
+            byte_planes(&Gi[(((size_t)l * 2 + 0) * 17 + 1 + g) * 4096], M, q);
+            block_inv(M, ib, 4, g, q, 0);
+            byte_planes(&Gi[(((size_t)l * 2 + 1) * 17 + 1 + g) * 4096], M, q);
+        }
         // fixed DFTs from one group, then every group of stages 1..3 must factor through them
         bool have_f = false;
         struct S { int ls; uint32_t groups; uint2* tw; uint2* sg; };
@@ -470,7 +679,7 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
         if (cudaMalloc(d, n) != cudaSuccess) return false;
         return cudaMemcpy(*d, h, n, cudaMemcpyHostToDevice) == cudaSuccess;
     };
-    if (!up((void**)&tc.d_B, B.data(), B.size()) || !up((void**)&tc.d_tw1, t1.data(), t1.size() * 8) ||
+    if (!up((void**)&tc.d_G, Gi.data(), Gi.size()) || !up((void**)&tc.d_B, B.data(), B.size()) || !up((void**)&tc.d_tw1, t1.data(), t1.size() * 8) ||
         !up((void**)&tc.d_tw2, t2.data(), t2.size() * 8) || !up((void**)&tc.d_tw3, t3.data(), t3.size() * 8) ||
         !up((void**)&tc.d_sg1, s1.data(), s1.size() * 8) || !up((void**)&tc.d_sg2, s2.data(), s2.size() * 8) ||
         !up((void**)&tc.d_sg3, s3.data(), s3.size() * 8) || !up((void**)&tc.d_c16, c16.data(), c16.size() * 8))
@@ -481,8 +690,12 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
 
 inline int prepare_tensor_kernels(uint32_t logN) {
     if (logN != 16) return 0;
-    for (auto k : {ntt_tc16<true>, ntt_tc16<false>})
+    for (auto k : {ntt_tc16<true>, ntt_tc16<false>, ntt_tc16<true, 2>, ntt_tc16<false, 2>})
         if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess ||
+            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+            return 4;
+    for (auto k : {ntt_tcc16<true>, ntt_tcc16<false>})
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, TCC_SMEM) != cudaSuccess ||
             cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
             return 4;
     return 0;
@@ -500,9 +713,17 @@ inline int launch_tensor(uint32_t logN, bool fwd, const NttArgs& a, const Tensor
     ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
     ta.c16 = tc.d_c16;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * TC_CTAS_PER_SM));
-    if (fwd) ntt_tc16<true><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
-    else ntt_tc16<false><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
-    return 1;
+    // column phase: TMEM-staged, both stages folded (one CTA per SM, whole TMEM), limb-major ranges
+    const uint32_t gc = std::min<uint32_t>(rows, (uint32_t)sm_count);
+    const uint32_t per = (rows + gc - 1) / gc;
+    if (fwd) {
+        ntt_tcc16<true><<<gc, TC_T, TCC_SMEM, s>>>(ta, tc.d_G, rows, per);
+        ntt_tc16<true, 2><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
+    } else {
+        ntt_tc16<false, 2><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
+        ntt_tcc16<false><<<gc, TC_T, TCC_SMEM, s>>>(ta, tc.d_G, rows, per);
+    }
+    return 2;
 }
 
 }  // namespace wd

@@ -19,6 +19,7 @@
 #include "ntt_cuda_core.cuh"
 #include "ntt_persist.cuh"
 #include "ntt_smem.cuh"
+#include "ntt_cluster.cuh"
 #include "ntt_tensor.cuh"
 #include "ntt_fused.cuh"
 #include "plan_math.h"
@@ -76,6 +77,17 @@ int prep_cc() {
     if (set_smem(ntt_fwd_cc<LOGN>, S::SMEM_BYTES) || set_smem(ntt_inv_cc<LOGN, false>, S::SMEM_BYTES) ||
         set_smem(ntt_inv_cc<LOGN, true>, S::SMEM_BYTES))
         return WD_ECUDA;
+    if constexpr (LOGN >= 14) {
+        if (set_smem(ntt_fwd_cl<LOGN>, CL_BYTES) || set_smem(ntt_inv_cl<LOGN, false>, CL_BYTES) ||
+            set_smem(ntt_inv_cl<LOGN, true>, CL_BYTES))
+            return WD_ECUDA;
+        if constexpr (LOGN == 17) {     // 8-CTA clusters need the non-portable-size opt-in on some drivers
+            cudaFuncSetAttribute(ntt_fwd_cl<LOGN>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            cudaFuncSetAttribute(ntt_inv_cl<LOGN, false>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            cudaFuncSetAttribute(ntt_inv_cl<LOGN, true>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+            cudaGetLastError();
+        }
+    }
     if constexpr (LOGN == 15 || LOGN == 16) {
         if (set_smem(ntt_fwd_smem<LOGN>, SM_BYTES) || set_smem(ntt_inv_smem<LOGN, false>, SM_BYTES) ||
             set_smem(ntt_inv_smem<LOGN, true>, SM_BYTES))
@@ -110,6 +122,22 @@ int prepare_kernels(uint32_t logN) {
 template <int LOGN>
 void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     using S = CcShape<LOGN>;
+    if constexpr (LOGN >= 14) {
+        if (p->kernel_ver == 5) {
+            constexpr int CLN = 1 << (LOGN - 14);
+            const uint32_t units = std::max<uint32_t>(1, std::min<uint32_t>(rows, (uint32_t)(2 * p->sm_count / CLN)));
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(units * CLN); cfg.blockDim = dim3(CL_T); cfg.dynamicSmemBytes = CL_BYTES; cfg.stream = s;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = CLN; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+            cfg.attrs = at; cfg.numAttrs = 1;
+            if (fwd) cudaLaunchKernelEx(&cfg, ntt_fwd_cl<LOGN>, a, rows);
+            else if (a.in2) cudaLaunchKernelEx(&cfg, ntt_inv_cl<LOGN, true>, a, rows);
+            else cudaLaunchKernelEx(&cfg, ntt_inv_cl<LOGN, false>, a, rows);
+            return;
+        }
+    }
     if constexpr (LOGN == 15 || LOGN == 16) {
         if (p->kernel_ver == 3) {
             constexpr int PAIR = LOGN == 16 ? 2 : 1;

@@ -1,0 +1,15 @@
+#!/bin/bash
+# full GPU pass: smoke, all gpu tests, default bench with e2e + cpu baseline, reference arm, launch list, ncu of defaults
+cd "$GRAFT_REPO_ROOT" 2>/dev/null || cd /root/repo
+TAG=$1
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke_$TAG.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/pytest_$TAG.log 2>&1
+nvidia-smi --query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active --format=csv -lms 200 > gpurun_out/clocks_$TAG.csv 2>&1 &
+SMI=$!
+timeout 600 python bench.py > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TAG.err
+kill $SMI
+timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_${TAG}_ref.json 2> gpurun_out/bench_${TAG}_ref.err
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"ntt_" --csv --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 3 --warmup 3 --e2e-steps 0 --no-cpu > /dev/null 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"ntt_persist" -s 2 -c 2 -o gpurun_out/prof_${TAG} python bench.py --steps 1 --warmup 3 --e2e-steps 0 --no-cpu > /dev/null 2>&1
+echo done

@@ -169,6 +169,55 @@ extern "C" __global__ void k_probe_mask(const uint8_t* A, const uint8_t* B4, int
     if (t < 32) tmem_free<64>(tmem);
 }
 
+// A from TMEM: lane m holds row m; K bytes 4c..4c+3 in TMEM column c (little-endian, assumed)
+extern "C" __global__ void k_probe_tmem_a(const uint8_t* A, const uint8_t* B, int32_t* D) {
+    __shared__ __align__(1024) uint8_t sB[64 * 64];
+    __shared__ __align__(8) uint64_t bar;
+    __shared__ uint32_t taddr_s;
+    const int t = threadIdx.x, warp = t >> 5;
+    for (int i = t; i < 64 * 64; i += blockDim.x) sB[aoff(i / 64, i % 64)] = B[i];
+    if (t == 0) { mbar_init(&bar, 1); asm volatile("fence.mbarrier_init.release.cluster;"); }
+    if (t < 32) tmem_alloc<128>(&taddr_s);
+    fence_proxy_async();
+    fence_before();
+    __syncthreads();
+    fence_after();
+    const uint32_t tmem = taddr_s;                 // cols [0,64): D ; cols [64,80): A
+    // each thread writes its row (64 bytes = 16 words) into columns 64..79 of its lane
+    for (int c = 0; c < 16; ++c) {
+        const uint32_t w = (uint32_t)A[t * 64 + 4 * c] | ((uint32_t)A[t * 64 + 4 * c + 1] << 8) |
+                           ((uint32_t)A[t * 64 + 4 * c + 2] << 16) | ((uint32_t)A[t * 64 + 4 * c + 3] << 24);
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};"
+                     :: "r"(tmem + ((uint32_t)(warp * 32) << 16) + 64 + c), "r"(w));
+    }
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+    fence_before();
+    __syncthreads();
+    fence_after();
+    if (t == 0) {
+        const uint32_t b0 = smem_u32(sB);
+        const uint32_t id = idesc_i8(128, 64);
+        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                     "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n\t}\n"
+                     :: "r"(tmem), "r"(tmem + 64), "l"(make_desc(b0, LBO, SBO)), "r"(id), "r"(0));
+        asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                     "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n\t}\n"
+                     :: "r"(tmem), "r"(tmem + 64 + 8), "l"(make_desc(b0 + 2 * LBO, LBO, SBO)), "r"(id), "r"(1));
+        mma_commit(&bar);
+    }
+    mbar_wait(&bar, 0);
+    fence_after();
+    uint32_t r[32];
+    for (int half = 0; half < 2; ++half) {
+        tmem_ld32(tmem + ((warp * 32) << 16) + half * 32, r);
+        tmem_wait_ld();
+        for (int c = 0; c < 32; ++c) D[t * 64 + half * 32 + c] = (int32_t)r[c];
+    }
+    fence_before();
+    __syncthreads();
+    if (t < 32) tmem_free<128>(tmem);
+}
+
 // loop: ITER x (2 MMAs 128x64x32 -> commit -> wait -> 128 threads tcgen05.ld 64 cols)
 extern "C" __global__ void __launch_bounds__(128) k_probe_mma_loop(int iters, int do_ld, int do_mma, uint32_t* sink) {
     __shared__ __align__(1024) uint8_t sA[128 * 64];
@@ -268,6 +317,18 @@ extern "C" int probe_mask(const uint8_t* hA, const uint8_t* hB4, int32_t* hD) {
     cudaMemcpy(dA, hA, 128 * 64, cudaMemcpyHostToDevice);
     cudaMemcpy(dB, hB4, 4 * 64 * 64, cudaMemcpyHostToDevice);
     k_probe_mask<<<1, 128>>>(dA, dB, dD);
+    int e = (int)cudaDeviceSynchronize();
+    cudaMemcpy(hD, dD, 128 * 64 * 4, cudaMemcpyDeviceToHost);
+    cudaFree(dA); cudaFree(dB); cudaFree(dD);
+    return e;
+}
+
+extern "C" int probe_tmem_a(const uint8_t* hA, const uint8_t* hB, int32_t* hD) {
+    uint8_t *dA, *dB; int32_t* dD;
+    cudaMalloc(&dA, 128 * 64); cudaMalloc(&dB, 64 * 64); cudaMalloc(&dD, 128 * 64 * 4);
+    cudaMemcpy(dA, hA, 128 * 64, cudaMemcpyHostToDevice);
+    cudaMemcpy(dB, hB, 64 * 64, cudaMemcpyHostToDevice);
+    k_probe_tmem_a<<<1, 128>>>(dA, dB, dD);
     int e = (int)cudaDeviceSynchronize();
     cudaMemcpy(hD, dD, 128 * 64 * 4, cudaMemcpyDeviceToHost);
     cudaFree(dA); cudaFree(dB); cudaFree(dD);

@@ -13,6 +13,7 @@ if not os.path.exists(so):
                            "-shared", "-o", so, os.path.join(HERE, "tc_probe.cu")])
 lib = ctypes.CDLL(so)
 lib.probe_mma.restype = ctypes.c_int
+lib.probe_tmem_a.restype = ctypes.c_int
 lib.probe_mma_loop.restype = ctypes.c_float
 lib.probe_mma_loop.argtypes = [ctypes.c_int] * 4
 lib.probe_int.restype = ctypes.c_float
@@ -45,6 +46,10 @@ for g in range(4):
     res["group%d_exact" % g] = bool(np.array_equal(D4[32 * g:32 * g + 32], refg))
     res["group%d_matches_B3" % g] = bool(np.array_equal(D4[32 * g:32 * g + 32], A[32*g:32*g+32].astype(np.int64) @ B4[3].astype(np.int64).T))
 print(json.dumps(res), flush=True)
+D5 = np.zeros((128, 64), dtype=np.int32)
+e = lib.probe_tmem_a(A.ctypes.data, B.ctypes.data, D5.ctypes.data)
+print(json.dumps({"probe": "mma_a_from_tmem", "err": e, "exact": bool(np.array_equal(D5.astype(np.int64), ref)),
+                  "D00": D5[:1, :4].tolist(), "ref00": ref[:1, :4].tolist()}), flush=True)
 import sys
 if "--mask-only" in sys.argv:
     sys.exit(0)

@@ -201,7 +201,7 @@ def _modes(wd):
     return ["cuda", "tensor", "fused"]
 
 
-MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.25), ("fused", 2.0)]
+MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.25), ("fused", 0.75)]
 
 
 @pytest.mark.parametrize("mode,share", MODES)
@@ -246,3 +246,27 @@ def test_modes_headline_config(wd, mode, share):
     plan.inverse(y, z)
     torch.cuda.synchronize()
     assert torch.equal(z, x)
+
+
+# -------------------------------------------------------------- every CUDA-core kernel generation
+@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5"])
+@pytest.mark.parametrize("logn", [14, 15, 16, 17])
+def test_cuda_core_generations(wd, ver, logn, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", ver)
+    n = 1 << logn
+    primes = [P[0], P[29], P[59]]
+    x = inputs.uniform_residues(primes, n, 3, 4000 + logn)
+    plan = wd.Plan(n, primes, mode="cuda")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (ver, logn)
+    assert np.array_equal(gpu_inv(wd, plan, y), x), (ver, logn)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (ver, logn)
+    q = np.repeat(inputs.structured("qm1", primes, n), 3, axis=0)          # same batch as x
+    assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes)), (ver, logn)
+    # the pointwise-product inverse (row f1) through the same kernel generation
+    a2 = to_dev(x)
+    o = torch.empty_like(a2)
+    plan.pointwise_inverse(a2, to_dev(q), o)
+    torch.cuda.synchronize()
+    prod = (x.astype(np.uint64) * q.astype(np.uint64)) % np.array(primes, np.uint64)[None, :, None]
+    assert np.array_equal(to_host(o), oracle.ntt_inverse(prod.astype(np.uint32), primes)), (ver, logn)
