@@ -21,6 +21,7 @@
 namespace wd {
 
 constexpr int FU_CC = 512, FU_TC = 128, FU_T = FU_CC + FU_TC;
+constexpr int FUP_TC = 256, FUP_T = FU_CC + FUP_TC;      // phase-split pipeline: 8 tensor warps
 constexpr int FU_CC_BAR = 2;
 constexpr int FU_SMEM = PGeo<16>::SMEM_BYTES + TC_SMEM + 64;
 constexpr int FUP_SMEM = PGeo<16>::SMEM_BYTES + TCC_SMEM + 64;
@@ -188,14 +189,14 @@ __device__ __forceinline__ void cc_row_phase2(const NttArgs& a, uint32_t* smem, 
 }
 
 template <bool FWD>
-__global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta) {
+__global__ void __launch_bounds__(FUP_T, 1) ntt_fused16_pipe(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta) {
     extern __shared__ __align__(1024) uint8_t fsm[];
     uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
     uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
     TccShared sh;
     sh.A0 = tcb;
-    sh.B = tcb + 3 * TC_TILE;
-    sh.bar = reinterpret_cast<uint64_t*>(tcb + 3 * TC_TILE + 17 * 4096);
+    sh.B = tcb + TCC_NBUF * TC_TILE;
+    sh.bar = reinterpret_cast<uint64_t*>(tcb + TCC_NBUF * TC_TILE + 17 * 4096);
     sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 4);
     uint32_t* loaded = sh.tslot + 1;
     int* ctl = reinterpret_cast<int*>(tcb + TCC_SMEM);          // [0] rows done by the leader, [1] by the follower
@@ -219,7 +220,7 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, const uin
     const bool is_tc = tid >= FU_CC;
     const bool leader = FWD ? is_tc : !is_tc;                    // who runs the first phase of a row
     const int gtid = is_tc ? tid - FU_CC : tid;
-    const int nthr = is_tc ? FU_TC : FU_CC;
+    const int nthr = is_tc ? FUP_TC : FU_CC;
     const int bar = is_tc ? TC_BAR_ID : FU_CC_BAR;
     int* mine = &ctl[leader ? 0 : 1];
     const int* other = &ctl[leader ? 1 : 0];
@@ -234,8 +235,8 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, const uin
         __threadfence_block();
         const uint32_t k = k0 + (uint32_t)i;
         const uint32_t limb = k / Bp, row = (k % Bp) * L + limb;
-        if (is_tc) tcc_columns<FWD, false>(ta, sh, tmem, ph, row, G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096,
-                                           loaded, TC_BAR_ID);
+        if (is_tc) tcc_columns<FWD, false, FUP_TC>(ta, sh, tmem, ph, row,
+                                                   G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096, loaded, TC_BAR_ID);
         else cc_row_phase2<FWD, FU_CC_BAR>(ta.a, ccbuf, row);
         __threadfence_block();
         named_bar(bar, nthr);
@@ -243,7 +244,7 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16_pipe(TcArgs ta, const uin
     }
     if (is_tc) {
         tc_fence_before();
-        named_bar(TC_BAR_ID, FU_TC);
+        named_bar(TC_BAR_ID, FUP_TC);
         if (gtid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem));
     }
 }
@@ -274,8 +275,8 @@ inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorT
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
     if (share > 1.5f || share < 0.0f) {   // default / tensor_share = 2: phase-split pipeline
         const uint32_t per = (rows + grid - 1) / grid;
-        if (fwd) ntt_fused16_pipe<true><<<grid, FU_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
-        else ntt_fused16_pipe<false><<<grid, FU_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
+        if (fwd) ntt_fused16_pipe<true><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
+        else ntt_fused16_pipe<false><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
         return 1;
     }
     if (fwd) ntt_fused16<true, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);

@@ -393,7 +393,8 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
 //            output = plain merged-CT intermediate (or pre-twisted by tau2 for the tensor P2).
 //   inverse (PH1' of the row): stage a = stage 1' (instance (c, i1), coeff j, p = 16 i1 + j,
 //            MI1_{i1}), stage b = stage 0' (instance (c, i0), coeff i1, p = i0 + 16 k, MI0).
-constexpr int TCC_SMEM = 3 * TC_TILE + 17 * 4096 + 64;     // stage-a A triple buffer + 17 B images
+constexpr int TCC_NBUF = 6;                                  // stage-a operand ring depth
+constexpr int TCC_SMEM = TCC_NBUF * TC_TILE + 17 * 4096 + 64;  // stage-a A ring + 17 B images
 constexpr uint32_t TCC_A1 = 0, TCC_D0 = 256, TCC_D1 = 384;
 
 struct TccShared { uint8_t* A0; uint8_t* B; uint64_t* bar; uint32_t* tslot; };
@@ -410,11 +411,16 @@ __device__ __forceinline__ void tc_mma_ts(uint32_t d, uint32_t a_tmem, uint64_t 
 
 // one row's column phase.  TWIST2 (forward only): pre-twist the output by tau2 for tc P2.
 // bar[0..1] stage-a accumulators, bar[2..3] stage-b accumulators; ph[4] their phases.
-template <bool FWD, bool TWIST2>
+// NT = 128: each warp owns TMEM lanes 32w..32w+31 and all 64 accumulator columns of a tile;
+// NT = 256: warps w and w+4 share lanes 32(w&3).. and split the columns (outputs k 0-7 / 8-15),
+// halving every epilogue.
+template <bool FWD, bool TWIST2, int NT = TC_T>
 __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& sh, uint32_t tmem, uint32_t* ph,
                                             uint32_t row_id, const uint8_t* Gl, uint32_t* loaded_limb, int bar_id) {
     const NttArgs& a = ta.a;
-    const int tid = threadIdx.x % TC_T, w = tid >> 5, lane = tid & 31;
+    const int tid = threadIdx.x % NT, w = tid >> 5, lane = tid & 31;
+    const int wq = w & 3;                        // TMEM lane quarter
+    const int h0 = NT == 256 ? (w >> 2) : 0;     // first accumulator half handled by this warp
     const uint32_t limb = row_id % a.L;
     const LimbConst lc = a.lc[limb];
     const uint32_t q = lc.q, q2 = lc.q2;
@@ -423,14 +429,14 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
     const uint32_t* src = FWD ? a.in + ((size_t)row_id << 16) : a.out + ((size_t)row_id << 16);
     uint32_t* out = a.out + ((size_t)row_id << 16);
     const uint2* T2 = ta.t2 + (size_t)limb * 4096;
-    const uint32_t lane_base = (uint32_t)(32 * w) << 16;
+    const uint32_t lane_base = (uint32_t)(32 * wq) << 16;
     if (*loaded_limb != limb) {                  // 17 B images of this limb (68 KB), once per limb
-        named_bar(bar_id, TC_T);
-        for (int i = tid; i < 17 * 4096 / 16; i += TC_T) cp_async16(sh.B + 16 * i, Gl + 16 * i);
+        named_bar(bar_id, NT);
+        for (int i = tid; i < 17 * 4096 / 16; i += NT) cp_async16(sh.B + 16 * i, Gl + 16 * i);
         cp_async_commit();
         cp_async_wait<0>();
         fence_async_smem();
-        named_bar(bar_id, TC_T);
+        named_bar(bar_id, NT);
         if (tid == 0) *loaded_limb = limb;
     }
     const uint32_t b_single = smem_addr(sh.B);
@@ -438,38 +444,40 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
     // stage-a tile t loader: element (coefficient j, row m) at p = FWD ? t + 16 j : 16 t + j
     auto load_a = [&](int t, int c0, uint8_t* buf) {
 #pragma unroll
-        for (int mq = 0; mq < 4; ++mq)
+        for (int mq = 0; mq < 16 / (NT / 32); ++mq)
 #pragma unroll
             for (int jh = 0; jh < 4; ++jh) {
-                const int mh = w + 4 * mq, m = 8 * mh + (lane & 7), j = 4 * jh + (lane >> 3);
+                const int mh = w + (NT / 32) * mq, m = 8 * mh + (lane & 7), j = 4 * jh + (lane >> 3);
                 const int p = FWD ? t + 16 * j : 16 * t + j;
                 cp_async4(buf + (lane & 7) * 16 + mh * 512 + jh * 128 + (lane >> 3) * 4, src + p * 256 + c0 + m);
             }
         cp_async_commit();
     };
+    // Stage-a operand ring of NB = TCC_NBUF tiles: tile te+NB is loaded into the buffer of tile
+    // te right after epilogue te has seen MMA te complete; the first NB tiles of a chunk are
+    // loaded while the previous chunk's stage b runs (or up front for the first chunk).  At the
+    // top of iteration t the issued tiles are 0 .. t+NB-2, so <= NB-2 groups may stay pending.
+    constexpr int NB = TCC_NBUF;
+    for (int t = 0; t < NB; ++t) load_a(t, 0, sh.A0 + t * TC_TILE);
 #pragma unroll 1
     for (int c0 = 0; c0 < 256; c0 += 128) {
         // ---------------- stage a: 16 tiles, A from smem, outputs -> TMEM stage-b operand tiles
-        // triple-buffered A: the load of tile t+1 overwrites the buffer of tile t-2, whose MMA
-        // completion was awaited by epilogue t-2 in the previous iteration
-        load_a(0, c0, sh.A0);
 #pragma unroll 1
         for (int t = 0; t <= 16; ++t) {
             if (t < 16) {
-                cp_async_wait<0>();
+                if (t + NB - 2 <= 15) cp_async_wait<NB - 2>(); else cp_async_wait<0>();
                 fence_async_smem();
                 tc_fence_before();
-                named_bar(bar_id, TC_T);
+                named_bar(bar_id, NT);
                 if (tid == 0) {
                     tc_fence_after();
-                    const uint32_t ab = smem_addr(sh.A0 + (t % 3) * TC_TILE);
+                    const uint32_t ab = smem_addr(sh.A0 + (t % NB) * TC_TILE);
                     const uint32_t bb = FWD ? b_single : b_group(t);
                     const uint32_t d = tmem + TCC_D0 + (t & 1) * 64;
                     tc_mma(d, umma_desc(ab), umma_desc(bb), 0);
                     tc_mma(d, umma_desc(ab + 256), umma_desc(bb + 256), 1);
                     tc_commit(&sh.bar[t & 1]);
                 }
-                if (t + 1 < 16) load_a(t + 1, c0, sh.A0 + ((t + 1) % 3) * TC_TILE);
             }
             if (t >= 1) {                             // epilogue of tile t-1
                 const int te = t - 1, r = te & 1;
@@ -478,7 +486,8 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
                 tc_fence_after();
                 uint32_t d[32];
 #pragma unroll
-                for (int hf = 0; hf < 2; ++hf) {
+                for (int hh = 0; hh < (NT == 256 ? 1 : 2); ++hh) {
+                    const int hf = h0 + hh;
                     tmem_ld32(tmem + lane_base + TCC_D0 + r * 64 + 32 * hf, d);
                     tmem_wait_ld();
 #pragma unroll
@@ -487,11 +496,14 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
                         tmem_st1(tmem + lane_base + TCC_A1 + 16 * k + te, combine(d + 4 * kk, q, c16s));
                     }
                 }
+                if (te + NB <= 15) load_a(te + NB, c0, sh.A0 + (te % NB) * TC_TILE);   // MMA te is done
             }
         }
+        if (c0 == 0)                                  // next chunk's first tiles overlap this stage b
+            for (int t = 0; t < NB; ++t) load_a(t, 128, sh.A0 + t * TC_TILE);
         tmem_wait_st();
         tc_fence_before();
-        named_bar(bar_id, TC_T);
+        named_bar(bar_id, NT);
         // ---------------- stage b: 16 tiles, A from TMEM, outputs -> global
 #pragma unroll 1
         for (int k = 0; k <= 16; ++k) {
@@ -509,9 +521,10 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
                 ph[2 + r] ^= 1;
                 tc_fence_after();
                 uint32_t d[32];
-                const int m = 32 * w + lane;
+                const int m = 32 * wq + lane;
 #pragma unroll
-                for (int hf = 0; hf < 2; ++hf) {
+                for (int hh = 0; hh < (NT == 256 ? 1 : 2); ++hh) {
+                    const int hf = h0 + hh;
                     tmem_ld32(tmem + lane_base + TCC_D1 + r * 64 + 32 * hf, d);
                     tmem_wait_ld();
 #pragma unroll
@@ -535,7 +548,7 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
                 }
                 tc_fence_before();
             }
-            named_bar(bar_id, TC_T);                      // D1 region of tile k-1 free for tile k+1
+            named_bar(bar_id, NT);                        // D1 region of tile k-1 free for tile k+1
         }
     }
     (void)q2;
@@ -547,8 +560,8 @@ __global__ void __launch_bounds__(TC_T, 1) ntt_tcc16(TcArgs ta, const uint8_t* G
     extern __shared__ __align__(1024) uint8_t tsm[];
     TccShared sh;
     sh.A0 = tsm;
-    sh.B = tsm + 3 * TC_TILE;
-    sh.bar = reinterpret_cast<uint64_t*>(tsm + 3 * TC_TILE + 17 * 4096);
+    sh.B = tsm + TCC_NBUF * TC_TILE;
+    sh.bar = reinterpret_cast<uint64_t*>(tsm + TCC_NBUF * TC_TILE + 17 * 4096);
     sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 4);
     uint32_t* loaded = sh.tslot + 1;
     const int tid = threadIdx.x;
