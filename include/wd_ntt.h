@@ -134,9 +134,11 @@ uint32_t wd_ntt_plan_psi(const wd_ntt_plan* plan, uint32_t limb);
 uint32_t wd_ntt_root(uint32_t q, uint32_t N);
 int      wd_ntt_check_prime(uint32_t q, uint32_t N);
 
-/* Select the execution path.  tensor_share in [0,1] is the fraction of
- * transform tiles given to the tensor path in WD_MODE_FUSED (ignored
- * otherwise; < 0 keeps the plan's measured default).  Returns WD_OK,
+/* Select the execution path.  tensor_share in [0,1] is, in WD_MODE_FUSED,
+ * the fraction of rows whose column phase runs on the tensor-core warps
+ * while the CUDA-core warps run the row phase (the rest of the rows run
+ * entirely on the CUDA-core warps).  Ignored otherwise; < 0
+ * keeps the plan's measured default.  Returns WD_OK,
  * WD_EINVAL or WD_EUNSUPPORTED.  Not thread-safe against concurrent calls
  * using the same plan. */
 int wd_ntt_plan_set_mode(wd_ntt_plan* plan, int mode, float tensor_share);

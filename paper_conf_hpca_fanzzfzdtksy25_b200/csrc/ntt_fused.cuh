@@ -16,6 +16,8 @@
 // tensor_share is given (0..1), rows are instead assigned statically:
 // row index i of the CTA goes to the tensor group iff frac(i*share) < share.
 #pragma once
+#include <cstdlib>
+#include <cstring>
 #include "ntt_tensor.cuh"
 
 namespace wd {
@@ -156,6 +158,8 @@ __global__ void __launch_bounds__(FU_T, 1) ntt_fused16(TcArgs ta, uint32_t rows,
 // CUDA-core group leads (P2' first), the tensor group finishes each row with P1'.
 // The leader stays at most FU_LEAD rows ahead, bounding the in-flight intermediates.
 constexpr int FU_LEAD = 2;
+// measured default tensor share of the pipeline (scripts/gpu_sweep.sh)
+constexpr float FUSED_DEFAULT_SHARE = 1.0f;
 
 __device__ __forceinline__ int ld_volatile(const int* p) { return *reinterpret_cast<const volatile int*>(p); }
 
@@ -189,7 +193,12 @@ __device__ __forceinline__ void cc_row_phase2(const NttArgs& a, uint32_t* smem, 
 }
 
 template <bool FWD>
-__global__ void __launch_bounds__(FUP_T, 1) ntt_fused16_pipe(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta) {
+// solo: 0 normal; 1 / 2 = DIAGNOSTIC ONLY (WD_NTT_PIPE_SOLO): only the tensor / CUDA-core group
+// computes, the other just passes rows on -- results are wrong, the time is one side's throughput.
+// share: fraction of rows whose column phase runs on the tensor warps (interleaved); the
+// CUDA-core warps run the remaining rows whole (the paper's tensor/CUDA ratio knob).
+__global__ void __launch_bounds__(FUP_T, 1) ntt_fused16_pipe(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta,
+                                                             int solo, float share, int lead) {
     extern __shared__ __align__(1024) uint8_t fsm[];
     uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
     uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
@@ -228,16 +237,22 @@ __global__ void __launch_bounds__(FUP_T, 1) ntt_fused16_pipe(TcArgs ta, const ui
     uint32_t ph[4] = {0, 0, 0, 0};
     for (int i = 0; i < nmine; ++i) {
         if (gtid == 0) {
-            if (leader) { while (i - ld_volatile(other) >= FU_LEAD) __nanosleep(256); }
+            if (leader) { while (i - ld_volatile(other) >= lead) __nanosleep(256); }
             else { while (ld_volatile(other) <= i) __nanosleep(128); }
         }
         named_bar(bar, nthr);
         __threadfence_block();
         const uint32_t k = k0 + (uint32_t)i;
         const uint32_t limb = k / Bp, row = (k % Bp) * L + limb;
-        if (is_tc) tcc_columns<FWD, false, FUP_TC>(ta, sh, tmem, ph, row,
-                                                   G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096, loaded, TC_BAR_ID);
-        else cc_row_phase2<FWD, FU_CC_BAR>(ta.a, ccbuf, row);
+        const bool tc_row = floorf((float)(i + 1) * share) > floorf((float)i * share);
+        if (is_tc) {
+            if (solo != 2 && tc_row)
+                tcc_columns<FWD, false, FUP_TC>(ta, sh, tmem, ph, row, G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096,
+                                                loaded, TC_BAR_ID);
+        } else if (solo != 1) {
+            if (tc_row) cc_row_phase2<FWD, FU_CC_BAR>(ta.a, ccbuf, row);
+            else cc_row<FWD, false, FU_CC_BAR>(ta.a, ccbuf, row);
+        }
         __threadfence_block();
         named_bar(bar, nthr);
         if (gtid == 0) atomicExch(mine, i + 1);
@@ -273,10 +288,14 @@ inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorT
     ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
     ta.c16 = tc.d_c16;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
-    if (share > 1.5f || share < 0.0f) {   // default / tensor_share = 2: phase-split pipeline
+    static const char* variant = getenv("WD_NTT_FUSED");          // "rows": whole-row split kernel (A/B runs)
+    if (!(variant && strcmp(variant, "rows") == 0)) {              // phase-split pipeline (default)
         const uint32_t per = (rows + grid - 1) / grid;
-        if (fwd) ntt_fused16_pipe<true><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
-        else ntt_fused16_pipe<false><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per);
+        static const int solo = getenv("WD_NTT_PIPE_SOLO") ? atoi(getenv("WD_NTT_PIPE_SOLO")) : 0;
+        static const int lead = getenv("WD_NTT_PIPE_LEAD") ? std::max(1, atoi(getenv("WD_NTT_PIPE_LEAD"))) : FU_LEAD;
+        const float sh = share < 0.0f ? FUSED_DEFAULT_SHARE : share;
+        if (fwd) ntt_fused16_pipe<true><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per, solo, sh, lead);
+        else ntt_fused16_pipe<false><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per, solo, sh, lead);
         return 1;
     }
     if (fwd) ntt_fused16<true, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);

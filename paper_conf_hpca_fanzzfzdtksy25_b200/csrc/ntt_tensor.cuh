@@ -395,7 +395,7 @@ __device__ __forceinline__ void tc_transform(const TcArgs& ta, const TcShared& s
 //            MI1_{i1}), stage b = stage 0' (instance (c, i0), coeff i1, p = i0 + 16 k, MI0).
 constexpr int TCC_NBUF = 6;                                  // stage-a operand ring depth
 constexpr int TCC_SMEM = TCC_NBUF * TC_TILE + 17 * 4096 + 64;  // stage-a A ring + 17 B images
-constexpr uint32_t TCC_A1 = 0, TCC_D0 = 256, TCC_D1 = 384;
+constexpr uint32_t TCC_A1 = 0, TCC_D0 = 256;          // D pool: 4 regions x 64 columns
 
 struct TccShared { uint8_t* A0; uint8_t* B; uint64_t* bar; uint32_t* tslot; };
 
@@ -453,51 +453,67 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
             }
         cp_async_commit();
     };
-    // Stage-a operand ring of NB = TCC_NBUF tiles: tile te+NB is loaded into the buffer of tile
-    // te right after epilogue te has seen MMA te complete; the first NB tiles of a chunk are
-    // loaded while the previous chunk's stage b runs (or up front for the first chunk).  At the
-    // top of iteration t the issued tiles are 0 .. t+NB-2, so <= NB-2 groups may stay pending.
+    // Both stages run as a distance-3 software pipeline over a pool of 4 TMEM accumulator
+    // regions (cols [256,512), region = tile & 3, mbarrier bar[region]): iteration t first makes
+    // sure operand tile t+3 is ready, issues MMA(t+3) into the region freed by epilogue t-1, then
+    // runs epilogue t.  Stage-a operands come through a ring of NB shared-memory tiles; tile t+NB
+    // is loaded into the buffer of tile t once epilogue t has seen MMA t complete.  At the top of
+    // iteration t the issued stage-a tiles are 0 .. t+NB-1, so <= NB-4 groups may stay pending.
     constexpr int NB = TCC_NBUF;
+    constexpr int PD = 3;                                  // MMA issue distance
+    auto issue_a = [&](int t) {
+        const uint32_t ab = smem_addr(sh.A0 + (t % NB) * TC_TILE);
+        const uint32_t bb = FWD ? b_single : b_group(t);
+        const uint32_t d = tmem + TCC_D0 + (t & 3) * 64;
+        tc_fence_after();
+        tc_mma(d, umma_desc(ab), umma_desc(bb), 0);
+        tc_mma(d, umma_desc(ab + 256), umma_desc(bb + 256), 1);
+        tc_commit(&sh.bar[t & 3]);
+    };
+    auto issue_b = [&](int k) {
+        const uint32_t bb = FWD ? b_group(k) : b_single;
+        const uint32_t d = tmem + TCC_D0 + (k & 3) * 64;
+        tc_fence_after();
+        tc_mma_ts(d, tmem + TCC_A1 + 16 * k, umma_desc(bb), 0);
+        tc_mma_ts(d, tmem + TCC_A1 + 16 * k + 8, umma_desc(bb + 256), 1);
+        tc_commit(&sh.bar[k & 3]);
+    };
     for (int t = 0; t < NB; ++t) load_a(t, 0, sh.A0 + t * TC_TILE);
 #pragma unroll 1
     for (int c0 = 0; c0 < 256; c0 += 128) {
         // ---------------- stage a: 16 tiles, A from smem, outputs -> TMEM stage-b operand tiles
+        cp_async_wait<NB - PD>();                     // tiles 0..PD-1 landed
+        fence_async_smem();
+        tc_fence_before();
+        named_bar(bar_id, NT);
+        if (tid == 0) for (int t = 0; t < PD; ++t) issue_a(t);
 #pragma unroll 1
-        for (int t = 0; t <= 16; ++t) {
-            if (t < 16) {
-                if (t + NB - 2 <= 15) cp_async_wait<NB - 2>(); else cp_async_wait<0>();
+        for (int t = 0; t < 16; ++t) {
+            const int tn = t + PD;                    // tile whose MMA is issued in this iteration
+            if (tn < 16) {
+                if (t + NB - 1 <= 15) cp_async_wait<NB - PD - 1>(); else cp_async_wait<0>();
                 fence_async_smem();
-                tc_fence_before();
-                named_bar(bar_id, NT);
-                if (tid == 0) {
-                    tc_fence_after();
-                    const uint32_t ab = smem_addr(sh.A0 + (t % NB) * TC_TILE);
-                    const uint32_t bb = FWD ? b_single : b_group(t);
-                    const uint32_t d = tmem + TCC_D0 + (t & 1) * 64;
-                    tc_mma(d, umma_desc(ab), umma_desc(bb), 0);
-                    tc_mma(d, umma_desc(ab + 256), umma_desc(bb + 256), 1);
-                    tc_commit(&sh.bar[t & 1]);
+            }
+            tc_fence_before();
+            named_bar(bar_id, NT);                    // operand tile tn visible; epilogue t-1 done with its region
+            if (tid == 0 && tn < 16) issue_a(tn);
+            const int r = t & 3;
+            mbar_wait(&sh.bar[r], (ph[0] >> r) & 1);
+            ph[0] ^= 1u << r;
+            tc_fence_after();
+            uint32_t d[32];
+#pragma unroll
+            for (int hh = 0; hh < (NT == 256 ? 1 : 2); ++hh) {
+                const int hf = h0 + hh;
+                tmem_ld32(tmem + lane_base + TCC_D0 + r * 64 + 32 * hf, d);
+                tmem_wait_ld();
+#pragma unroll
+                for (int kk = 0; kk < 8; ++kk) {
+                    const int k = 8 * hf + kk;
+                    tmem_st1(tmem + lane_base + TCC_A1 + 16 * k + t, combine(d + 4 * kk, q, c16s));
                 }
             }
-            if (t >= 1) {                             // epilogue of tile t-1
-                const int te = t - 1, r = te & 1;
-                mbar_wait(&sh.bar[r], ph[r]);
-                ph[r] ^= 1;
-                tc_fence_after();
-                uint32_t d[32];
-#pragma unroll
-                for (int hh = 0; hh < (NT == 256 ? 1 : 2); ++hh) {
-                    const int hf = h0 + hh;
-                    tmem_ld32(tmem + lane_base + TCC_D0 + r * 64 + 32 * hf, d);
-                    tmem_wait_ld();
-#pragma unroll
-                    for (int kk = 0; kk < 8; ++kk) {
-                        const int k = 8 * hf + kk;
-                        tmem_st1(tmem + lane_base + TCC_A1 + 16 * k + te, combine(d + 4 * kk, q, c16s));
-                    }
-                }
-                if (te + NB <= 15) load_a(te + NB, c0, sh.A0 + (te % NB) * TC_TILE);   // MMA te is done
-            }
+            if (t + NB <= 15) load_a(t + NB, c0, sh.A0 + (t % NB) * TC_TILE);   // MMA t is done
         }
         if (c0 == 0)                                  // next chunk's first tiles overlap this stage b
             for (int t = 0; t < NB; ++t) load_a(t, 128, sh.A0 + t * TC_TILE);
@@ -505,51 +521,45 @@ __device__ __forceinline__ void tcc_columns(const TcArgs& ta, const TccShared& s
         tc_fence_before();
         named_bar(bar_id, NT);
         // ---------------- stage b: 16 tiles, A from TMEM, outputs -> global
+        if (tid == 0) for (int k = 0; k < PD; ++k) issue_b(k);
 #pragma unroll 1
-        for (int k = 0; k <= 16; ++k) {
-            if (k < 16 && tid == 0) {
-                tc_fence_after();
-                const uint32_t bb = FWD ? b_group(k) : b_single;
-                const uint32_t d = tmem + TCC_D1 + (k & 1) * 64;
-                tc_mma_ts(d, tmem + TCC_A1 + 16 * k, umma_desc(bb), 0);
-                tc_mma_ts(d, tmem + TCC_A1 + 16 * k + 8, umma_desc(bb + 256), 1);
-                tc_commit(&sh.bar[2 + (k & 1)]);
-            }
-            if (k >= 1) {
-                const int ke = k - 1, r = ke & 1;
-                mbar_wait(&sh.bar[2 + r], ph[2 + r]);
-                ph[2 + r] ^= 1;
-                tc_fence_after();
-                uint32_t d[32];
-                const int m = 32 * wq + lane;
+        for (int k = 0; k < 16; ++k) {
+            const int kn = k + PD;
+            if (k > 0) { tc_fence_before(); named_bar(bar_id, NT); }   // epilogue k-1 done with region (k+3)&3
+            if (tid == 0 && kn < 16) issue_b(kn);
+            const int r = k & 3;
+            mbar_wait(&sh.bar[r], (ph[0] >> r) & 1);
+            ph[0] ^= 1u << r;
+            tc_fence_after();
+            uint32_t d[32];
+            const int m = 32 * wq + lane;
 #pragma unroll
-                for (int hh = 0; hh < (NT == 256 ? 1 : 2); ++hh) {
-                    const int hf = h0 + hh;
-                    tmem_ld32(tmem + lane_base + TCC_D1 + r * 64 + 32 * hf, d);
-                    tmem_wait_ld();
+            for (int hh = 0; hh < (NT == 256 ? 1 : 2); ++hh) {
+                const int hf = h0 + hh;
+                tmem_ld32(tmem + lane_base + TCC_D0 + r * 64 + 32 * hf, d);
+                tmem_wait_ld();
 #pragma unroll
-                    for (int kk = 0; kk < 8; ++kk) {
-                        const int ko = 8 * hf + kk;
-                        const int p = FWD ? 16 * ke + ko : ke + 16 * ko;
-                        uint32_t y = combine(d + 4 * kk, q, c16s);
-                        if (FWD) {
-                            if (TWIST2) {
-                                const uint2 tw = __ldg(T2 + p * 16 + ((c0 + m) >> 4));
-                                y = shoup_mul(y, tw.x, tw.y, q);
-                            } else {
-                                y = shoup_mul(y, 1u, one_s, q);                  // [0, 2q) for the butterflies
-                            }
-                            out[p * 256 + c0 + m] = y;
+                for (int kk = 0; kk < 8; ++kk) {
+                    const int ko = 8 * hf + kk;
+                    const int p = FWD ? 16 * k + ko : k + 16 * ko;
+                    uint32_t y = combine(d + 4 * kk, q, c16s);
+                    if (FWD) {
+                        if (TWIST2) {
+                            const uint2 tw = __ldg(T2 + p * 16 + ((c0 + m) >> 4));
+                            y = shoup_mul(y, tw.x, tw.y, q);
                         } else {
-                            y = shoup_mul(y, 1u, one_s, q);
-                            __stcs(out + p * 256 + c0 + m, umin32(y, y - q));
+                            y = shoup_mul(y, 1u, one_s, q);                  // [0, 2q) for the butterflies
                         }
+                        out[p * 256 + c0 + m] = y;
+                    } else {
+                        y = shoup_mul(y, 1u, one_s, q);
+                        __stcs(out + p * 256 + c0 + m, umin32(y, y - q));
                     }
                 }
-                tc_fence_before();
             }
-            named_bar(bar_id, NT);                        // D1 region of tile k-1 free for tile k+1
         }
+        tc_fence_before();
+        named_bar(bar_id, NT);                        // all stage-b epilogues done before A1 / D reuse
     }
     (void)q2;
 }

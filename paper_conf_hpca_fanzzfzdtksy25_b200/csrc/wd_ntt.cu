@@ -383,7 +383,7 @@ int wd_ntt_check_prime(uint32_t q, uint32_t N) {
 int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
     if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_FUSED) return set_err(WD_EINVAL);
     if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED) && !tensor_supported(p->logN)) return set_err(WD_EUNSUPPORTED);
-    if (tensor_share > 2.0f) return set_err(WD_EINVAL);
+    if (tensor_share > 1.0f) return set_err(WD_EINVAL);
     p->mode = mode;
     if (tensor_share >= 0.0f) p->tensor_share = tensor_share;
     return set_err(WD_OK);

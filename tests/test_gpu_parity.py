@@ -201,7 +201,7 @@ def _modes(wd):
     return ["cuda", "tensor", "fused"]
 
 
-MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.25), ("fused", 0.75)]
+MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.0), ("fused", 0.6)]
 
 
 @pytest.mark.parametrize("mode,share", MODES)
