@@ -40,9 +40,9 @@ template <> struct PCfg<15> { static constexpr int A0 = 4, A1 = 3; };
 template <> struct PCfg<16> { static constexpr int A0 = 4, A1 = 4; };
 template <> struct PCfg<17> { static constexpr int A0 = 5, A1 = 4; };
 
-template <int LOGN>
+template <int LOGN, int TT = 512>
 struct PGeo {
-    static constexpr int T = 512;
+    static constexpr int T = TT;
     static constexpr int A0 = PCfg<LOGN>::A0, A1 = PCfg<LOGN>::A1;
     static constexpr int B1 = LOGN - 8, N1 = 1 << B1;
     static constexpr int R0 = 1 << A0, R1 = 1 << A1;
@@ -63,9 +63,9 @@ struct PGeo {
 
 // ---- chunk loads (all T threads) --------------------------------------------------------
 // phase-1 chunk: columns [c0, c0+W1) of every one of the N1 256-word rows -> S[p*W1 + w]
-template <int LOGN>
+template <int LOGN, int TT = 512>
 __device__ __forceinline__ void load_p1(uint32_t* S, const uint32_t* src, int c0) {
-    using G = PGeo<LOGN>;
+    using G = PGeo<LOGN, TT>;
     constexpr int SEG = G::W1 / 4, NSEG = G::N1 * SEG;
     static_assert(NSEG % G::T == 0, "whole segments per thread");
 #pragma unroll
@@ -76,9 +76,9 @@ __device__ __forceinline__ void load_p1(uint32_t* S, const uint32_t* src, int c0
     }
 }
 // phase-2 chunk: rows [r0, r0+W2), 256 words each -> swizzled ywords() layout
-template <int LOGN>
+template <int LOGN, int TT = 512>
 __device__ __forceinline__ void load_p2(uint32_t* S, const uint32_t* src, int r0) {
-    using G = PGeo<LOGN>;
+    using G = PGeo<LOGN, TT>;
     constexpr int NSEG = G::W2 * 64;
     static_assert(NSEG % G::T == 0, "whole segments per thread");
 #pragma unroll
@@ -90,10 +90,10 @@ __device__ __forceinline__ void load_p2(uint32_t* S, const uint32_t* src, int r0
 }
 
 // ---- forward chunk compute ------------------------------------------------------------
-template <int LOGN, int BAR = 0>
+template <int LOGN, int BAR = 0, int TT = 512>
 __device__ __forceinline__ void fwd_p1_chunk(uint32_t* S, uint32_t* out, int c0, const uint2* __restrict__ tw,
                                              uint32_t q, uint32_t q2) {
-    using G = PGeo<LOGN>;
+    using G = PGeo<LOGN, TT>;
     const int w = threadIdx.x % G::W1, j = threadIdx.x / G::W1;
     uint32_t x[G::E1];
 #pragma unroll
@@ -157,10 +157,10 @@ __device__ __forceinline__ void inv16_tw(uint32_t* x, const uint2* w, uint32_t q
     }
 }
 
-template <int LOGN, int BAR = 0>
+template <int LOGN, int BAR = 0, int TT = 512>
 __device__ __forceinline__ void fwd_p2_chunk(uint32_t* S, uint32_t* out, int r0, const uint2* __restrict__ tw,
                                              uint32_t q, uint32_t q2) {
-    using G = PGeo<LOGN>;
+    using G = PGeo<LOGN, TT>;
     const int c = threadIdx.x & 15, w = threadIdx.x >> 4;
     const int row = r0 + w;
     uint32_t x[16];
@@ -186,10 +186,10 @@ __device__ __forceinline__ void fwd_p2_chunk(uint32_t* S, uint32_t* out, int r0,
 }
 
 // ---- inverse chunk compute (phase 2' then phase 1') ---------------------------------------
-template <int LOGN, bool PW, int BAR = 0>
+template <int LOGN, bool PW, int BAR = 0, int TT = 512>
 __device__ __forceinline__ void inv_p2_chunk(uint32_t* S, uint32_t* out, const uint32_t* in2, int r0,
                                              const uint2* __restrict__ tw, const LimbConst& lc) {
-    using G = PGeo<LOGN>;
+    using G = PGeo<LOGN, TT>;
     const int c = threadIdx.x & 15, w = threadIdx.x >> 4;
     const int row = r0 + w;
     uint32_t x[16];
@@ -222,10 +222,10 @@ __device__ __forceinline__ void inv_p2_chunk(uint32_t* S, uint32_t* out, const u
     for (int r = 0; r < 16; ++r) out[row * 256 + c + 16 * r] = x[r];
 }
 
-template <int LOGN, int BAR = 0>
+template <int LOGN, int BAR = 0, int TT = 512>
 __device__ __forceinline__ void inv_p1_chunk(uint32_t* S, uint32_t* out, int c0, const uint2* __restrict__ tw,
                                              const LimbConst& lc) {
-    using G = PGeo<LOGN>;
+    using G = PGeo<LOGN, TT>;
     const int w = threadIdx.x % G::W1, j = threadIdx.x / G::W1;
     uint32_t x[G::E1];
 #pragma unroll
@@ -254,9 +254,9 @@ __device__ __forceinline__ void inv_p1_chunk(uint32_t* S, uint32_t* out, int c0,
 // ---- the persistent kernel ---------------------------------------------------------------
 // chunk k of a row: forward  k <  C1 -> phase-1 chunk k (src = in),  else phase-2 chunk k-C1 (src = out)
 //                   inverse  k <  C2 -> phase-2' chunk k (src = in), else phase-1' chunk k-C2 (src = out)
-template <int LOGN, bool FWD, bool PW>
-__global__ void __launch_bounds__(512, 2) ntt_persist_cc(NttArgs a, uint32_t rows) {
-    using G = PGeo<LOGN>;
+template <int LOGN, bool FWD, bool PW, int TT = 512>
+__global__ void __launch_bounds__(TT, 1024 / TT) ntt_persist_cc(NttArgs a, uint32_t rows) {
+    using G = PGeo<LOGN, TT>;
     constexpr int CA = FWD ? G::C1 : G::C2;          // chunks of the first phase
     constexpr int CH = G::C1 + G::C2;
     extern __shared__ __align__(16) uint32_t smem[];
@@ -271,11 +271,11 @@ __global__ void __launch_bounds__(512, 2) ntt_persist_cc(NttArgs a, uint32_t row
         const uint32_t* in = a.in + ((size_t)row_id << LOGN);
         const uint32_t* mid = a.out + ((size_t)row_id << LOGN);
         if (FWD) {
-            if (kk < G::C1) load_p1<LOGN>(S, in, kk * G::W1);
-            else load_p2<LOGN>(S, mid, (kk - G::C1) * G::W2);
+            if (kk < G::C1) load_p1<LOGN, TT>(S, in, kk * G::W1);
+            else load_p2<LOGN, TT>(S, mid, (kk - G::C1) * G::W2);
         } else {
-            if (kk < G::C2) load_p2<LOGN>(S, in, kk * G::W2);
-            else load_p1<LOGN>(S, mid, (kk - G::C2) * G::W1);
+            if (kk < G::C2) load_p2<LOGN, TT>(S, in, kk * G::W2);
+            else load_p1<LOGN, TT>(S, mid, (kk - G::C2) * G::W1);
         }
         cp_async_commit();
     };
@@ -300,12 +300,12 @@ __global__ void __launch_bounds__(512, 2) ntt_persist_cc(NttArgs a, uint32_t row
         const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
         uint32_t* out = a.out + ((size_t)row_id << LOGN);
         if (FWD) {
-            if (kk < G::C1) fwd_p1_chunk<LOGN>(S, out, kk * G::W1, tw, lc.q, lc.q2);
-            else fwd_p2_chunk<LOGN>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
+            if (kk < G::C1) fwd_p1_chunk<LOGN, 0, TT>(S, out, kk * G::W1, tw, lc.q, lc.q2);
+            else fwd_p2_chunk<LOGN, 0, TT>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
         } else {
             const uint32_t* in2 = a.in2 + ((size_t)row_id << LOGN);
-            if (kk < G::C2) inv_p2_chunk<LOGN, PW>(S, out, in2, kk * G::W2, tw, lc);
-            else inv_p1_chunk<LOGN>(S, out, (kk - G::C2) * G::W1, tw, lc);
+            if (kk < G::C2) inv_p2_chunk<LOGN, PW, 0, TT>(S, out, in2, kk * G::W2, tw, lc);
+            else inv_p1_chunk<LOGN, 0, TT>(S, out, (kk - G::C2) * G::W1, tw, lc);
         }
         __threadfence_block();
         __syncthreads();

@@ -36,7 +36,8 @@ struct wd_ntt_plan {
     uint32_t N = 0, logN = 0, L = 0;
     int device = -1;
     int sm_count = 148;
-    int kernel_ver = 2;            // WD_NTT_KERNEL=v1|v2|v3 selects the CUDA-core kernel generation (A/B runs)
+    int kernel_ver = 0;            // 0 = measured default per N (v6 at 2^16, v2 at 2^15/2^17, v1 below);
+                                   // WD_NTT_KERNEL=v1|v2|v3|v5|v6 forces a generation (A/B runs)
     std::vector<uint32_t> primes, psi;
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
     uint2* d_inv = nullptr;        // [L][N]  (psi^-brv(i), Shoup)
@@ -100,6 +101,13 @@ int prep_cc() {
             set_smem(ntt_persist_cc<LOGN, false, true>, G::SMEM_BYTES))
             return WD_ECUDA;
     }
+    if constexpr (LOGN == 16) {
+        using G = PGeo<LOGN, 256>;
+        if (set_smem(ntt_persist_cc<LOGN, true, false, 256>, G::SMEM_BYTES) ||
+            set_smem(ntt_persist_cc<LOGN, false, false, 256>, G::SMEM_BYTES) ||
+            set_smem(ntt_persist_cc<LOGN, false, true, 256>, G::SMEM_BYTES))
+            return WD_ECUDA;
+    }
     return WD_OK;
 }
 
@@ -152,6 +160,16 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             if (fwd) cudaLaunchKernelEx(&cfg, ntt_fwd_smem<LOGN>, a, rows);
             else if (a.in2) cudaLaunchKernelEx(&cfg, ntt_inv_smem<LOGN, true>, a, rows);
             else cudaLaunchKernelEx(&cfg, ntt_inv_smem<LOGN, false>, a, rows);
+            return;
+        }
+    }
+    if constexpr (LOGN == 16) {
+        if (p->kernel_ver == 6) {             // v2 with 256-thread CTAs, 4 per SM
+            using G = PGeo<LOGN, 256>;
+            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * 4));
+            if (fwd) ntt_persist_cc<LOGN, true, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
+            else if (a.in2) ntt_persist_cc<LOGN, false, true, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
+            else ntt_persist_cc<LOGN, false, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
             return;
         }
     }
@@ -317,7 +335,8 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     // ---- device upload (the only H2D copy of the plan's life)
     if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
     cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
-    if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : 2;
+    p->kernel_ver = p->logN == 16 ? 6 : 2;
+    if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
         cudaMalloc(&p->d_lc, sizeof(LimbConst) * L) != cudaSuccess) {
