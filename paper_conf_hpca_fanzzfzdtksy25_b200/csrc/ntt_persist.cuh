@@ -260,14 +260,11 @@ __global__ void __launch_bounds__(TT, 1024 / TT) ntt_persist_cc(NttArgs a, uint3
     constexpr int CA = FWD ? G::C1 : G::C2;          // chunks of the first phase
     constexpr int CH = G::C1 + G::C2;
     extern __shared__ __align__(16) uint32_t smem[];
+    if (blockIdx.x >= rows) return;
 
-    const uint32_t nmine = rows > blockIdx.x ? (rows - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-    const uint32_t total = nmine * CH;
-    if (total == 0) return;
-
-    auto issue = [&](uint32_t k, uint32_t* S) {
-        const uint32_t row_id = blockIdx.x + (k / CH) * gridDim.x;
-        const int kk = k % CH;
+    // row-outer / chunk-inner: per-row constants (limb, LimbConst, pointers) are computed once
+    // per row, and the next row's LimbConst is fetched one row ahead
+    auto issue = [&](uint32_t row_id, int kk, uint32_t* S) {
         const uint32_t* in = a.in + ((size_t)row_id << LOGN);
         const uint32_t* mid = a.out + ((size_t)row_id << LOGN);
         if (FWD) {
@@ -279,37 +276,46 @@ __global__ void __launch_bounds__(TT, 1024 / TT) ntt_persist_cc(NttArgs a, uint3
         }
         cp_async_commit();
     };
-
-    issue(0, smem);
-    for (uint32_t k = 0; k < total; ++k) {
-        uint32_t* S = smem + (k & 1) * G::BUF_WORDS;
-        const int kk = k % CH;
-        // chunk k+1 may be the first chunk of phase B of this row: it reads what this chunk writes
-        const bool dep = (k + 1 < total) && ((k + 1) % CH == (uint32_t)CA);
-        if (k + 1 < total && !dep) {
-            issue(k + 1, smem + ((k + 1) & 1) * G::BUF_WORDS);
-            cp_async_wait<1>();
-        } else {
-            cp_async_wait<0>();
-        }
-        __syncthreads();
-
-        const uint32_t row_id = blockIdx.x + (k / CH) * gridDim.x;
+    uint32_t row_id = blockIdx.x;
+    LimbConst lc = a.lc[row_id % a.L];
+    uint32_t buf = 0;
+    issue(row_id, 0, smem);
+#pragma unroll 1
+    while (row_id < rows) {
+        const uint32_t next = row_id + gridDim.x;
         const uint32_t limb = row_id % a.L;
-        const LimbConst lc = a.lc[limb];
+        const LimbConst lcn = a.lc[(next < rows ? next : row_id) % a.L];    // in flight during this row
         const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
         uint32_t* out = a.out + ((size_t)row_id << LOGN);
-        if (FWD) {
-            if (kk < G::C1) fwd_p1_chunk<LOGN, 0, TT>(S, out, kk * G::W1, tw, lc.q, lc.q2);
-            else fwd_p2_chunk<LOGN, 0, TT>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
-        } else {
-            const uint32_t* in2 = a.in2 + ((size_t)row_id << LOGN);
-            if (kk < G::C2) inv_p2_chunk<LOGN, PW, 0, TT>(S, out, in2, kk * G::W2, tw, lc);
-            else inv_p1_chunk<LOGN, 0, TT>(S, out, (kk - G::C2) * G::W1, tw, lc);
+        const uint32_t* in2 = a.in2 + ((size_t)row_id << LOGN);
+#pragma unroll 1
+        for (int kk = 0; kk < CH; ++kk, buf ^= 1) {
+            uint32_t* S = smem + buf * G::BUF_WORDS;
+            uint32_t* Sn = smem + (buf ^ 1) * G::BUF_WORDS;
+            // chunk kk+1 may be the first chunk of phase B of this row: it reads what this chunk writes
+            const bool dep = (kk + 1 == CA);
+            const bool more = kk + 1 < CH || next < rows;
+            if (more && !dep) {
+                if (kk + 1 < CH) issue(row_id, kk + 1, Sn);
+                else issue(next, 0, Sn);
+                cp_async_wait<1>();
+            } else {
+                cp_async_wait<0>();
+            }
+            __syncthreads();
+            if (FWD) {
+                if (kk < G::C1) fwd_p1_chunk<LOGN, 0, TT>(S, out, kk * G::W1, tw, lc.q, lc.q2);
+                else fwd_p2_chunk<LOGN, 0, TT>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
+            } else {
+                if (kk < G::C2) inv_p2_chunk<LOGN, PW, 0, TT>(S, out, in2, kk * G::W2, tw, lc);
+                else inv_p1_chunk<LOGN, 0, TT>(S, out, (kk - G::C2) * G::W1, tw, lc);
+            }
+            __threadfence_block();
+            __syncthreads();
+            if (dep) issue(row_id, kk + 1, Sn);
         }
-        __threadfence_block();
-        __syncthreads();
-        if (dep) issue(k + 1, smem + ((k + 1) & 1) * G::BUF_WORDS);
+        lc = lcn;
+        row_id = next;
     }
 }
 

@@ -36,6 +36,7 @@ struct wd_ntt_plan {
     uint32_t N = 0, logN = 0, L = 0;
     int device = -1;
     int sm_count = 148;
+    int v6_ctas = 4;               // resident 256-thread CTAs per SM for v6 (WD_NTT_CTAS: 2..4, A/B runs)
     int kernel_ver = 0;            // 0 = measured default per N (v6 at 2^16, v2 at 2^15/2^17, v1 below);
                                    // WD_NTT_KERNEL=v1|v2|v3|v5|v6 forces a generation (A/B runs)
     std::vector<uint32_t> primes, psi;
@@ -166,7 +167,7 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
     if constexpr (LOGN == 16) {
         if (p->kernel_ver == 6) {             // v2 with 256-thread CTAs, 4 per SM
             using G = PGeo<LOGN, 256>;
-            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * 4));
+            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * p->v6_ctas));
             if (fwd) ntt_persist_cc<LOGN, true, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
             else if (a.in2) ntt_persist_cc<LOGN, false, true, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
             else ntt_persist_cc<LOGN, false, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
@@ -336,6 +337,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
     cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
     p->kernel_ver = p->logN == 16 ? 6 : 2;
+    if (const char* ev = getenv("WD_NTT_CTAS")) p->v6_ctas = std::max(1, std::min(4, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||

@@ -3,7 +3,7 @@ cd "$GRAFT_REPO_ROOT" 2>/dev/null || cd /root/repo
 TAG=$1
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build_$TAG.log 2>&1
-timeout 900 python -m pytest tests -m gpu -q -k "generations and v6" > gpurun_out/pytest_$TAG.log 2>&1
+timeout 900 python -m pytest tests -m gpu -q -k "generations and (v6 or v2) or config3 or in_place or pointwise" > gpurun_out/pytest_$TAG.log 2>&1
 for v in v2 v6; do
   WD_NTT_KERNEL=$v timeout 300 python bench.py --steps 20 --warmup 3 --e2e-steps 0 --no-cpu --mode cuda > gpurun_out/bench_${TAG}_$v.json 2> gpurun_out/bench_${TAG}_$v.err
 done
