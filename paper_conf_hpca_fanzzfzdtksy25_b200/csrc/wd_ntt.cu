@@ -132,7 +132,10 @@ template <int LOGN>
 void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     using S = CcShape<LOGN>;
     if constexpr (LOGN >= 14) {
-        if (p->kernel_ver == 5) {
+        // measured: a row split over a CTA cluster wins when there are fewer rows than SMs
+        // (config 2: one ciphertext = 72 rows -> 1648 vs 1010 KOPS); one row per CTA wins above
+        const bool small = p->kernel_ver == 0 && rows < (uint32_t)p->sm_count && (LOGN == 15 || LOGN == 16);
+        if (p->kernel_ver == 5 || small) {
             constexpr int CLN = 1 << (LOGN - 14);
             const uint32_t units = std::max<uint32_t>(1, std::min<uint32_t>(rows, (uint32_t)(2 * p->sm_count / CLN)));
             cudaLaunchConfig_t cfg = {};
@@ -165,7 +168,7 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         }
     }
     if constexpr (LOGN == 16) {
-        if (p->kernel_ver == 6) {             // v2 with 256-thread CTAs, 4 per SM
+        if (p->kernel_ver == 6 || p->kernel_ver == 0) {   // v2 with 256-thread CTAs, 4 per SM
             using G = PGeo<LOGN, 256>;
             const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * p->v6_ctas));
             if (fwd) ntt_persist_cc<LOGN, true, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
@@ -336,7 +339,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     // ---- device upload (the only H2D copy of the plan's life)
     if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
     cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
-    p->kernel_ver = p->logN == 16 ? 6 : 2;
+    p->kernel_ver = p->logN == 16 ? 0 : 2;          // 0 = AUTO at 2^16: v5 for < SM-count rows, else v6
     if (const char* ev = getenv("WD_NTT_CTAS")) p->v6_ctas = std::max(1, std::min(4, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
