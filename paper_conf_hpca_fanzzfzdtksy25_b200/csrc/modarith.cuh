@@ -76,49 +76,86 @@ __device__ __forceinline__ uint32_t canon2(uint32_t v, uint32_t q) {            
 // Psi[2^(ls+t) + (hi << t) + (r >> (K-t))], hi = g0 >> (logN - ls) (the
 // group index of the block at its first layer).  Same index rule as the
 // textbook merged-psi loop, restricted to one block.
+// One CT layer t (t >= 1) of a radix-2^K block: 2^t twiddle groups, the twiddle
+// pairs of adjacent groups fetched as one 16-byte vector.  A template per layer
+// (instead of a nested runtime-bounded loop) so NVVM always fully unrolls and x[]
+// stays in registers even at K = 5.
+template <int K, int t>
+__device__ __forceinline__ void fwd_layer(uint32_t* x, const uint2* __restrict__ tw, int ls,
+                                          uint32_t hi, uint32_t q, uint32_t q2) {
+    constexpr int h = 1 << (K - 1 - t);
+    const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
+#pragma unroll
+    for (int g = 0; g < (1 << t); g += 2) {
+        const uint4 v = __ldg(tp + g / 2);
+        const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
+#pragma unroll
+        for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], wa, q, q2);
+#pragma unroll
+        for (int r = 0; r < h; ++r) ct_bfly(x[2 * (g + 1) * h + r], x[2 * (g + 1) * h + r + h], wb, q, q2);
+    }
+    if constexpr (t + 1 < K) fwd_layer<K, t + 1>(x, tw, ls, hi, q, q2);
+}
+
+// fwd_radix with the first layer's twiddle w0 = Psi[2^ls + hi] already loaded by the
+// caller (issued before a barrier so its latency is hidden).
+template <int K>
+__device__ __forceinline__ void fwd_radix_w0(uint32_t* x, uint2 w0, const uint2* __restrict__ tw, int ls,
+                                             uint32_t hi, uint32_t q, uint32_t q2) {
+#pragma unroll
+    for (int r = 0; r < (1 << (K - 1)); ++r) ct_bfly(x[r], x[r + (1 << (K - 1))], w0, q, q2);
+    if constexpr (K > 1) fwd_layer<K, 1>(x, tw, ls, hi, q, q2);   // layers ls+1..ls+K-1
+}
+
 template <int K>
 __device__ __forceinline__ void fwd_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
                                           uint32_t hi, uint32_t q, uint32_t q2) {
-    {   // layer ls: one twiddle
-        const uint2 w = __ldg(tw + (1u << ls) + hi);
-#pragma unroll
-        for (int r = 0; r < (1 << (K - 1)); ++r) ct_bfly(x[r], x[r + (1 << (K - 1))], w, q, q2);
-    }
-#pragma unroll
-    for (int t = 1; t < K; ++t) {            // layers ls+1..: twiddle pairs are adjacent -> 16-byte loads
-        const int h = 1 << (K - 1 - t);
-        const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
-#pragma unroll
-        for (int g = 0; g < (1 << t); g += 2) {
-            const uint4 v = __ldg(tp + g / 2);
-            const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
-#pragma unroll
-            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], wa, q, q2);
-#pragma unroll
-            for (int r = 0; r < h; ++r) ct_bfly(x[2 * (g + 1) * h + r], x[2 * (g + 1) * h + r + h], wb, q, q2);
-        }
-    }
+    fwd_radix_w0<K>(x, __ldg(tw + (1u << ls) + hi), tw, ls, hi, q, q2);
 }
 
 // K inverse (GS) layers, mirror of fwd_radix: layers ls+K-1 down to ls.
 // LAST: this block ends at global layer 0 (ls == 0), fold N^-1 there.
-template <int K, bool LAST>
-__device__ __forceinline__ void inv_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
-                                          uint32_t hi, const LimbConst& c) {
+template <int K, int t>
+__device__ __forceinline__ void inv_layer(uint32_t* x, const uint2* __restrict__ tw, int ls,
+                                          uint32_t hi, uint32_t q, uint32_t q2) {
+    constexpr int h = 1 << (K - 1 - t);
+    const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
 #pragma unroll
-    for (int t = K - 1; t >= 1; --t) {
-        const int h = 1 << (K - 1 - t);
-        const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
+    for (int g = 0; g < (1 << t); g += 2) {
+        const uint4 v = __ldg(tp + g / 2);
+        const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
 #pragma unroll
-        for (int g = 0; g < (1 << t); g += 2) {
-            const uint4 v = __ldg(tp + g / 2);
-            const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
+        for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], wa, q, q2);
 #pragma unroll
-            for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], wa, c.q, c.q2);
-#pragma unroll
-            for (int r = 0; r < h; ++r) gs_bfly(x[2 * (g + 1) * h + r], x[2 * (g + 1) * h + r + h], wb, c.q, c.q2);
-        }
+        for (int r = 0; r < h; ++r) gs_bfly(x[2 * (g + 1) * h + r], x[2 * (g + 1) * h + r + h], wb, q, q2);
     }
+    if constexpr (t > 1) inv_layer<K, t - 1>(x, tw, ls, hi, q, q2);
+}
+
+// The first (top, t = K-1) layer of an inverse radix-2^K block reads 2^(K-1) adjacent
+// twiddles Psi[2^(ls+K-1) + (hi << (K-1)) ..]: InvTop holds them so a caller can
+// issue the loads early (before a barrier / while other work is in flight).
+template <int K>
+struct InvTop { uint4 v[(1 << (K - 1)) / 2]; };
+
+template <int K>
+__device__ __forceinline__ void inv_top_load(InvTop<K>& p, const uint2* __restrict__ tw, int ls, uint32_t hi) {
+    const uint4* tp = reinterpret_cast<const uint4*>(tw + (1u << (ls + K - 1)) + (hi << (K - 1)));
+#pragma unroll
+    for (int g = 0; g < (1 << (K - 1)) / 2; ++g) p.v[g] = __ldg(tp + g);
+}
+
+template <int K, bool LAST>
+__device__ __forceinline__ void inv_radix_p(uint32_t* x, const InvTop<K>& p, const uint2* __restrict__ tw, int ls,
+                                            uint32_t hi, const LimbConst& c) {
+    static_assert(K >= 2, "top layer needs two groups");
+#pragma unroll
+    for (int g = 0; g < (1 << (K - 1)); g += 2) {      // layer ls+K-1, h = 1
+        const uint4 v = p.v[g / 2];
+        gs_bfly(x[2 * g], x[2 * g + 1], make_uint2(v.x, v.y), c.q, c.q2);
+        gs_bfly(x[2 * g + 2], x[2 * g + 3], make_uint2(v.z, v.w), c.q, c.q2);
+    }
+    if constexpr (K > 2) inv_layer<K, K - 2>(x, tw, ls, hi, c.q, c.q2);
     if (LAST) {
 #pragma unroll
         for (int r = 0; r < (1 << (K - 1)); ++r) gs_bfly_last(x[r], x[r + (1 << (K - 1))], c);
@@ -126,6 +163,20 @@ __device__ __forceinline__ void inv_radix(uint32_t* x, const uint2* __restrict__
         const uint2 w = __ldg(tw + (1u << ls) + hi);
 #pragma unroll
         for (int r = 0; r < (1 << (K - 1)); ++r) gs_bfly(x[r], x[r + (1 << (K - 1))], w, c.q, c.q2);
+    }
+}
+
+template <int K, bool LAST>
+__device__ __forceinline__ void inv_radix(uint32_t* x, const uint2* __restrict__ tw, int ls,
+                                          uint32_t hi, const LimbConst& c) {
+    if constexpr (K >= 2) {
+        InvTop<K> p;
+        inv_top_load<K>(p, tw, ls, hi);
+        inv_radix_p<K, LAST>(x, p, tw, ls, hi, c);
+    } else if (LAST) {
+        gs_bfly_last(x[0], x[1], c);
+    } else {
+        gs_bfly(x[0], x[1], __ldg(tw + (1u << ls) + hi), c.q, c.q2);
     }
 }
 

@@ -310,7 +310,8 @@ __global__ void __launch_bounds__(TT, 1024 / TT) ntt_persist_cc(NttArgs a, uint3
                 if (kk < G::C2) inv_p2_chunk<LOGN, PW, 0, TT>(S, out, in2, kk * G::W2, tw, lc);
                 else inv_p1_chunk<LOGN, 0, TT>(S, out, (kk - G::C2) * G::W1, tw, lc);
             }
-            __threadfence_block();
+            // bar.sync orders this chunk's global stores of the intermediate before the
+            // next chunk's cp.async reads of it (CTA-scope synchronisation, PTX memory model)
             __syncthreads();
             if (dep) issue(row_id, kk + 1, Sn);
         }

@@ -37,7 +37,7 @@ struct wd_ntt_plan {
     int device = -1;
     int sm_count = 148;
     int v6_ctas = 4;               // resident 256-thread CTAs per SM for v6 (WD_NTT_CTAS: 2..4, A/B runs)
-    int kernel_ver = 0;            // 0 = measured default per N (v6 at 2^16, v2 at 2^15/2^17, v1 below);
+    int kernel_ver = 0;            // 0 = measured default per N (v6 at 2^16 and 2^17, v2 at 2^15, v1 below);
                                    // WD_NTT_KERNEL=v1|v2|v3|v5|v6 forces a generation (A/B runs)
     std::vector<uint32_t> primes, psi;
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
@@ -102,7 +102,7 @@ int prep_cc() {
             set_smem(ntt_persist_cc<LOGN, false, true>, G::SMEM_BYTES))
             return WD_ECUDA;
     }
-    if constexpr (LOGN == 16) {
+    if constexpr (LOGN == 16 || LOGN == 17) {
         using G = PGeo<LOGN, 256>;
         if (set_smem(ntt_persist_cc<LOGN, true, false, 256>, G::SMEM_BYTES) ||
             set_smem(ntt_persist_cc<LOGN, false, false, 256>, G::SMEM_BYTES) ||
@@ -167,10 +167,13 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             return;
         }
     }
-    if constexpr (LOGN == 16) {
-        if (p->kernel_ver == 6 || p->kernel_ver == 0) {   // v2 with 256-thread CTAs, 4 per SM
+    if constexpr (LOGN == 16 || LOGN == 17) {
+        if (p->kernel_ver == 6 || p->kernel_ver == 0) {   // v2 with 256-thread CTAs, 4 (2^16) / 3 (2^17) per SM
             using G = PGeo<LOGN, 256>;
-            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * p->v6_ctas));
+            int occ = 1;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_persist_cc<LOGN, true, false, 256>, 256, G::SMEM_BYTES);
+            const int ctas = std::max(1, std::min(p->v6_ctas, occ));   // never a second, non-resident wave
+            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * ctas));
             if (fwd) ntt_persist_cc<LOGN, true, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
             else if (a.in2) ntt_persist_cc<LOGN, false, true, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
             else ntt_persist_cc<LOGN, false, false, 256><<<grid, 256, G::SMEM_BYTES, s>>>(a, rows);
@@ -339,7 +342,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     // ---- device upload (the only H2D copy of the plan's life)
     if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
     cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
-    p->kernel_ver = p->logN == 16 ? 0 : 2;          // 0 = AUTO at 2^16: v5 for < SM-count rows, else v6
+    p->kernel_ver = (p->logN == 16 || p->logN == 17) ? 0 : 2;   // AUTO: v5 for < SM-count rows at 2^16, else v6
     if (const char* ev = getenv("WD_NTT_CTAS")) p->v6_ctas = std::max(1, std::min(4, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
