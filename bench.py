@@ -35,8 +35,13 @@ CONFIGS = {
     "c3": (16, 36, 64),        # headline (BASELINE.json metric / configs[2])
     "c4": (17, 48, 32),
 }
+# config 5 (the N sweep, BASELINE configs[4]) at batch 128 polynomials, 16 limbs: parity cases
+# and kernel-selection data, not bench lines
+for _lg in range(12, 18):
+    CONFIGS["s%d" % _lg] = (_lg, 16, 64)
 CONFIG_NAMES = {"c1": "config1 (BASELINE configs[0])", "c2": "config2 (one ciphertext)",
                 "c3": "config3 (BASELINE configs[2], headline)", "c4": "config4 per-GPU shard"}
+CONFIG_NAMES.update({"s%d" % _lg: "config5 sweep point N=2^%d, L=16, 128 polynomials" % _lg for _lg in range(12, 18)})
 METRIC = "NTT KOPS (N=2^16, L=36) at 1/2/4/8 B200; % of HBM / int8 tensor roofline"
 FALLBACK_HBM_GBS = 6650.0
 
@@ -325,7 +330,8 @@ def main():
                      "peak_kind": "%s (MEASURED_PEAKS.json hbm_gbs copy bandwidth)" % pk_kind,
                      "algorithmic_bytes_per_launch": alg_bytes},
         "gpu_launches": launches,
-        "occupancy_ctas_per_sm": {"cuda": wdntt.wd_ntt_occupancy(plan.handle, "cuda"),
+        "occupancy_ctas_per_sm": {"cuda_fwd": wdntt.wd_ntt_occupancy(plan.handle, "cuda", True),
+                                  "cuda_inv": wdntt.wd_ntt_occupancy(plan.handle, "cuda", False),
                                   "tensor_fwd": wdntt.wd_ntt_occupancy(plan.handle, "tensor", True),
                                   "tensor_inv": wdntt.wd_ntt_occupancy(plan.handle, "tensor", False)},
         "clocks": clk.summary(),

@@ -148,7 +148,7 @@ int wd_ntt_plan_get_mode(const wd_ntt_plan* plan);
 uint32_t wd_ntt_last_launches(void);
 
 /* Resident CTAs per SM the driver reports for the plan's main kernel in `mode`
- * (WD_MODE_CUDA / WD_MODE_TENSOR, N = 2^16), fwd != 0 for the forward kernel;
+ * (WD_MODE_CUDA: N = 2^16, 2^17; WD_MODE_TENSOR: N = 2^16), fwd != 0 for the forward kernel;
  * a negative value is -(cudaError_t).  Diagnostic only. */
 int wd_ntt_occupancy(const wd_ntt_plan* plan, int mode, int fwd);
 

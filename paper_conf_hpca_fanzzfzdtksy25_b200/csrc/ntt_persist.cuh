@@ -53,11 +53,17 @@ struct PGeo {
     static constexpr int INST0 = E1 / R0, INST1 = E1 / R1;
     static constexpr int W2 = T / 16;                // rows per phase-2 chunk
     static constexpr int C2 = N1 / W2;               // phase-2 chunks per row
-    static constexpr int P1_WORDS = N1 * W1;
+    // phase-1 word of (row p, column w) is p1(p) + w.  With W1 = 8 a warp spans 4 values of
+    // j whose stage-1 rows (p = j*R1 + r) would sit 8*R1 words apart, i.e. in the same banks:
+    // one extra W1 of padding per 2^A1 rows (monotone, so rows never overlap) moves them
+    // to 4 different bank groups; in stage 0 (p = j + r*R1) it is a warp-uniform offset.
+    static constexpr int P1_PAD = W1 >= 16 ? 0 : (N1 >> A1) * W1;
+    __device__ __forceinline__ static int p1(int p) { return p * W1 + (W1 >= 16 ? 0 : (p >> A1) * W1); }
+    static constexpr int P1_WORDS = N1 * W1 + P1_PAD;
     static constexpr int P2_WORDS = W2 * RS;
     static constexpr int BUF_WORDS = P1_WORDS > P2_WORDS ? P1_WORDS : P2_WORDS;
     static constexpr int SMEM_BYTES = 2 * 4 * BUF_WORDS;
-    static_assert(W1 % 4 == 0 && W1 >= 16 && 256 % W1 == 0, "phase-1 chunk");
+    static_assert(W1 % 4 == 0 && (W1 >= 16 || W1 == 8) && 256 % W1 == 0, "phase-1 chunk");
     static_assert(N1 % W2 == 0, "phase-2 chunk");
 };
 
@@ -72,7 +78,7 @@ __device__ __forceinline__ void load_p1(uint32_t* S, const uint32_t* src, int c0
     for (int k = 0; k < NSEG / G::T; ++k) {
         const int i = threadIdx.x % G::T + k * G::T;
         const int p = i / SEG, s = i % SEG;
-        cp_async16(S + p * G::W1 + 4 * s, src + p * 256 + c0 + 4 * s);
+        cp_async16(S + G::p1(p) + 4 * s, src + p * 256 + c0 + 4 * s);
     }
 }
 // phase-2 chunk: rows [r0, r0+W2), 256 words each -> swizzled ywords() layout
@@ -100,10 +106,10 @@ __device__ __forceinline__ void fwd_p1_chunk(uint32_t* S, uint32_t* out, int c0,
     for (int u = 0; u < G::INST0; ++u) {
         const int i0 = j * G::INST0 + u;
 #pragma unroll
-        for (int r = 0; r < G::R0; ++r) x[u * G::R0 + r] = S[(i0 + (r << G::A1)) * G::W1 + w];
+        for (int r = 0; r < G::R0; ++r) x[u * G::R0 + r] = S[G::p1((i0 + (r << G::A1))) + w];
         fwd_radix<G::A0>(x + u * G::R0, tw, 0, 0, q, q2);
 #pragma unroll
-        for (int r = 0; r < G::R0; ++r) S[(i0 + (r << G::A1)) * G::W1 + w] = x[u * G::R0 + r];
+        for (int r = 0; r < G::R0; ++r) S[G::p1((i0 + (r << G::A1))) + w] = x[u * G::R0 + r];
     }
     pbar<BAR>();
     const int c = c0 + w;
@@ -111,7 +117,7 @@ __device__ __forceinline__ void fwd_p1_chunk(uint32_t* S, uint32_t* out, int c0,
     for (int u = 0; u < G::INST1; ++u) {
         const int i1 = j * G::INST1 + u;
 #pragma unroll
-        for (int r = 0; r < G::R1; ++r) x[r] = S[((i1 << G::A1) + r) * G::W1 + w];
+        for (int r = 0; r < G::R1; ++r) x[r] = S[G::p1(((i1 << G::A1) + r)) + w];
         fwd_radix<G::A1>(x, tw, G::A0, i1, q, q2);
 #pragma unroll
         for (int r = 0; r < G::R1; ++r) out[((i1 << G::A1) + r) * 256 + c] = x[r];
@@ -232,10 +238,10 @@ __device__ __forceinline__ void inv_p1_chunk(uint32_t* S, uint32_t* out, int c0,
     for (int u = 0; u < G::INST1; ++u) {
         const int i1 = j * G::INST1 + u;
 #pragma unroll
-        for (int r = 0; r < G::R1; ++r) x[r] = S[((i1 << G::A1) + r) * G::W1 + w];
+        for (int r = 0; r < G::R1; ++r) x[r] = S[G::p1(((i1 << G::A1) + r)) + w];
         inv_radix<G::A1, false>(x, tw, G::A0, i1, lc);
 #pragma unroll
-        for (int r = 0; r < G::R1; ++r) S[((i1 << G::A1) + r) * G::W1 + w] = x[r];
+        for (int r = 0; r < G::R1; ++r) S[G::p1(((i1 << G::A1) + r)) + w] = x[r];
     }
     pbar<BAR>();
     const int c = c0 + w;
@@ -243,7 +249,7 @@ __device__ __forceinline__ void inv_p1_chunk(uint32_t* S, uint32_t* out, int c0,
     for (int u = 0; u < G::INST0; ++u) {
         const int i0 = j * G::INST0 + u;
 #pragma unroll
-        for (int r = 0; r < G::R0; ++r) x[u * G::R0 + r] = S[(i0 + (r << G::A1)) * G::W1 + w];
+        for (int r = 0; r < G::R0; ++r) x[u * G::R0 + r] = S[G::p1((i0 + (r << G::A1))) + w];
         inv_radix<G::A0, true>(x + u * G::R0, tw, 0, 0, lc);
 #pragma unroll
         for (int r = 0; r < G::R0; ++r)

@@ -18,6 +18,7 @@
 #include "modarith.cuh"
 #include "ntt_cuda_core.cuh"
 #include "ntt_persist.cuh"
+#include "ntt_v8.cuh"
 #include "ntt_smem.cuh"
 #include "ntt_cluster.cuh"
 #include "ntt_tensor.cuh"
@@ -37,7 +38,9 @@ struct wd_ntt_plan {
     int device = -1;
     int sm_count = 148;
     int v6_ctas = 4;               // resident 256-thread CTAs per SM for v6 (WD_NTT_CTAS: 2..4, A/B runs)
-    int kernel_ver = 0;            // 0 = measured default per N (v6 at 2^16 and 2^17, v2 at 2^15, v1 below);
+    int v8_minb = 0;               // v8 CTAs per SM (WD_NTT_MINB: 4..6; 0 = measured default)
+    int v8_cl = 0;                 // v8 CTAs per row cluster (WD_NTT_CL: 1, 2, 4; 0 = measured default)
+    int kernel_ver = 0;            // 0 = AUTO, the measured default per N and row count (launch_cc);
                                    // WD_NTT_KERNEL=v1|v2|v3|v5|v6 forces a generation (A/B runs)
     std::vector<uint32_t> primes, psi;
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
@@ -79,6 +82,14 @@ int prep_cc() {
     if (set_smem(ntt_fwd_cc<LOGN>, S::SMEM_BYTES) || set_smem(ntt_inv_cc<LOGN, false>, S::SMEM_BYTES) ||
         set_smem(ntt_inv_cc<LOGN, true>, S::SMEM_BYTES))
         return WD_ECUDA;
+    if constexpr (LOGN >= 12) {
+        if (set_smem(ntt_v8<LOGN, true, false, 0, 4>, V8_SMEM) || set_smem(ntt_v8<LOGN, false, false, 0, 4>, V8_SMEM) ||
+            set_smem(ntt_v8<LOGN, false, true, 0, 4>, V8_SMEM) || set_smem(ntt_v8<LOGN, true, false, 0, 5>, V8_SMEM) ||
+            set_smem(ntt_v8<LOGN, false, false, 0, 5>, V8_SMEM) || set_smem(ntt_v8<LOGN, false, true, 0, 5>, V8_SMEM) ||
+            set_smem(ntt_v8<LOGN, true, false, 0, 6>, V8_SMEM) || set_smem(ntt_v8<LOGN, false, false, 0, 6>, V8_SMEM) ||
+            set_smem(ntt_v8<LOGN, false, true, 0, 6>, V8_SMEM))
+            return WD_ECUDA;
+    }
     if constexpr (LOGN >= 14) {
         if (set_smem(ntt_fwd_cl<LOGN>, CL_BYTES) || set_smem(ntt_inv_cl<LOGN, false>, CL_BYTES) ||
             set_smem(ntt_inv_cl<LOGN, true>, CL_BYTES))
@@ -103,6 +114,11 @@ int prep_cc() {
             return WD_ECUDA;
     }
     if constexpr (LOGN == 16 || LOGN == 17) {
+        using G7 = PGeo<LOGN, 128>;
+        if (set_smem(ntt_persist_cc<LOGN, true, false, 128>, G7::SMEM_BYTES) ||
+            set_smem(ntt_persist_cc<LOGN, false, false, 128>, G7::SMEM_BYTES) ||
+            set_smem(ntt_persist_cc<LOGN, false, true, 128>, G7::SMEM_BYTES))
+            return WD_ECUDA;
         using G = PGeo<LOGN, 256>;
         if (set_smem(ntt_persist_cc<LOGN, true, false, 256>, G::SMEM_BYTES) ||
             set_smem(ntt_persist_cc<LOGN, false, false, 256>, G::SMEM_BYTES) ||
@@ -128,6 +144,48 @@ int prepare_kernels(uint32_t logN) {
     }
 }
 
+constexpr int V8_DEFAULT_MINB = 4;   // measured, see DESIGN.md 5.1
+constexpr int V8_DEFAULT_CL = 2;
+
+// v8 with a CL-CTA cluster per row: grid = resident clusters x CL
+template <int LOGN, int MINB, int CL>
+void launch_v8_cluster(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    if constexpr ((1 << (LOGN - 12)) % CL != 0) {
+        return;
+    } else {
+        cudaLaunchConfig_t cfg = {};
+        cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM; cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = CL; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+        cfg.attrs = at; cfg.numAttrs = 1;
+        auto kf = ntt_v8<LOGN, true, false, 0, MINB, CL>;
+        auto ki = ntt_v8<LOGN, false, false, 0, MINB, CL>;
+        auto kp = ntt_v8<LOGN, false, true, 0, MINB, CL>;
+        auto k = fwd ? kf : (a.in2 ? kp : ki);
+        int ncl = 0;
+        cfg.gridDim = dim3(148 * MINB / CL * CL);
+        if (cudaOccupancyMaxActiveClusters(&ncl, k, &cfg) != cudaSuccess || ncl < 1) { cudaGetLastError(); ncl = 1; }
+        cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)ncl) * CL);
+        cudaLaunchKernelEx(&cfg, k, a, rows);
+    }
+}
+
+// v8 (ntt_v8.cuh): persistent grid of min(rows, SMs x MINB) 256-thread CTAs
+template <int LOGN, int MINB>
+void launch_v8_minb(bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
+    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * MINB));
+    if (fwd) ntt_v8<LOGN, true, false, 0, MINB><<<grid, V8_T, V8_SMEM, s>>>(a, rows);
+    else if (a.in2) ntt_v8<LOGN, false, true, 0, MINB><<<grid, V8_T, V8_SMEM, s>>>(a, rows);
+    else ntt_v8<LOGN, false, false, 0, MINB><<<grid, V8_T, V8_SMEM, s>>>(a, rows);
+}
+template <int LOGN>
+void launch_v8(int minb, bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
+    if (minb == 6) launch_v8_minb<LOGN, 6>(fwd, a, rows, sm_count, s);
+    else if (minb == 5) launch_v8_minb<LOGN, 5>(fwd, a, rows, sm_count, s);
+    else launch_v8_minb<LOGN, 4>(fwd, a, rows, sm_count, s);
+}
+
 template <int LOGN>
 void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     using S = CcShape<LOGN>;
@@ -150,6 +208,33 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             return;
         }
     }
+    if constexpr (LOGN >= 12) {
+        if (p->kernel_ver == 81 || p->kernel_ver == 82) {   // timing experiment: one phase of v8 only
+            if (fwd && p->kernel_ver == 81) ntt_v8<LOGN, true, false, 1><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            else if (fwd) ntt_v8<LOGN, true, false, 2><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            else if (p->kernel_ver == 81) ntt_v8<LOGN, false, false, 1><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            else ntt_v8<LOGN, false, false, 2><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            return;
+        }
+        // AUTO at or above the SM count: v8 (see DESIGN.md 5.1 for the measured (CTAs/SM,
+        // cluster) choice; WD_NTT_MINB / WD_NTT_CL override it for A/B runs)
+        const bool autov8 = p->kernel_ver == 0 && rows >= (uint32_t)p->sm_count;
+        if (p->kernel_ver == 8 || autov8) {
+            int minb = p->v8_minb ? p->v8_minb : V8_DEFAULT_MINB;
+            int cl = p->v8_cl ? p->v8_cl : V8_DEFAULT_CL;
+            if (LOGN == 17 && fwd && !p->v8_minb) minb = 4;     // radix-32 column phase spills at 48 regs
+            if ((1 << (LOGN - 12)) < cl) cl = 1;
+            if (cl == 1) launch_v8<LOGN>(minb, fwd, a, rows, p->sm_count, s);
+            else if (cl == 2) {
+                if (minb == 4) launch_v8_cluster<LOGN, 4, 2>(fwd, a, rows, s);
+                else launch_v8_cluster<LOGN, 5, 2>(fwd, a, rows, s);
+            } else {
+                if (minb == 4) launch_v8_cluster<LOGN, 4, 4>(fwd, a, rows, s);
+                else launch_v8_cluster<LOGN, 5, 4>(fwd, a, rows, s);
+            }
+            return;
+        }
+    }
     if constexpr (LOGN == 15 || LOGN == 16) {
         if (p->kernel_ver == 3) {
             constexpr int PAIR = LOGN == 16 ? 2 : 1;
@@ -168,6 +253,16 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         }
     }
     if constexpr (LOGN == 16 || LOGN == 17) {
+        if (p->kernel_ver == 7) {   // v6 with 128-thread CTAs (barriers over 4 warps), up to 8 per SM
+            using G = PGeo<LOGN, 128>;
+            int occ = 1;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_persist_cc<LOGN, true, false, 128>, 128, G::SMEM_BYTES);
+            const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(p->sm_count * std::max(1, occ)));
+            if (fwd) ntt_persist_cc<LOGN, true, false, 128><<<grid, 128, G::SMEM_BYTES, s>>>(a, rows);
+            else if (a.in2) ntt_persist_cc<LOGN, false, true, 128><<<grid, 128, G::SMEM_BYTES, s>>>(a, rows);
+            else ntt_persist_cc<LOGN, false, false, 128><<<grid, 128, G::SMEM_BYTES, s>>>(a, rows);
+            return;
+        }
         if (p->kernel_ver == 6 || p->kernel_ver == 0) {   // v2 with 256-thread CTAs, 4 (2^16) / 3 (2^17) per SM
             using G = PGeo<LOGN, 256>;
             int occ = 1;
@@ -342,8 +437,10 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     // ---- device upload (the only H2D copy of the plan's life)
     if (cudaGetDevice(&p->device) != cudaSuccess) { cudaGetLastError(); p->device = -1; delete p; set_err(WD_ECUDA); return nullptr; }
     cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
-    p->kernel_ver = (p->logN == 16 || p->logN == 17) ? 0 : 2;   // AUTO: v5 for < SM-count rows at 2^16, else v6
+    p->kernel_ver = 0;   // AUTO: v8 at >= SM-count rows; below: v5 (2^15, 2^16), v6 (2^17), v1 (<= 2^14)
     if (const char* ev = getenv("WD_NTT_CTAS")) p->v6_ctas = std::max(1, std::min(4, atoi(ev)));
+    if (const char* ev = getenv("WD_NTT_MINB")) p->v8_minb = std::max(4, std::min(6, atoi(ev)));
+    if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
@@ -426,8 +523,12 @@ int wd_ntt_occupancy(const wd_ntt_plan* p, int mode, int fwd) {
     if (p->logN == 16 && mode == WD_MODE_TENSOR)
         e = fwd ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_tc16<true>, TC_T, TC_SMEM)
                 : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_tc16<false>, TC_T, TC_SMEM);
-    else if (p->logN == 16 && mode == WD_MODE_CUDA)
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_persist_cc<16, true, false>, 512, PGeo<16>::SMEM_BYTES);
+    else if (p->logN == 16 && mode == WD_MODE_CUDA)      // the AUTO kernel at >= SM-count rows (v8)
+        e = fwd ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_v8<16, true, false, 0, 5>, V8_T, V8_SMEM)
+                : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_v8<16, false, false, 0, 5>, V8_T, V8_SMEM);
+    else if (p->logN == 17 && mode == WD_MODE_CUDA)
+        e = fwd ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_v8<17, true, false, 0, 4>, V8_T, V8_SMEM)
+                : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ntt_v8<17, false, false, 0, 5>, V8_T, V8_SMEM);
     if (e != cudaSuccess) { cudaGetLastError(); return -(int)e; }
     return occ;
 }

@@ -11,5 +11,9 @@ timeout 600 python bench.py > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TA
 kill $SMI
 timeout 300 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_${TAG}_ref.json 2> gpurun_out/bench_${TAG}_ref.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"ntt_" --csv --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 3 --warmup 3 --e2e-steps 0 --no-cpu > /dev/null 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"ntt_persist" -s 2 -c 2 -o gpurun_out/prof_${TAG} python bench.py --steps 1 --warmup 3 --e2e-steps 0 --no-cpu > /dev/null 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"ntt_v8" -s 2 -c 2 -o gpurun_out/prof_${TAG} python bench.py --steps 1 --warmup 3 --e2e-steps 0 --no-cpu > /dev/null 2>&1
 echo done
+for cfg in c2 c4 c1; do
+  timeout 300 python bench.py --steps 20 --warmup 3 --e2e-steps 0 --no-cpu --config $cfg > gpurun_out/bench_${TAG}_$cfg.json 2> gpurun_out/bench_${TAG}_$cfg.err
+done
+echo done2

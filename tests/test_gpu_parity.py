@@ -249,8 +249,8 @@ def test_modes_headline_config(wd, mode, share):
 
 
 # -------------------------------------------------------------- every CUDA-core kernel generation
-@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6"])
-@pytest.mark.parametrize("logn", [14, 15, 16, 17])
+@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8"])
+@pytest.mark.parametrize("logn", [12, 13, 14, 15, 16, 17])
 def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
     n = 1 << logn
