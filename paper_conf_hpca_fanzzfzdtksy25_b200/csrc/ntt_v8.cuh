@@ -25,6 +25,7 @@
 #pragma once
 #include "ntt_persist.cuh"
 #include "ntt_smem.cuh"     // cluster_sync
+#include "ntt_tensor.cuh"   // tcgen05 helpers, byte-plane tables (v10)
 
 namespace wd {
 
@@ -248,6 +249,469 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
         }
         __syncthreads();                                 // smem buffers free for the next row
     }
+}
+
+
+// ---------------------------------------------------------------------------------------------
+// v9: v8 with the column phase staged through shared memory by cp.async (N = 2^13 .. 2^16).
+// ncu of v8 (profiles/r01/g1) puts ~20% of the stall samples on the first use of the column
+// loads (long scoreboard): a thread issues its 2^A column loads and waits for them.  Here each
+// warp prefetches its OWN slice of the next column pass (2^A rows x 32 words, 16-byte
+// cp.async) while it computes the current one, so no CTA barrier is added; a third buffer
+// takes the first unit of the NEXT row (forward: its first column pass, issued at the start of
+// this row's sub-row phase; inverse: its first sub-row, issued at the start of the column
+// phase), so the HBM latency of every input unit is hidden behind the current row's work.
+constexpr int V9_SMEM = 3 * V8_SUBW * 4;     // B0, B1 (ping-pong), B2 (next-row unit) = 48 KB
+
+// column pass slice of warp w: rows k = 0..R-1 of columns c0 + 32w .. c0 + 32w + 31 of `src`
+// -> buf[w*32R + 32k + lane] (warp-private: the warp alone writes and reads it)
+template <int R>
+__device__ __forceinline__ void v9_load_cols(uint32_t* buf, const uint32_t* src, int c0) {
+    const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    uint32_t* b = buf + w * 32 * R;
+    const uint32_t* g = src + c0 + 32 * w;
+#pragma unroll
+    for (int G = l; G < R * 8; G += 32)                 // granule G: row G/8, words 4(G%8)..+3
+        cp_async16(b + (G >> 3) * 32 + 4 * (G & 7), g + (G >> 3) * V8_SUBW + 4 * (G & 7));
+    cp_async_commit();
+}
+
+template <int LOGN, bool FWD, bool PW, int CL = 1>
+__global__ void __launch_bounds__(V8_T, 4) ntt_v9(NttArgs a, uint32_t rows) {
+    constexpr int A = LOGN - 12;
+    constexpr int R = 1 << A;
+    static_assert(A >= 1 && A <= 4, "v9: N = 2^13 .. 2^16 (a column pass must fit one 16 KB buffer)");
+    static_assert(R % CL == 0 && (V8_SUBW / V8_T) % CL == 0, "cluster splits passes and sub-rows evenly");
+    constexpr int NP = V8_SUBW / V8_T / CL;
+    constexpr int NS = R / CL;
+    const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
+    const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
+    extern __shared__ __align__(16) uint32_t smem[];
+    uint32_t* const B0 = smem;
+    uint32_t* const B1 = smem + V8_SUBW;
+    uint32_t* const B2 = smem + 2 * V8_SUBW;
+    const int t = threadIdx.x, w = t >> 5, lane = t & 31;
+    const int hi4 = t >> 4, lo4 = t & 15;
+    const uint32_t rstep = gridDim.x / CL;
+    uint32_t row = blockIdx.x / CL;
+
+    // prologue: the first unit of the first row into B2 (forward) / B0 (inverse)
+    if (row < rows) {
+        if constexpr (FWD) v9_load_cols<R>(B2, a.in + ((size_t)row << LOGN), p0 * V8_T);
+        else v8_load_inv_slice(B0, a.in + ((size_t)row << LOGN) + s0 * V8_SUBW);
+    }
+#pragma unroll 1
+    for (; row < rows; row += rstep) {
+        const uint32_t nrow = row + rstep;
+        const uint32_t limb = row % a.L;
+        const LimbConst lc = a.lc[limb];
+        const uint32_t q = lc.q, q2 = lc.q2;
+        const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+        const uint32_t* in = a.in + ((size_t)row << LOGN);
+        uint32_t* out = a.out + ((size_t)row << LOGN);
+
+        if constexpr (FWD) {
+            // ---- phase 1: layers 0..A-1 on columns; pass i in B2 (i = 0) or B[(i-1)&1]
+#pragma unroll 1
+            for (int i = 0; i < NP; ++i) {
+                const uint32_t* buf = i == 0 ? B2 : ((i - 1) & 1 ? B1 : B0);
+                if (i + 1 < NP) {
+                    __syncwarp();                                   // pass i-1's slice fully read
+                    v9_load_cols<R>(i & 1 ? B1 : B0, in, (p0 + i + 1) * V8_T);
+                    cp_async_wait<1>();
+                } else {
+                    cp_async_wait<0>();
+                }
+                __syncwarp();
+                uint32_t x[R];
+#pragma unroll
+                for (int k = 0; k < R; ++k) x[k] = buf[w * 32 * R + 32 * k + lane];
+                fwd_radix<A>(x, tw, 0, 0, q, q2);
+                const int c = (p0 + i) * V8_T + t;
+#pragma unroll
+                for (int k = 0; k < R; ++k) out[k * V8_SUBW + c] = x[k];
+            }
+            if constexpr (CL > 1) cluster_sync(); else __syncthreads();
+            // ---- phase 2: layers A..A+11 on sub-rows; the next row's first pass goes to B2
+            v8_load_fwd_slice(B0, out + s0 * V8_SUBW);
+            if (nrow < rows) v9_load_cols<R>(B2, a.in + ((size_t)nrow << LOGN), p0 * V8_T);
+            else cp_async_commit();                                 // keep the group count uniform
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = (s - s0) & 1 ? B1 : B0;
+                if (s == s0) cp_async_wait<1>(); else cp_async_wait<0>();
+                __syncwarp();
+                uint32_t x[16];
+                {
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    fwd_radix<4>(x, tw, A, (uint32_t)s, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
+                }
+                __syncthreads();
+                if (s + 1 < s1) v8_load_fwd_slice((s + 1 - s0) & 1 ? B1 : B0, out + (s + 1) * V8_SUBW);
+                uint2 w3[15];
+                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                {
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    fwd_radix<4>(x, tw, A + 4, (uint32_t)s * 16 + aa, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncwarp();
+                {
+                    const int aa = hi4, b = lo4;
+                    const uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    fwd16_tw(x, w3, q, q2);
+                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
+                                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                }
+            }
+        } else {
+            // ---- phase 2': layers A+11..A on sub-rows (the first one is already in flight in B0)
+            const uint32_t* in2 = a.in2 + ((size_t)row << LOGN);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = (s - s0) & 1 ? B1 : B0;
+                uint2 w3[15];
+                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                cp_async_wait<0>();
+                __syncwarp();
+                uint32_t x[16];
+                {
+                    const int aa = hi4, b = lo4;
+                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    if constexpr (PW) {
+                        const uint4* ip2 = reinterpret_cast<const uint4*>(in2 + s * V8_SUBW + t * 16);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            const uint4 u = __ldcs(ip2 + v);
+                            x[4 * v] = mul_mod(x[4 * v], u.x, lc); x[4 * v + 1] = mul_mod(x[4 * v + 1], u.y, lc);
+                            x[4 * v + 2] = mul_mod(x[4 * v + 2], u.z, lc); x[4 * v + 3] = mul_mod(x[4 * v + 3], u.w, lc);
+                        }
+                    }
+                    inv16_tw(x, w3, q, q2);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                }
+                __syncwarp();
+                {
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    inv_radix<4, false>(x, tw, A + 4, (uint32_t)s * 16 + aa, lc);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncthreads();
+                if (s + 1 < s1) v8_load_inv_slice((s + 1 - s0) & 1 ? B1 : B0, in + (s + 1) * V8_SUBW);
+                {
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    inv_radix<4, false>(x, tw, A, (uint32_t)s, lc);
+                    uint32_t* o = out + s * V8_SUBW + b * 16 + c;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) o[i * 256] = x[i];             // lazy intermediate, [0,2q)
+                }
+            }
+            if constexpr (CL > 1) cluster_sync(); else __syncthreads();
+            // ---- phase 1': layers A-1..0 on columns (N^-1 folded); pass i in B2 / B1 alternately,
+            // the next row's first sub-row goes to B0
+            v9_load_cols<R>(B2, out, p0 * V8_T);
+            if (nrow < rows) v8_load_inv_slice(B0, a.in + ((size_t)nrow << LOGN) + s0 * V8_SUBW);
+            else cp_async_commit();
+#pragma unroll 1
+            for (int i = 0; i < NP; ++i) {
+                const uint32_t* buf = i & 1 ? B1 : B2;
+                if (i + 1 < NP) {
+                    __syncwarp();
+                    v9_load_cols<R>(i & 1 ? B2 : B1, out, (p0 + i + 1) * V8_T);
+                    if (i == 0) cp_async_wait<2>();                 // the next row's sub-row may stay in flight
+                    else cp_async_wait<1>();
+                } else {
+                    cp_async_wait<0>();
+                }
+                __syncwarp();
+                uint32_t x[R];
+#pragma unroll
+                for (int k = 0; k < R; ++k) x[k] = buf[w * 32 * R + 32 * k + lane];
+                inv_radix<A, true>(x, tw, 0, 0, lc);
+                const int c = (p0 + i) * V8_T + t;
+#pragma unroll
+                for (int k = 0; k < R; ++k) __stcs(out + k * V8_SUBW + c, canon2(x[k], q));
+            }
+        }
+        __syncthreads();                                 // B0/B1 free for the next row
+    }
+    cp_async_wait<0>();
+}
+
+
+// ---------------------------------------------------------------------------------------------
+// v10 (N = 2^16): v8 with its column phase on the tensor cores -- the concurrent tensor +
+// CUDA-core design of SURVEY.md 8 row a9 (PAPER.md:316-330 WD-FUSE, re-derived for sm_100a).
+// The column phase (layers 0..3, forward; layers 3..0 with N^-1, inverse) is ONE 16x16 matrix
+// M0 (MI0) applied to all 4096 columns of the row, i.e. a plain GEMM X[4096 x 16] . M0^T: it runs
+// as tcgen05.mma.kind::i8 tiles of 128 columns (byte-plane identity of ntt_tensor.cuh: the u8 view
+// of the 16 input words is K = 64, the 4 pre-shifted byte planes of M0 are N = 64).  The
+// per-element-twiddle layers 4..15 stay on the CUDA cores (v8 phase 2).  Warps of the 4
+// co-resident CTAs of an SM are in different phases at any time, so the tensor pipe and the
+// CUDA-core butterflies overlap on the same SM.  Per 128-column tile: the 8 warps load the tile
+// (warp w: 32 columns x 8 coefficients, coalesced) straight into TMEM (tcgen05.st, lane =
+// column, column = coefficient: the A operand), one thread issues 2 MMAs (K = 2 x 32 bytes),
+// every warp reads its 8 outputs x 4 planes back (tcgen05.ld) and recombines them:
+//   y = (D0 + 2^8 D1) + Shoup(D2 + 2^8 D3, 2^16)   (D_b < 2^22, so D0 + 2^8 D1 < 2^30)
+// which is < 2^30 + 2q, i.e. < 4q (the CT butterflies' input range) once q > 2^29.
+// TMEM: 128 columns per CTA (4 CTAs per SM = all 512): [0,16) A, [64,128) D.
+constexpr int V10_SMEM = V8_SMEM + 4096 + 64;            // sub-row buffers, B planes, mbarrier + TMEM slot
+
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t* v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+                 :: "r"(taddr), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+                 : "memory");
+}
+
+// y = sum_b 2^(8b) D_b (mod q) in [0, 4q) for every q < 2^30 (the q <= 2^29 branch reduces the
+// low half first); uniform branch per limb
+__device__ __forceinline__ uint32_t v10_combine(const uint32_t* d, uint32_t q, uint32_t q2, uint32_t c16s,
+                                                uint32_t one_s) {
+    const uint32_t lo = d[0] + (d[1] << 8);
+    const uint32_t hi = shoup_mul(d[2] + (d[3] << 8), 65536u, c16s, q);
+    if (q > (1u << 29)) return lo + hi;
+    return shoup_mul(lo, 1u, one_s, q) + hi;
+}
+
+// the column phase of one row on the tensor cores: tiles of 128 columns [c_lo, c_hi)
+// FWD: src = input row, dst = intermediate (lazy [0,4q)); inverse: src = dst = row's out slot,
+// canonical result.  Bt = the 4 KB byte-plane image of M0 / MI0 (already in smem, fenced).
+template <bool FWD>
+__device__ __forceinline__ void v10_columns(const uint32_t* src, uint32_t* dst, int c_lo, int c_hi,
+                                            uint32_t tmem, uint32_t bt, uint64_t* bar, uint32_t& ph,
+                                            uint32_t q, uint32_t q2, uint32_t c16s, uint32_t one_s) {
+    const int t = threadIdx.x, w = t >> 5, lane = t & 31;
+    const int lq = w & 3, kh = w >> 2;                     // TMEM lane quarter, coefficient half
+    const uint32_t tl = tmem + ((uint32_t)(32 * lq) << 16);
+    uint32_t x[8];
+    int c = c_lo + 32 * lq + lane;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x[i] = FWD ? __ldcs(src + (8 * kh + i) * V8_SUBW + c) : src[(8 * kh + i) * V8_SUBW + c];
+#pragma unroll 1
+    for (int c0 = c_lo; c0 < c_hi; c0 += 128) {
+        tmem_st8(tl + 8 * kh, x);                          // A: lane = column, TMEM column = coefficient
+        tmem_wait_st();
+        tc_fence_before();
+        __syncthreads();                                   // A complete; the previous tile's D fully read
+        if (t == 0) {
+            tc_fence_after();
+            tc_mma_ts(tmem + 64, tmem, umma_desc(bt), 0);
+            tc_mma_ts(tmem + 64, tmem + 8, umma_desc(bt + 256), 1);
+            tc_commit(bar);
+        }
+        c = c0 + 32 * lq + lane;
+        if (c0 + 128 < c_hi) {                             // next tile's loads in flight during the MMA
+            const int cn = c + 128;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) x[i] = FWD ? __ldcs(src + (8 * kh + i) * V8_SUBW + cn) : src[(8 * kh + i) * V8_SUBW + cn];
+        }
+        mbar_wait(bar, ph);
+        ph ^= 1;
+        tc_fence_after();
+        uint32_t d[32];
+        tmem_ld32(tl + 64 + 32 * kh, d);                   // outputs k = 8 kh .. 8 kh + 7, 4 planes each
+        tmem_wait_ld();
+        tc_fence_before();
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk) {
+            const uint32_t y = v10_combine(d + 4 * kk, q, q2, c16s, one_s);
+            if (FWD) dst[(8 * kh + kk) * V8_SUBW + c] = y;
+            else __stcs(dst + (8 * kh + kk) * V8_SUBW + c, canon4(y, q, q2));
+        }
+    }
+}
+
+template <bool FWD, bool PW, int CL = 2>
+__global__ void __launch_bounds__(V8_T, 4) ntt_v10(NttArgs a, const uint8_t* G, const uint2* c16, uint32_t rows) {
+    constexpr int LOGN = 16, A = 4;
+    constexpr int NP = V8_SUBW / V8_T / CL;
+    constexpr int NS = 16 / CL;
+    const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
+    const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
+    extern __shared__ __align__(1024) uint32_t smem[];
+    uint8_t* Bt = reinterpret_cast<uint8_t*>(smem + 2 * V8_SUBW);
+    uint64_t* bar = reinterpret_cast<uint64_t*>(Bt + 4096);
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(bar + 1);
+    const int t = threadIdx.x;
+    const int hi4 = t >> 4, lo4 = t & 15;
+    if (t == 0) {
+        mbar_init(bar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (t < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tslot;
+    const uint32_t bt = smem_addr(Bt);
+    uint32_t ph = 0;
+
+#pragma unroll 1
+    for (uint32_t row = blockIdx.x / CL; row < rows; row += gridDim.x / CL) {
+        const uint32_t limb = row % a.L;
+        const LimbConst lc = a.lc[limb];
+        const uint32_t q = lc.q, q2 = lc.q2;
+        const uint2 cc = c16[limb];
+        const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+        const uint32_t* in = a.in + ((size_t)row << LOGN);
+        uint32_t* out = a.out + ((size_t)row << LOGN);
+        // B planes of this limb's single-group column matrix (M0 forward, MI0 inverse)
+        cp_async16(Bt + 16 * t, G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096 + 16 * t);
+        cp_async_commit();
+
+        if constexpr (FWD) {
+            cp_async_wait<0>();
+            fence_async_smem();
+            // ---- phase 1 on the tensor cores (the __syncthreads inside publishes Bt)
+            v10_columns<true>(in, out, p0 * V8_T, (p0 + NP) * V8_T, tmem, bt, bar, ph, q, q2, cc.x, cc.y);
+            if constexpr (CL > 1) cluster_sync(); else __syncthreads();
+            // ---- phase 2: layers 4..15 on sub-rows (v8)
+            v8_load_fwd_slice(smem, out + s0 * V8_SUBW);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
+                cp_async_wait<0>();
+                __syncwarp();
+                uint32_t x[16];
+                {
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    fwd_radix<4>(x, tw, A, (uint32_t)s, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
+                }
+                __syncthreads();
+                if (s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, out + (s + 1) * V8_SUBW);
+                uint2 w3[15];
+                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                {
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    fwd_radix<4>(x, tw, A + 4, (uint32_t)s * 16 + aa, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncwarp();
+                {
+                    const int aa = hi4, b = lo4;
+                    const uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    fwd16_tw(x, w3, q, q2);
+                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
+                                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                }
+            }
+        } else {
+            // ---- phase 2': layers 15..4 on sub-rows (v8)
+            const uint32_t* in2 = a.in2 + ((size_t)row << LOGN);
+            v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
+                uint2 w3[15];
+                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                cp_async_wait<0>();
+                __syncwarp();
+                uint32_t x[16];
+                {
+                    const int aa = hi4, b = lo4;
+                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    if constexpr (PW) {
+                        const uint4* ip2 = reinterpret_cast<const uint4*>(in2 + s * V8_SUBW + t * 16);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            const uint4 u = __ldcs(ip2 + v);
+                            x[4 * v] = mul_mod(x[4 * v], u.x, lc); x[4 * v + 1] = mul_mod(x[4 * v + 1], u.y, lc);
+                            x[4 * v + 2] = mul_mod(x[4 * v + 2], u.z, lc); x[4 * v + 3] = mul_mod(x[4 * v + 3], u.w, lc);
+                        }
+                    }
+                    inv16_tw(x, w3, q, q2);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                }
+                __syncwarp();
+                {
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    inv_radix<4, false>(x, tw, A + 4, (uint32_t)s * 16 + aa, lc);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncthreads();
+                if (s + 1 < s1) v8_load_inv_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, in + (s + 1) * V8_SUBW);
+                {
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    inv_radix<4, false>(x, tw, A, (uint32_t)s, lc);
+                    uint32_t* o = out + s * V8_SUBW + b * 16 + c;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) o[i * 256] = x[i];
+                }
+            }
+            cp_async_wait<0>();
+            fence_async_smem();
+            if constexpr (CL > 1) cluster_sync(); else __syncthreads();
+            // ---- phase 1' on the tensor cores: layers 3..0 with N^-1 (MI0), canonical output
+            v10_columns<false>(out, out, p0 * V8_T, (p0 + NP) * V8_T, tmem, bt, bar, ph, q, q2, cc.x, cc.y);
+        }
+        __syncthreads();                                 // smem buffers / Bt free for the next row
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (t < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
 }
 
 }  // namespace wd

@@ -90,6 +90,18 @@ int prep_cc() {
             set_smem(ntt_v8<LOGN, false, true, 0, 6>, V8_SMEM))
             return WD_ECUDA;
     }
+    if constexpr (LOGN == 16) {
+        if (set_smem(ntt_v10<true, false, 1>, V10_SMEM) || set_smem(ntt_v10<false, false, 1>, V10_SMEM) ||
+            set_smem(ntt_v10<false, true, 1>, V10_SMEM) || set_smem(ntt_v10<true, false, 2>, V10_SMEM) ||
+            set_smem(ntt_v10<false, false, 2>, V10_SMEM) || set_smem(ntt_v10<false, true, 2>, V10_SMEM))
+            return WD_ECUDA;
+    }
+    if constexpr (LOGN >= 13 && LOGN <= 16) {
+        if (set_smem(ntt_v9<LOGN, true, false, 1>, V9_SMEM) || set_smem(ntt_v9<LOGN, false, false, 1>, V9_SMEM) ||
+            set_smem(ntt_v9<LOGN, false, true, 1>, V9_SMEM) || set_smem(ntt_v9<LOGN, true, false, 2>, V9_SMEM) ||
+            set_smem(ntt_v9<LOGN, false, false, 2>, V9_SMEM) || set_smem(ntt_v9<LOGN, false, true, 2>, V9_SMEM))
+            return WD_ECUDA;
+    }
     if constexpr (LOGN >= 14) {
         if (set_smem(ntt_fwd_cl<LOGN>, CL_BYTES) || set_smem(ntt_inv_cl<LOGN, false>, CL_BYTES) ||
             set_smem(ntt_inv_cl<LOGN, true>, CL_BYTES))
@@ -171,6 +183,31 @@ void launch_v8_cluster(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s
     }
 }
 
+// v9 (ntt_v8.cuh): v8 with cp.async-staged column passes; grid = resident clusters x CL
+template <int LOGN, int CL>
+void launch_v9(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    if constexpr (LOGN < 13 || LOGN > 16 || (1 << (LOGN - 12)) % CL != 0) {
+        return;
+    } else {
+        cudaLaunchConfig_t cfg = {};
+        cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V9_SMEM; cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = CL; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+        cfg.attrs = at; cfg.numAttrs = 1;
+        auto k = fwd ? ntt_v9<LOGN, true, false, CL> : (a.in2 ? ntt_v9<LOGN, false, true, CL> : ntt_v9<LOGN, false, false, CL>);
+        int ncl = 0;
+        cfg.gridDim = dim3(148 * 4 / CL * CL);
+        if (cudaOccupancyMaxActiveClusters(&ncl, k, &cfg) != cudaSuccess || ncl < 1) { cudaGetLastError(); ncl = 1; }
+        cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)ncl) * CL);
+        cudaLaunchKernelEx(&cfg, k, a, rows);
+    }
+}
+
+// v10 (ntt_v8.cuh, N = 2^16): v8 with the column phase on the tensor cores; 2-CTA cluster per row
+template <int CL>
+void launch_v10(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s);
+
 // v8 (ntt_v8.cuh): persistent grid of min(rows, SMs x MINB) 256-thread CTAs
 template <int LOGN, int MINB>
 void launch_v8_minb(bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
@@ -218,6 +255,19 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         }
         // AUTO at or above the SM count: v8 (see DESIGN.md 5.1 for the measured (CTAs/SM,
         // cluster) choice; WD_NTT_MINB / WD_NTT_CL override it for A/B runs)
+        if constexpr (LOGN == 16) {
+            if (p->kernel_ver == 10 && p->tc.ok) {
+                if ((p->v8_cl ? p->v8_cl : V8_DEFAULT_CL) >= 2) launch_v10<2>(p, fwd, a, rows, s);
+                else launch_v10<1>(p, fwd, a, rows, s);
+                return;
+            }
+        }
+        if (p->kernel_ver == 9 && LOGN >= 13 && LOGN <= 16) {
+            const int cl = (p->v8_cl ? p->v8_cl : V8_DEFAULT_CL) >= 2 && LOGN >= 13 ? 2 : 1;
+            if (cl == 2) launch_v9<LOGN, 2>(fwd, a, rows, s);
+            else launch_v9<LOGN, 1>(fwd, a, rows, s);
+            return;
+        }
         const bool autov8 = p->kernel_ver == 0 && rows >= (uint32_t)p->sm_count;
         if (p->kernel_ver == 8 || autov8) {
             int minb = p->v8_minb ? p->v8_minb : V8_DEFAULT_MINB;
@@ -290,6 +340,28 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
     if (fwd) ntt_fwd_cc<LOGN><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
     else if (a.in2) ntt_inv_cc<LOGN, true><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
     else ntt_inv_cc<LOGN, false><<<rows, S::T, S::SMEM_BYTES, s>>>(a);
+}
+
+template <int CL>
+void launch_v10(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V10_SMEM; cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = CL; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+    cfg.attrs = at; cfg.numAttrs = 1;
+    auto k = fwd ? ntt_v10<true, false, CL> : (a.in2 ? ntt_v10<false, true, CL> : ntt_v10<false, false, CL>);
+    // 4 CTAs per SM, each holding 128 of the SM's 512 TMEM columns.  (The occupancy API
+    // reports 1 block/SM for this kernel; measured, 4 co-resident CTAs run: 1.48 -> 1.29 ms.)
+    int ncl = p->sm_count * 4 / CL;
+    if (const char* ev = getenv("WD_NTT_V10_CLUSTERS")) ncl = std::max(1, atoi(ev));
+    if (getenv("WD_NTT_DEBUG")) {
+        int occ = -1;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, V8_T, V10_SMEM);
+        fprintf(stderr, "v10: clusters %d, blocks/SM %d\n", ncl, occ);
+    }
+    cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)ncl) * CL);
+    cudaLaunchKernelEx(&cfg, k, a, (const uint8_t*)p->tc.d_G, (const uint2*)p->tc.d_c16, rows);
 }
 
 int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {

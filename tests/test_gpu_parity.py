@@ -249,7 +249,7 @@ def test_modes_headline_config(wd, mode, share):
 
 
 # -------------------------------------------------------------- every CUDA-core kernel generation
-@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8"])
+@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8", "v9", "v10"])
 @pytest.mark.parametrize("logn", [12, 13, 14, 15, 16, 17])
 def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
@@ -270,3 +270,41 @@ def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     torch.cuda.synchronize()
     prod = (x.astype(np.uint64) * q.astype(np.uint64)) % np.array(primes, np.uint64)[None, :, None]
     assert np.array_equal(to_host(o), oracle.ntt_inverse(prod.astype(np.uint32), primes)), (ver, logn)
+
+
+# -------------------------------------------------------------- persistent kernels over many rows
+# More rows than resident CTAs (clusters), so every CTA walks several rows and the cross-row
+# prefetches (v9: next row's first unit staged during the current row) are exercised; the row
+# count is ragged with respect to the grid.
+@pytest.mark.parametrize("ver", ["v8", "v9", "v10"])
+@pytest.mark.parametrize("logn,batch", [(14, 161), (16, 83)])
+def test_persistent_many_rows(wd, ver, logn, batch, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", ver)
+    n = 1 << logn
+    primes = [P[1], P[7], P[30], P[58]]
+    x = inputs.uniform_residues(primes, n, batch, 5100 + logn)
+    plan = wd.Plan(n, primes, mode="cuda")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (ver, logn)
+    assert np.array_equal(gpu_inv(wd, plan, y), x), (ver, logn)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (ver, logn)
+
+
+# Primes across the range the ABI accepts: the tensor column phase (v10) recombines its byte
+# planes with a cheaper reduction when q > 2^29 and a general one below; both must be exact.
+# 786433 = 3 * 2^18 + 1; the others are the first primes = 1 (mod 2^17) above 2^28, 2^29, 1.5*2^29.
+@pytest.mark.parametrize("ver", ["v8", "v10"])
+def test_prime_sizes_n16(wd, ver, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", ver)
+    n = 1 << 16
+    primes = [786433, 269221889, 537133057, 805961729, P[0]]
+    for q in primes:
+        assert oracle.is_prime(q) and (q - 1) % (2 * n) == 0
+    x = inputs.uniform_residues(primes, n, 3, 5200)
+    plan = wd.Plan(n, primes, mode="cuda")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), ver
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), ver
+    q = np.repeat(inputs.structured("qm1", primes, n), 3, axis=0)
+    assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes)), ver
+    assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes)), ver
