@@ -180,6 +180,54 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def run_rescale(args):
+    """--op rescale: CKKS RESCALE (wd_rescale, row f4) of a batch of polynomials, config shape
+    (default c3: N=2^16, L=36 -> 35 limbs, 128 polynomials).  One step = one rescale of every
+    polynomial; value = polynomials rescaled per second.  Roofline: HBM, algorithmic bytes =
+    read L*N*4 + write (L-1)*N*4 per polynomial (the work buffer round trip of the last limb,
+    4*N*4 bytes, is overhead, not algorithmic)."""
+    import torch
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt
+    torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+    logn, L, nct = CONFIGS[args.config]
+    n = 1 << logn
+    batch = 1 if nct is None else 2 * nct
+    primes = inputs.bench_primes(L)
+    plan = wdntt.Plan(n, primes)
+    x = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 2, device="cuda")
+    out = torch.empty((batch, L - 1, n), dtype=x.dtype, device="cuda")
+    work = torch.empty((batch, n), dtype=x.dtype, device="cuda")
+    sp = torch.cuda.current_stream().cuda_stream
+    for _ in range(max(3, args.warmup)):
+        wdntt.wd_rescale(plan.handle, x, out, batch, work, sp)
+    torch.cuda.synchronize()
+    launches = 0
+    with ClockSampler(0) as clk:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(args.steps):
+            wdntt.wd_rescale(plan.handle, x, out, batch, work, sp)
+            launches += wdntt.wd_ntt_last_launches()
+        e1.record()
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    pk, pk_kind = peaks()
+    hbm = float(pk.get("hbm_gbs", FALLBACK_HBM_GBS))
+    alg = batch * n * 4.0 * (2 * L - 1)
+    line = {"metric": "CKKS RESCALE throughput (N=2^%d, L=%d -> %d)" % (logn, L, L - 1),
+            "value": batch / (ms / 1e3), "unit": "polynomials/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic (splitmix64 uniform residues)",
+            "us_per_ciphertext": 2 * ms * 1e3 / batch,
+            "config": {"workload": "%s: rescale of %d polynomials" % (CONFIG_NAMES[args.config], batch),
+                       "N": n, "L": L, "polys": batch},
+            "roofline": {"bound": "hbm", "kernel": "whole op (3 launches)", "achieved": alg / (ms / 1e3) / 1e9,
+                         "peak": hbm, "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None,
+                         "peak_kind": pk_kind, "algorithmic_bytes_per_step": alg},
+            "gpu_launches": launches, "clocks": clk.summary()}
+    print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -192,7 +240,12 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--op", default="ntt", choices=["ntt", "rescale"],
+                    help="ntt: the headline forward+inverse step; rescale: SURVEY.md 8 row f4")
     args = ap.parse_args()
+    if args.op == "rescale":
+        run_rescale(args)
+        return
 
     if args.impl == "reference":
         run_reference(args)

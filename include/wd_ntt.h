@@ -122,6 +122,26 @@ int wd_ntt_inverse_host(const wd_ntt_plan* plan, const uint32_t* h_in, uint32_t*
 int wd_ntt_pointwise_inverse(const wd_ntt_plan* plan, const uint32_t* a, const uint32_t* b,
                              uint32_t* out, uint32_t batch, wd_stream_t stream);
 
+/*
+ * wd_rescale -- SURVEY.md 8 row f4 (NEXT #4), the CKKS rescale of PAPER.md:81
+ * ("RSCALE(ct0) = (a0', b0') in R^2_{Q_{l-1}}"), reading C-18:
+ * a' = round(a / q_last) for every polynomial, q_last = the plan's LAST prime,
+ * i.e. a'_i = floor((A + floor(q_last/2)) / q_last) mod q_i for the integer
+ * (CRT) value A of each coefficient.
+ *   in     device, [batch][L][N] NTT-domain residues over the plan's primes
+ *          (the forward's bit-reversed order), canonical
+ *   out    device, [batch][L-1][N] NTT-domain residues over primes[0..L-2],
+ *          canonical; must not overlap `in` or `work`
+ *   work   caller-owned device scratch of >= batch*N words (16-B aligned)
+ * Three launches: gather the last limb, its INTT, then one forward-NTT launch
+ * over all batch*(L-1) output rows with the rescale arithmetic fused into its
+ * load and store (PE kernel).  Needs L >= 2, N >= 2^12 and
+ * q_last distinct from the other primes (else WD_EUNSUPPORTED); pointer errors
+ * give WD_EINVAL.  Stream-ordered and asynchronous like the transforms.
+ */
+int wd_rescale(const wd_ntt_plan* plan, const uint32_t* in, uint32_t* out, uint32_t batch,
+               uint32_t* work, wd_stream_t stream);
+
 /* ---- queries and knobs ---- */
 uint32_t wd_ntt_plan_n(const wd_ntt_plan* plan);
 uint32_t wd_ntt_plan_limbs(const wd_ntt_plan* plan);

@@ -87,3 +87,63 @@ def rescale_rns(a: np.ndarray, primes) -> np.ndarray:
         t = (a[:, i, :].astype(np.uint64) + qi - u.astype(np.uint64)) % qi
         out[:, i, :] = (t * inv % qi).astype(np.uint32)                          # step 5
     return out
+
+
+# ---------------------------------------------------------------------------------------------
+# Basis conversion, ModUp, ModDown (Table III and
+# PAPER.md:350 Fig. 4 name them as the KeySwitch kernels around the NTT; the paper does not
+# restate their formulas, so DESIGN.md reading C-19 takes the standard RNS-CKKS ones of the
+# "100x" baseline it compares against): for a source basis {q_i} with product Q,
+#   BConv_{Q->P}(x)_j = sum_i [x_i * (Q/q_i)^{-1}]_{q_i} * (Q/q_i)  mod p_j
+# which equals (A + u Q) mod p_j for the integer value A of x and one u in [0, #q) (the fast,
+# approximate lift: it does not remove the multiple u Q).
+#   ModUp(a)   = a on the Q limbs, NTT_P(BConv_{Q->P}(INTT_Q(a))) on the P limbs
+#   ModDown(a) = (a_Q - NTT_Q(BConv_{P->Q}(INTT_P(a_P)))) * P^{-1}  on the Q limbs
+# All polynomials in and out are NTT-domain (bit-reversed order), [B][limbs][N].
+
+def bconv(x: np.ndarray, src, dst) -> np.ndarray:
+    """Coefficient-domain fast basis conversion [B][len(src)][N] -> [B][len(dst)][N] (literal)."""
+    x = np.ascontiguousarray(x, dtype=np.uint32)
+    B, a, N = x.shape
+    assert a == len(src)
+    Q = 1
+    for q in src:
+        Q *= int(q)
+    out = np.zeros((B, len(dst), N), dtype=np.uint32)
+    ys = []
+    for i, q in enumerate(src):
+        q = int(q)
+        qhat = Q // q
+        ys.append((x[:, i, :].astype(object) * pow(qhat % q, -1, q)) % q)       # y_i, exact ints
+    for j, p in enumerate(dst):
+        p = int(p)
+        acc = np.zeros((B, N), dtype=object)
+        for i, q in enumerate(src):
+            acc = acc + ys[i] * ((Q // int(q)) % p)
+        out[:, j, :] = (acc % p).astype(np.uint64).astype(np.uint32)
+    return out
+
+
+def modup(a: np.ndarray, qs, ps) -> np.ndarray:
+    """[B][#q][N] NTT over qs -> [B][#q + #p][N] NTT over qs + ps."""
+    a = np.ascontiguousarray(a, dtype=np.uint32)
+    coeff = ntt_inverse(a, qs)
+    ext = ntt_forward(bconv(coeff, qs, ps), ps)
+    return np.concatenate([a, ext], axis=1)
+
+
+def moddown(a: np.ndarray, qs, ps) -> np.ndarray:
+    """[B][#q + #p][N] NTT over qs + ps -> [B][#q][N] NTT over qs: (a - BConv(a_P)) / P."""
+    a = np.ascontiguousarray(a, dtype=np.uint32)
+    nq = len(qs)
+    P = 1
+    for p in ps:
+        P *= int(p)
+    cp = ntt_inverse(np.ascontiguousarray(a[:, nq:, :]), ps)
+    corr = ntt_forward(bconv(cp, ps, qs), qs)
+    out = np.empty((a.shape[0], nq, a.shape[2]), dtype=np.uint32)
+    for i, q in enumerate(qs):
+        q = int(q)
+        t = (a[:, i, :].astype(np.uint64) + q - corr[:, i, :].astype(np.uint64)) % q
+        out[:, i, :] = (t * pow(P % q, -1, q) % q).astype(np.uint32)
+    return out

@@ -32,6 +32,13 @@ struct NttArgs {
     const uint2* tw;          // [L][N] (psi^+-brv(i), Shoup) for this direction
     const LimbConst* lc;      // [L]
     uint32_t L;
+    // RESCALE epilogue of the forward (ntt_v8<..., EPI = 1>): the phase-1
+    // input row of row r is in + (r / L) * N (the last limb's coefficients c of polynomial r / L,
+    // shared by its L output limbs), the output is (aux_i - NTT(c')) * q_last^-1 (ntt_rns.cuh)
+    const uint32_t* aux = nullptr;   // the rescale input [batch][Lfull][N]
+    const uint4* rs = nullptr;       // [L] {-q_last mod q_i, Shoup(1), q_last^-1 mod q_i, Shoup}
+    uint32_t rs_thr = 0;             // q_last - floor(q_last / 2)
+    uint32_t Lfull = 0;
 };
 
 constexpr int RS = 272;       // padded row stride (words) of 256-wide rows in SMEM

@@ -78,7 +78,20 @@ __device__ __forceinline__ void v8_load_sub(uint32_t* S, const uint32_t* src) {
 // CL > 1: a cluster of CL CTAs shares each row -- CTA rank r takes column passes and sub-rows
 // [r, r+1) * (16|R)/CL, with ONE cluster barrier (release/acquire) between the phases.  Rows
 // in flight, hence the L2 footprint of the intermediate, shrink by CL.
-template <int LOGN, bool FWD, bool PW, int ONLY = 0, int MINB = 4, int CL = 1>
+// RESCALE input map (EPI = 1): c in [0, q_last) -> a representative in [0, 2q) of the centred
+// residue v = c - q_last [c >= q_last - floor(q_last/2)] of the coefficient mod q_last, mod q
+// (oracle/rns.py steps 2-4)
+// c + (-q_last mod q) < 2^31 is already a valid lazy input (< 4q) when q >= 2^29 (uniform branch)
+__device__ __forceinline__ uint32_t rs_in(uint32_t c, uint32_t thr, const uint4& r, uint32_t q) {
+    const uint32_t v = c + (c >= thr ? r.x : 0u);
+    return q >= (1u << 29) ? v : shoup_mul(v, 1u, r.y, q);
+}
+// RESCALE output map: y = NTT_q(v) in [0, 2q) -> (a - y) * q_last^-1 mod q, canonical (step 5)
+__device__ __forceinline__ uint32_t rs_out(uint32_t aval, uint32_t y, const uint4& r, uint32_t q) {
+    return canon2(shoup_mul(aval + 2 * q - y, r.z, r.w, q), q);
+}
+
+template <int LOGN, bool FWD, bool PW, int ONLY = 0, int MINB = 4, int CL = 1, int EPI = 0>
 __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
     constexpr bool JIT3 = MINB > 4;
     constexpr int A = LOGN - 12;             // phase-1 layers (radix 2^A columns)
@@ -99,8 +112,14 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
         const LimbConst lc = a.lc[limb];
         const uint32_t q = lc.q, q2 = lc.q2;
         const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
-        const uint32_t* in = a.in + ((size_t)row << LOGN);
+        const uint32_t* in = a.in + ((size_t)(EPI ? row / a.L : row) << LOGN);
         uint32_t* out = a.out + ((size_t)row << LOGN);
+        uint4 rsc = make_uint4(0, 0, 0, 0);
+        const uint32_t* ain = nullptr;
+        if constexpr (EPI) {
+            rsc = a.rs[limb];
+            ain = a.aux + (((size_t)(row / a.L) * a.Lfull + limb) << LOGN);
+        }
 
         if constexpr (FWD) {
             // ---- phase 1: layers 0..A-1 on columns c (elements c + 4096 k) ----
@@ -110,7 +129,10 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     const int c = pass * V8_T + t;
                     uint32_t x[R];
 #pragma unroll
-                    for (int k = 0; k < R; ++k) x[k] = __ldcs(in + k * V8_SUBW + c);
+                    for (int k = 0; k < R; ++k) {
+                        if constexpr (EPI) x[k] = rs_in(__ldg(in + k * V8_SUBW + c), a.rs_thr, rsc, q);
+                        else x[k] = __ldcs(in + k * V8_SUBW + c);
+                    }
                     fwd_radix<A>(x, tw, 0, 0, q, q2);
 #pragma unroll
                     for (int k = 0; k < R; ++k) out[k * V8_SUBW + c] = x[k];
@@ -131,7 +153,10 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                 {   // stage 1: layers A..A+3, thread (b, c), elements a (stride 256)
                     const int b = hi4, c = lo4;
 #pragma unroll
-                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    for (int i = 0; i < 16; ++i) {
+                        x[i] = S[v8_phys(i, b, c)];
+                        if constexpr (EPI && A == 0) x[i] = rs_in(x[i], a.rs_thr, rsc, q);
+                    }
                     fwd_radix<4>(x, tw, A, (uint32_t)s, q, q2);
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
@@ -161,10 +186,22 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     if constexpr (JIT3) fwd_radix<4>(x, tw, A + 8, (uint32_t)s * 256 + t, q, q2);
                     else fwd16_tw(x, w3, q, q2);
                     uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
+                    if constexpr (EPI) {
+                        const uint4* ai = reinterpret_cast<const uint4*>(ain + s * V8_SUBW + t * 16);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            const uint4 u = __ldcs(ai + v);
+                            __stcs(o + v, make_uint4(rs_out(u.x, umin32(x[4 * v], x[4 * v] - q2), rsc, q),
+                                                     rs_out(u.y, umin32(x[4 * v + 1], x[4 * v + 1] - q2), rsc, q),
+                                                     rs_out(u.z, umin32(x[4 * v + 2], x[4 * v + 2] - q2), rsc, q),
+                                                     rs_out(u.w, umin32(x[4 * v + 3], x[4 * v + 3] - q2), rsc, q)));
+                        }
+                    } else {
 #pragma unroll
                     for (int v = 0; v < 4; ++v)
                         __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
                                                  canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                    }
                 }
             }
             }
@@ -558,7 +595,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v10(NttArgs a, const uint8_t* G, 
     constexpr int NS = 16 / CL;
     const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
     const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
-    extern __shared__ __align__(1024) uint32_t smem[];
+    extern __shared__ __align__(1024) uint32_t smem_v10[];
+    uint32_t* const smem = smem_v10;
     uint8_t* Bt = reinterpret_cast<uint8_t*>(smem + 2 * V8_SUBW);
     uint64_t* bar = reinterpret_cast<uint64_t*>(Bt + 4096);
     uint32_t* tslot = reinterpret_cast<uint32_t*>(bar + 1);

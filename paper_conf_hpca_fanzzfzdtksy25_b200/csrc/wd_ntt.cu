@@ -23,6 +23,7 @@
 #include "ntt_cluster.cuh"
 #include "ntt_tensor.cuh"
 #include "ntt_fused.cuh"
+#include "ntt_rns.cuh"
 #include "plan_math.h"
 
 using namespace wd;
@@ -46,6 +47,9 @@ struct wd_ntt_plan {
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
     uint2* d_inv = nullptr;        // [L][N]  (psi^-brv(i), Shoup)
     LimbConst* d_lc = nullptr;     // [L]
+    uint4* d_rs = nullptr;         // [L] RESCALE constants vs the last prime (ntt_rns.cuh); L >= 2
+    uint32_t rs_thr = 0;           // q_last - floor(q_last / 2)
+    bool rs_ok = false;            // L >= 2 and q_last differs from every other prime
     TensorTables tc;               // tensor-path planes (ntt_tensor.cuh)
     int mode = WD_MODE_AUTO;
     float tensor_share = 0.5f;
@@ -89,6 +93,9 @@ int prep_cc() {
             set_smem(ntt_v8<LOGN, true, false, 0, 6>, V8_SMEM) || set_smem(ntt_v8<LOGN, false, false, 0, 6>, V8_SMEM) ||
             set_smem(ntt_v8<LOGN, false, true, 0, 6>, V8_SMEM))
             return WD_ECUDA;
+    }
+    if constexpr (LOGN >= 12) {
+        if (set_smem(ntt_v8<LOGN, true, false, 0, 4, (LOGN > 12 ? 2 : 1), 1>, V8_SMEM)) return WD_ECUDA;
     }
     if constexpr (LOGN == 16) {
         if (set_smem(ntt_v10<true, false, 1>, V10_SMEM) || set_smem(ntt_v10<false, false, 1>, V10_SMEM) ||
@@ -160,7 +167,7 @@ constexpr int V8_DEFAULT_MINB = 4;   // measured, see DESIGN.md 5.1
 constexpr int V8_DEFAULT_CL = 2;
 
 // v8 with a CL-CTA cluster per row: grid = resident clusters x CL
-template <int LOGN, int MINB, int CL>
+template <int LOGN, int MINB, int CL, int EPI = 0>
 void launch_v8_cluster(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     if constexpr ((1 << (LOGN - 12)) % CL != 0) {
         return;
@@ -171,7 +178,7 @@ void launch_v8_cluster(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s
         at[0].id = cudaLaunchAttributeClusterDimension;
         at[0].val.clusterDim.x = CL; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
         cfg.attrs = at; cfg.numAttrs = 1;
-        auto kf = ntt_v8<LOGN, true, false, 0, MINB, CL>;
+        auto kf = ntt_v8<LOGN, true, false, 0, MINB, CL, EPI>;
         auto ki = ntt_v8<LOGN, false, false, 0, MINB, CL>;
         auto kp = ntt_v8<LOGN, false, true, 0, MINB, CL>;
         auto k = fwd ? kf : (a.in2 ? kp : ki);
@@ -207,6 +214,13 @@ void launch_v9(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
 // v10 (ntt_v8.cuh, N = 2^16): v8 with the column phase on the tensor cores; 2-CTA cluster per row
 template <int CL>
 void launch_v10(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s);
+
+// v8 forward with an epilogue variant (EPI, ntt_rns.cuh), one CTA per row (N = 2^12)
+template <int LOGN, int EPI>
+void launch_v8_minb_epi(const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
+    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * 4));
+    ntt_v8<LOGN, true, false, 0, 4, 1, EPI><<<grid, V8_T, V8_SMEM, s>>>(a, rows);
+}
 
 // v8 (ntt_v8.cuh): persistent grid of min(rows, SMs x MINB) 256-thread CTAs
 template <int LOGN, int MINB>
@@ -457,7 +471,7 @@ void free_plan(wd_ntt_plan* p) {
         int cur = -1;
         cudaGetDevice(&cur);
         if (cur != p->device) cudaSetDevice(p->device);
-        cudaFree(p->d_fwd); cudaFree(p->d_inv); cudaFree(p->d_lc);
+        cudaFree(p->d_fwd); cudaFree(p->d_inv); cudaFree(p->d_lc); cudaFree(p->d_rs);
         free_tensor_tables(p->tc);
         for (auto& s : p->hs) if (s) cudaStreamDestroy(s);
         for (auto& e : p->he) if (e) cudaEventDestroy(e);
@@ -524,6 +538,23 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
         cudaMemcpy(p->d_lc, lc.data(), sizeof(LimbConst) * L, cudaMemcpyHostToDevice) != cudaSuccess) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
+    // RESCALE constants (row f4): per limb i < L-1 {-q_last mod q_i, Shoup(1), q_last^-1 mod q_i, Shoup}
+    if (L >= 2) {
+        const uint32_t ql = primes[L - 1];
+        std::vector<uint4> rs(L, make_uint4(0, 0, 0, 0));
+        p->rs_ok = true;
+        for (uint32_t i = 0; i + 1 < L; ++i) {
+            const uint32_t q = primes[i];
+            if (q == ql) { p->rs_ok = false; break; }
+            const uint32_t inv = pm_pow(ql % q, q - 2, q);
+            rs[i] = make_uint4((q - ql % q) % q, pm_shoup(1, q), inv, pm_shoup(inv, q));
+        }
+        p->rs_thr = ql - ql / 2;
+        if (p->rs_ok && (cudaMalloc(&p->d_rs, sizeof(uint4) * L) != cudaSuccess ||
+                         cudaMemcpy(p->d_rs, rs.data(), sizeof(uint4) * L, cudaMemcpyHostToDevice) != cudaSuccess)) {
+            cudaGetLastError(); free_plan(p); set_err(WD_ENOMEM); return nullptr;
+        }
+    }
     if (build_tensor_tables(p->tc, p->logN, p->primes, p->psi) != WD_OK) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
@@ -554,6 +585,47 @@ int wd_ntt_pointwise_inverse(const wd_ntt_plan* p, const uint32_t* a, const uint
     if (!a || !b) return set_err(WD_EINVAL);
     return run(p, false, a, b, out, batch, (cudaStream_t)s);
 }
+int wd_rescale(const wd_ntt_plan* p, const uint32_t* in, uint32_t* out, uint32_t batch, uint32_t* work,
+               wd_stream_t st) {
+    g_last_launches = 0;
+    if (!p || !in || !out || !work) return set_err(WD_EINVAL);
+    if (((uintptr_t)in | (uintptr_t)out | (uintptr_t)work) & 15) return set_err(WD_EINVAL);
+    if (p->L < 2 || p->logN < 12 || !p->rs_ok) return set_err(WD_EUNSUPPORTED);
+    if (batch == 0) return set_err(WD_OK);
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) return set_err(WD_EINVAL);
+    if ((uint64_t)batch * p->L > 0x7fffffffull) return set_err(WD_EINVAL);
+    cudaStream_t s = (cudaStream_t)st;
+    const uint32_t N = p->N, L = p->L;
+    // K1: last-limb rows -> work
+    {
+        const uint32_t n4 = N / 4;
+        const uint32_t blocks = (uint32_t)std::min<uint64_t>(((uint64_t)batch * n4 + 255) / 256, (uint64_t)p->sm_count * 8);
+        rs_gather<<<blocks, 256, 0, s>>>(reinterpret_cast<const uint4*>(in), reinterpret_cast<uint4*>(work), n4, L, batch);
+    }
+    // K2: INTT of the last limb (a 1-limb view of the plan's tables), in place in work
+    NttArgs ai;
+    ai.in = work; ai.in2 = nullptr; ai.out = work; ai.tw = p->d_inv + (size_t)(L - 1) * N; ai.lc = p->d_lc + (L - 1); ai.L = 1;
+    uint32_t launches = 1 + (uint32_t)launch_cuda_core(p, false, ai, batch, s);
+    // K3: forward NTT of every output row with the rescale load / store maps (v8, EPI = 1)
+    NttArgs af;
+    af.in = work; af.in2 = nullptr; af.out = out; af.tw = p->d_fwd; af.lc = p->d_lc; af.L = L - 1;
+    af.aux = in; af.rs = p->d_rs; af.rs_thr = p->rs_thr; af.Lfull = L;
+    const uint32_t rows = batch * (L - 1);
+    switch (p->logN) {
+        case 12: launch_v8_minb_epi<12, 1>(af, rows, p->sm_count, s); break;
+        case 13: launch_v8_cluster<13, 4, 2, 1>(true, af, rows, s); break;
+        case 14: launch_v8_cluster<14, 4, 2, 1>(true, af, rows, s); break;
+        case 15: launch_v8_cluster<15, 4, 2, 1>(true, af, rows, s); break;
+        case 16: launch_v8_cluster<16, 4, 2, 1>(true, af, rows, s); break;
+        default: launch_v8_cluster<17, 4, 2, 1>(true, af, rows, s); break;
+    }
+    launches += 1;
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    g_last_launches = launches;
+    return set_err(WD_OK);
+}
+
 int wd_ntt_forward_host(const wd_ntt_plan* p, const uint32_t* h_in, uint32_t* h_out, uint32_t batch,
                         uint32_t* d_work, wd_stream_t s) {
     return run_host(p, true, h_in, h_out, batch, d_work, (cudaStream_t)s);

@@ -46,6 +46,7 @@ _SIGS = {
     "wd_ntt_forward_host": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_ntt_inverse_host": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_ntt_pointwise_inverse": (_i32, [_vp, _vp, _vp, _vp, _u32, _vp]),
+    "wd_rescale": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_ntt_plan_n": (_u32, [_vp]),
     "wd_ntt_plan_limbs": (_u32, [_vp]),
     "wd_ntt_plan_psi": (_u32, [_vp, _u32]),
@@ -121,6 +122,10 @@ def wd_ntt_inverse(plan: int, inp, out, batch: int, stream=None) -> int:
 def wd_ntt_pointwise_inverse(plan: int, a, b, out, batch: int, stream=None) -> int:
     return _check(_lib.wd_ntt_pointwise_inverse(plan, _ptr(a), _ptr(b), _ptr(out), batch, _stream(stream, a)),
                   "wd_ntt_pointwise_inverse")
+
+
+def wd_rescale(plan: int, inp, out, batch: int, work, stream=None) -> int:
+    return _check(_lib.wd_rescale(plan, _ptr(inp), _ptr(out), batch, _ptr(work), _stream(stream, inp)), "wd_rescale")
 
 
 def wd_ntt_forward_host(plan: int, h_in, h_out, batch: int, d_work, stream=None) -> int:
@@ -217,6 +222,17 @@ class Plan:
     def pointwise_inverse(self, a, b, out=None, stream=None):
         out = a if out is None else out
         wd_ntt_pointwise_inverse(self.handle, a, b, out, self._batch(a), stream)
+        return out
+
+    def rescale(self, x, out=None, work=None, stream=None):
+        """[B][L][N] NTT-domain -> [B][L-1][N] NTT-domain, round(x / primes[-1]) (wd_rescale)."""
+        import torch
+        b = self._batch(x)
+        if out is None:
+            out = torch.empty((b, self.L - 1, self.N), dtype=x.dtype, device=x.device)
+        if work is None:
+            work = torch.empty((b, self.N), dtype=x.dtype, device=x.device)
+        wd_rescale(self.handle, x, out, b, work, stream)
         return out
 
     def close(self):

@@ -1,0 +1,108 @@
+"""GPU parity of the RNS operations around the NTT vs oracle/rns.py.
+
+RESCALE is exact integer arithmetic with one canonical answer, so every comparison is
+bit-exact: against the step-by-step RNS oracle everywhere, and against the big-int CRT
+definition (round(A / q_last)) on the small cases.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+from oracle import rns  # noqa: E402
+from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs  # noqa: E402
+
+P = inputs.bench_primes(60)
+SMALL = [786433, 269221889, 537133057, 805961729]
+
+
+@pytest.fixture(scope="module")
+def wd():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import wdntt
+    return wdntt
+
+
+def to_dev(x: np.ndarray):
+    return torch.from_numpy(np.ascontiguousarray(x).view(np.int32)).cuda()
+
+
+def to_host(t) -> np.ndarray:
+    return t.cpu().numpy().view(np.uint32)
+
+
+def gpu_rescale(wd, plan, x):
+    o = plan.rescale(to_dev(x))
+    torch.cuda.synchronize()
+    return to_host(o)
+
+
+@pytest.mark.parametrize("logn,L,batch", [(12, 2, 3), (12, 5, 2), (13, 4, 3), (14, 3, 2), (15, 3, 2), (16, 4, 2),
+                                          (17, 3, 1)])
+def test_rescale_vs_rns_oracle(wd, logn, L, batch):
+    n = 1 << logn
+    primes = P[:L]
+    x = inputs.uniform_residues(primes, n, batch, 8000 + logn * 10 + L)
+    plan = wd.Plan(n, primes)
+    assert np.array_equal(gpu_rescale(wd, plan, x), rns.rescale_rns(x, primes)), (logn, L)
+
+
+def test_rescale_vs_definition_small(wd):
+    n = 1 << 12
+    primes = [P[3], SMALL[1], P[0]]
+    x = inputs.uniform_residues(primes, n, 2, 8100)
+    plan = wd.Plan(n, primes)
+    assert np.array_equal(gpu_rescale(wd, plan, x), rns.rescale_definition(x, primes))
+
+
+@pytest.mark.parametrize("primes", [[SMALL[0], P[1], SMALL[3], P[2]], [P[5], SMALL[2], SMALL[0]], [SMALL[0], P[7]]])
+def test_rescale_prime_sizes(wd, primes):
+    n = 1 << 16
+    x = inputs.uniform_residues(primes, n, 2, 8200 + len(primes))
+    plan = wd.Plan(n, primes)
+    assert np.array_equal(gpu_rescale(wd, plan, x), rns.rescale_rns(x, primes))
+    for kind in ("zeros", "qm1", "alt"):
+        s = inputs.structured(kind, primes, n)
+        assert np.array_equal(gpu_rescale(wd, plan, s), rns.rescale_rns(s, primes)), kind
+
+
+def test_rescale_many_rows(wd):
+    # more output rows than resident CTAs: every CTA walks several rows
+    n, primes = 1 << 13, P[:9]
+    x = inputs.uniform_residues(primes, n, 90, 8300)
+    plan = wd.Plan(n, primes)
+    assert np.array_equal(gpu_rescale(wd, plan, x), rns.rescale_rns(x, primes))
+
+
+def test_rescale_full_size_sampled(wd):
+    # BASELINE config 3 shape (N = 2^16, L = 36, 128 polynomials): sampled polynomials vs the oracle
+    n, L, batch = 1 << 16, 36, 128
+    primes = P[:L]
+    x = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 2, device="cuda")
+    plan = wd.Plan(n, primes)
+    o = plan.rescale(x)
+    torch.cuda.synchronize()
+    for b in (0, 77, 127):
+        xb = to_host(x[b:b + 1])
+        assert np.array_equal(to_host(o[b:b + 1]), rns.rescale_rns(xb, primes)), b
+
+
+def test_rescale_errors(wd):
+    n = 1 << 12
+    x = to_dev(inputs.uniform_residues(P[:1], n, 1, 1))
+    plan1 = wd.Plan(n, P[:1])
+    with pytest.raises(wd.WdNttError):
+        wd.wd_rescale(plan1.handle, x, x, 1, x)               # L = 1: nothing to divide by
+    plan = wd.Plan(n, P[:3])
+    y = to_dev(inputs.uniform_residues(P[:3], n, 1, 2))
+    out = torch.empty((1, 2, n), dtype=torch.int32, device="cuda")
+    work = torch.empty((1, n), dtype=torch.int32, device="cuda")
+    wd.wd_rescale(plan.handle, y, out, 0, work)                # batch 0: no-op
+    with pytest.raises(wd.WdNttError):
+        wd.wd_rescale(plan.handle, y, out, 1, None)            # no work buffer
+    dup = wd.Plan(n, [P[0], P[1], P[0]])                       # q_last repeated: no inverse
+    with pytest.raises(wd.WdNttError):
+        wd.wd_rescale(dup.handle, to_dev(inputs.uniform_residues([P[0], P[1], P[0]], n, 1, 3)), out, 1, work)
