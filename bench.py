@@ -228,6 +228,58 @@ def run_rescale(args):
     print(json.dumps(line), flush=True)
 
 
+def run_modupdown(args):
+    """--op modup|moddown: the KeySwitch basis changes (row f3) at the config shape (default c3:
+    N=2^16, a = L = 36 ciphertext limbs, k = --k special primes, 128 polynomials).  One step = one
+    ModUp (a -> a+k limbs) or ModDown (a+k -> a) of every polynomial; value = polynomials/s.
+    Roofline: HBM, algorithmic bytes = read + write of the polynomial (ModUp: a*N*4 in,
+    (a+k)*N*4 out; ModDown: (a+k)*N*4 in, a*N*4 out)."""
+    import torch
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt
+    torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+    logn, a, nct = CONFIGS[args.config]
+    n = 1 << logn
+    batch = 1 if nct is None else 2 * nct
+    allp = inputs.bench_primes(a + args.k)
+    qs, ps = allp[:a], allp[a:]
+    pq, pp = wdntt.Plan(n, qs), wdntt.Plan(n, ps)
+    conv = wdntt.RnsConv(pq, pp)
+    up = args.op == "modup"
+    lin, lout = (a, a + args.k) if up else (a + args.k, a)
+    x = inputs.uniform_residues_torch(qs if up else allp, n, batch, inputs.SEED_BASE + 2, device="cuda")
+    out = torch.empty((batch, lout, n), dtype=x.dtype, device="cuda")
+    work = torch.empty((batch, a + args.k, n), dtype=x.dtype, device="cuda")
+    sp = torch.cuda.current_stream().cuda_stream
+    fn = wdntt.wd_modup if up else wdntt.wd_moddown
+    for _ in range(max(3, args.warmup)):
+        fn(conv.handle, x, out, batch, work, sp)
+    torch.cuda.synchronize()
+    launches = 0
+    with ClockSampler(0) as clk:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(args.steps):
+            fn(conv.handle, x, out, batch, work, sp)
+            launches += wdntt.wd_ntt_last_launches()
+        e1.record()
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    pk, pk_kind = peaks()
+    hbm = float(pk.get("hbm_gbs", FALLBACK_HBM_GBS))
+    alg = batch * n * 4.0 * (lin + lout)
+    line = {"metric": "CKKS %s throughput (N=2^%d, %d -> %d limbs)" % ("ModUp" if up else "ModDown", logn, lin, lout),
+            "value": batch / (ms / 1e3), "unit": "polynomials/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic (splitmix64 uniform residues)",
+            "config": {"workload": "%s: %s of %d polynomials, a=%d, k=%d" % (CONFIG_NAMES[args.config], args.op, batch,
+                                                                           a, args.k), "N": n, "polys": batch},
+            "roofline": {"bound": "hbm", "kernel": "whole op", "achieved": alg / (ms / 1e3) / 1e9, "peak": hbm,
+                         "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None, "peak_kind": pk_kind,
+                         "algorithmic_bytes_per_step": alg},
+            "gpu_launches": launches, "clocks": clk.summary()}
+    print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -240,11 +292,16 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
-    ap.add_argument("--op", default="ntt", choices=["ntt", "rescale"],
-                    help="ntt: the headline forward+inverse step; rescale: SURVEY.md 8 row f4")
+    ap.add_argument("--op", default="ntt", choices=["ntt", "rescale", "modup", "moddown"],
+                    help="ntt: the headline forward+inverse step; rescale: SURVEY.md 8 row f4; "
+                         "modup / moddown: row f3 (KeySwitch basis changes)")
+    ap.add_argument("--k", type=int, default=1, help="special primes for --op modup/moddown (PAPER.md Table III: K=1)")
     args = ap.parse_args()
     if args.op == "rescale":
         run_rescale(args)
+        return
+    if args.op in ("modup", "moddown"):
+        run_modupdown(args)
         return
 
     if args.impl == "reference":

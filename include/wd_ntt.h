@@ -142,6 +142,36 @@ int wd_ntt_pointwise_inverse(const wd_ntt_plan* plan, const uint32_t* a, const u
 int wd_rescale(const wd_ntt_plan* plan, const uint32_t* in, uint32_t* out, uint32_t batch,
                uint32_t* work, wd_stream_t stream);
 
+/*
+ * ModUp / ModDown -- SURVEY.md 8 row f3 (NEXT #3): the KeySwitch basis changes
+ * around the NTT (Table III, Fig. 4 "PE kernel"
+ * for ModUp and ModDown), in the standard RNS-CKKS form (DESIGN.md reading
+ * C-19).  A conversion object pairs a plan over the ciphertext basis
+ * Q = {q_0..q_{a-1}} with a plan over the special basis P = {p_0..p_{k-1}}
+ * (same N >= 2^12, same device, all a + k primes distinct, a, k <= 64).
+ *   BConv_{Q->P}(x)_j = sum_i [x_i (Q/q_i)^-1]_{q_i} (Q/q_i) mod p_j
+ *   wd_modup:   in  [batch][a][N]   NTT domain over Q
+ *               out [batch][a+k][N] NTT domain over Q then P: the Q limbs of
+ *               `in` unchanged, the P limbs NTT_P(BConv(INTT_Q(in)))
+ *               work >= batch*a*N words
+ *   wd_moddown: in  [batch][a+k][N] NTT domain over Q then P
+ *               out [batch][a][N]   (in_Q - NTT_Q(BConv_{P->Q}(INTT_P(in_P)))) * P^-1
+ *               work >= batch*(a+k)*N words
+ * out must not overlap in or work.  Three launches each (plus one 2-D copy in
+ * ModUp), every polynomial of the batch in each.  Errors as for the
+ * transforms; wd_rns_conv_create returns NULL (WD_EINVAL: NULL plan or a
+ * repeated prime; WD_EUNSUPPORTED: N/device mismatch, N < 2^12, > 64 limbs;
+ * WD_ENOMEM).  The conversion object references the two plans: destroy it
+ * before them.
+ */
+typedef struct wd_rns_conv wd_rns_conv;
+wd_rns_conv* wd_rns_conv_create(const wd_ntt_plan* plan_q, const wd_ntt_plan* plan_p);
+void wd_rns_conv_destroy(wd_rns_conv* conv);
+int wd_modup(const wd_rns_conv* conv, const uint32_t* in, uint32_t* out, uint32_t batch,
+             uint32_t* work, wd_stream_t stream);
+int wd_moddown(const wd_rns_conv* conv, const uint32_t* in, uint32_t* out, uint32_t batch,
+               uint32_t* work, wd_stream_t stream);
+
 /* ---- queries and knobs ---- */
 uint32_t wd_ntt_plan_n(const wd_ntt_plan* plan);
 uint32_t wd_ntt_plan_limbs(const wd_ntt_plan* plan);

@@ -39,7 +39,14 @@ struct NttArgs {
     const uint4* rs = nullptr;       // [L] {-q_last mod q_i, Shoup(1), q_last^-1 mod q_i, Shoup}
     uint32_t rs_thr = 0;             // q_last - floor(q_last / 2)
     uint32_t Lfull = 0;
+    // v8 only: rows between consecutive polynomials in `in` / `out` (0 = L, contiguous); lets a
+    // launch cover a limb SECTION of a wider [batch][Lfull][N] tensor (ModUp / ModDown, ntt_rns.cuh)
+    uint32_t in_ls = 0, out_ls = 0;
 };
+
+__device__ __forceinline__ uint32_t row_map(uint32_t row, uint32_t L, uint32_t ls) {
+    return ls ? (row / L) * ls + row % L : row;
+}
 
 constexpr int RS = 272;       // padded row stride (words) of 256-wide rows in SMEM
 

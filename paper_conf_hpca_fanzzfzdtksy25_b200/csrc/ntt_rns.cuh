@@ -30,3 +30,66 @@ __global__ void __launch_bounds__(256) rs_gather(const uint4* __restrict__ in, u
 }
 
 }  // namespace wd
+
+// ---------------------------------------------------------------------------------------------
+// Fast basis conversion (ModUp / ModDown; reading C-19):
+//   out_j = sum_i [x_i * (Q/q_i)^-1]_{q_i} * [(Q/q_i) mod p_j]  mod p_j,  coefficient domain.
+// One thread per (polynomial, coefficient): the S source residues are scaled (Shoup) into shared
+// memory, then each of the D outputs is a 64-bit multiply-accumulate over them, reduced every 15
+// terms (15 * 2^60 + 2^30 < 2^64) with a 64-bit Barrett step.  Loads and stores walk the
+// coefficient index across the warp, so every access is a coalesced 128-byte line.
+namespace wd {
+
+constexpr int BC_T = 128;                 // coefficients per CTA
+constexpr int BC_MAX = 64;                // max source / target limbs
+
+struct BconvTab {
+    const uint4* src;       // [S] {q_i, (Q/q_i)^-1 mod q_i, Shoup, 0}
+    const uint32_t* w;      // [S][D] (Q/q_i) mod p_j
+    const uint4* dst;       // [D] {p_j, mu_lo, mu_hi, 0}: mu = floor((2^64 - 1) / p_j)
+    uint32_t S, D;
+};
+
+__device__ __forceinline__ uint32_t reduce64(uint64_t v, uint32_t p, uint64_t mu) {
+    const uint64_t quo = __umul64hi(v, mu);
+    uint64_t r = v - quo * p;                 // < 3p
+    while (r >= p) r -= p;
+    return (uint32_t)r;
+}
+
+// x: [batch][x_ls][N] (source limbs start at row 0 of each polynomial's block);
+// y: [batch][y_ls][N], targets written at rows y_off .. y_off + D - 1 of each block
+__global__ void __launch_bounds__(BC_T) rns_bconv(const uint32_t* __restrict__ x, uint32_t x_ls,
+                                                  uint32_t* __restrict__ y, uint32_t y_ls, uint32_t y_off,
+                                                  BconvTab tab, uint32_t N, uint32_t batch) {
+    extern __shared__ uint32_t bsm[];
+    uint32_t* ys = bsm;                                  // [S][BC_T]
+    uint32_t* ws = bsm + tab.S * BC_T;                   // [S][D]
+    for (uint32_t i = threadIdx.x; i < tab.S * tab.D; i += BC_T) ws[i] = tab.w[i];
+    const uint32_t per_poly = N / BC_T;
+    __syncthreads();
+    for (uint32_t blk = blockIdx.x; blk < batch * per_poly; blk += gridDim.x) {
+        const uint32_t b = blk / per_poly, n = (blk % per_poly) * BC_T + threadIdx.x;
+        const uint32_t* xb = x + (size_t)b * x_ls * N + n;
+        for (uint32_t i = 0; i < tab.S; ++i) {
+            const uint4 s = tab.src[i];
+            const uint32_t v = shoup_mul(__ldcs(xb + (size_t)i * N), s.y, s.z, s.x);
+            ys[i * BC_T + threadIdx.x] = canon2(v, s.x);
+        }
+        uint32_t* yb = y + ((size_t)b * y_ls + y_off) * N + n;
+        for (uint32_t j = 0; j < tab.D; ++j) {
+            const uint4 d = tab.dst[j];
+            const uint64_t mu = ((uint64_t)d.z << 32) | d.y;
+            uint64_t acc = 0;
+            uint32_t i = 0;
+            while (i < tab.S) {
+                const uint32_t e = min(tab.S, i + 15);
+                for (; i < e; ++i) acc += (uint64_t)ys[i * BC_T + threadIdx.x] * ws[i * tab.D + j];
+                acc = reduce64(acc, d.x, mu);
+            }
+            __stcs(yb + (size_t)j * N, (uint32_t)acc);
+        }
+    }
+}
+
+}  // namespace wd

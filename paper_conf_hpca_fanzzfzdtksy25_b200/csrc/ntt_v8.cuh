@@ -91,6 +91,8 @@ __device__ __forceinline__ uint32_t rs_out(uint32_t aval, uint32_t y, const uint
     return canon2(shoup_mul(aval + 2 * q - y, r.z, r.w, q), q);
 }
 
+// EPI (forward only): 0 = plain NTT; 1 = RESCALE (shared last-limb input row through rs_in, output
+// through rs_out against aux); 2 = ModDown (plain input rows, output through rs_out against aux)
 template <int LOGN, bool FWD, bool PW, int ONLY = 0, int MINB = 4, int CL = 1, int EPI = 0>
 __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
     constexpr bool JIT3 = MINB > 4;
@@ -112,8 +114,8 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
         const LimbConst lc = a.lc[limb];
         const uint32_t q = lc.q, q2 = lc.q2;
         const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
-        const uint32_t* in = a.in + ((size_t)(EPI ? row / a.L : row) << LOGN);
-        uint32_t* out = a.out + ((size_t)row << LOGN);
+        const uint32_t* in = a.in + ((size_t)(EPI == 1 ? row / a.L : row_map(row, a.L, a.in_ls)) << LOGN);
+        uint32_t* out = a.out + ((size_t)row_map(row, a.L, a.out_ls) << LOGN);
         uint4 rsc = make_uint4(0, 0, 0, 0);
         const uint32_t* ain = nullptr;
         if constexpr (EPI) {
@@ -130,7 +132,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     uint32_t x[R];
 #pragma unroll
                     for (int k = 0; k < R; ++k) {
-                        if constexpr (EPI) x[k] = rs_in(__ldg(in + k * V8_SUBW + c), a.rs_thr, rsc, q);
+                        if constexpr (EPI == 1) x[k] = rs_in(__ldg(in + k * V8_SUBW + c), a.rs_thr, rsc, q);
                         else x[k] = __ldcs(in + k * V8_SUBW + c);
                     }
                     fwd_radix<A>(x, tw, 0, 0, q, q2);
@@ -155,7 +157,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
 #pragma unroll
                     for (int i = 0; i < 16; ++i) {
                         x[i] = S[v8_phys(i, b, c)];
-                        if constexpr (EPI && A == 0) x[i] = rs_in(x[i], a.rs_thr, rsc, q);
+                        if constexpr (EPI == 1 && A == 0) x[i] = rs_in(x[i], a.rs_thr, rsc, q);
                     }
                     fwd_radix<4>(x, tw, A, (uint32_t)s, q, q2);
 #pragma unroll

@@ -95,7 +95,9 @@ int prep_cc() {
             return WD_ECUDA;
     }
     if constexpr (LOGN >= 12) {
-        if (set_smem(ntt_v8<LOGN, true, false, 0, 4, (LOGN > 12 ? 2 : 1), 1>, V8_SMEM)) return WD_ECUDA;
+        if (set_smem(ntt_v8<LOGN, true, false, 0, 4, (LOGN > 12 ? 2 : 1), 1>, V8_SMEM) ||
+            set_smem(ntt_v8<LOGN, true, false, 0, 4, (LOGN > 12 ? 2 : 1), 2>, V8_SMEM))
+            return WD_ECUDA;
     }
     if constexpr (LOGN == 16) {
         if (set_smem(ntt_v10<true, false, 1>, V10_SMEM) || set_smem(ntt_v10<false, false, 1>, V10_SMEM) ||
@@ -482,6 +484,80 @@ void free_plan(wd_ntt_plan* p) {
 
 }  // namespace
 
+// ---------------------------------------------------------------- ModUp / ModDown (row f3)
+struct wd_rns_conv {
+    const wd_ntt_plan* pq = nullptr;   // Q basis (a limbs)
+    const wd_ntt_plan* pp = nullptr;   // P basis (k special limbs)
+    uint4* d_up_src = nullptr; uint32_t* d_up_w = nullptr; uint4* d_up_dst = nullptr;   // BConv Q -> P
+    uint4* d_dn_src = nullptr; uint32_t* d_dn_w = nullptr; uint4* d_dn_dst = nullptr;   // BConv P -> Q
+    uint4* d_pinv = nullptr;           // [a] {0, 0, P^-1 mod q_i, Shoup} (EPI = 2 store map)
+};
+
+namespace {
+
+void free_conv(wd_rns_conv* c) {
+    if (!c) return;
+    cudaFree(c->d_up_src); cudaFree(c->d_up_w); cudaFree(c->d_up_dst);
+    cudaFree(c->d_dn_src); cudaFree(c->d_dn_w); cudaFree(c->d_dn_dst); cudaFree(c->d_pinv);
+    delete c;
+}
+
+// host tables of BConv src -> dst: {q_i, (Q/q_i)^-1, Shoup}, (Q/q_i) mod p_j, {p_j, mu}
+void bconv_tables(const std::vector<uint32_t>& src, const std::vector<uint32_t>& dst, std::vector<uint4>& hs,
+                  std::vector<uint32_t>& hw, std::vector<uint4>& hd) {
+    const size_t S = src.size(), D = dst.size();
+    hs.resize(S); hw.resize(S * D); hd.resize(D);
+    for (size_t i = 0; i < S; ++i) {
+        uint32_t qh = 1;                                   // (Q/q_i) mod q_i
+        for (size_t k = 0; k < S; ++k) if (k != i) qh = pm_mul(qh, src[k] % src[i], src[i]);
+        const uint32_t inv = pm_pow(qh, src[i] - 2, src[i]);
+        hs[i] = make_uint4(src[i], inv, pm_shoup(inv, src[i]), 0);
+        for (size_t j = 0; j < D; ++j) {
+            uint32_t v = 1;
+            for (size_t k = 0; k < S; ++k) if (k != i) v = pm_mul(v, src[k] % dst[j], dst[j]);
+            hw[i * D + j] = v;
+        }
+    }
+    for (size_t j = 0; j < D; ++j) {
+        const uint64_t mu = ~0ull / dst[j];
+        hd[j] = make_uint4(dst[j], (uint32_t)mu, (uint32_t)(mu >> 32), 0);
+    }
+}
+
+template <typename T>
+bool upload(T** d, const std::vector<T>& h) {
+    if (cudaMalloc(d, sizeof(T) * h.size()) != cudaSuccess) return false;
+    return cudaMemcpy(*d, h.data(), sizeof(T) * h.size(), cudaMemcpyHostToDevice) == cudaSuccess;
+}
+
+// v8 launch over `rows` rows of `a` (any direction / EPI), default shape for N
+template <int EPI>
+void launch_v8_rows(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    switch (p->logN) {
+        case 12:
+            if (fwd) launch_v8_minb_epi<12, EPI>(a, rows, p->sm_count, s);
+            else launch_v8<12>(4, false, a, rows, p->sm_count, s);
+            break;
+        case 13: launch_v8_cluster<13, 4, 2, EPI>(fwd, a, rows, s); break;
+        case 14: launch_v8_cluster<14, 4, 2, EPI>(fwd, a, rows, s); break;
+        case 15: launch_v8_cluster<15, 4, 2, EPI>(fwd, a, rows, s); break;
+        case 16: launch_v8_cluster<16, 4, 2, EPI>(fwd, a, rows, s); break;
+        default: launch_v8_cluster<17, 4, 2, EPI>(fwd, a, rows, s); break;
+    }
+}
+
+int launch_bconv(const wd_ntt_plan* p, const uint32_t* x, uint32_t x_ls, uint32_t* y, uint32_t y_ls, uint32_t y_off,
+                 const BconvTab& t, uint32_t batch, cudaStream_t s) {
+    const size_t smem = sizeof(uint32_t) * (t.S * BC_T + t.S * t.D);
+    if (smem > 48 * 1024 && cudaFuncSetAttribute(rns_bconv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+        return WD_ECUDA;
+    const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)batch * (p->N / BC_T), (uint64_t)p->sm_count * 8);
+    rns_bconv<<<blocks, BC_T, smem, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch);
+    return WD_OK;
+}
+
+}  // namespace
+
 extern "C" {
 
 wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) {
@@ -623,6 +699,106 @@ int wd_rescale(const wd_ntt_plan* p, const uint32_t* in, uint32_t* out, uint32_t
     launches += 1;
     if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
     g_last_launches = launches;
+    return set_err(WD_OK);
+}
+
+wd_rns_conv* wd_rns_conv_create(const wd_ntt_plan* pq, const wd_ntt_plan* pp) {
+    if (!pq || !pp) { set_err(WD_EINVAL); return nullptr; }
+    if (pq->N != pp->N || pq->device != pp->device || pq->logN < 12 || pq->L > BC_MAX || pp->L > BC_MAX) {
+        set_err(WD_EUNSUPPORTED); return nullptr;
+    }
+    for (uint32_t a : pq->primes) {
+        for (uint32_t b : pp->primes) if (a == b) { set_err(WD_EINVAL); return nullptr; }
+    }
+    for (size_t i = 0; i < pq->primes.size(); ++i)
+        for (size_t k = i + 1; k < pq->primes.size(); ++k) if (pq->primes[i] == pq->primes[k]) { set_err(WD_EINVAL); return nullptr; }
+    for (size_t i = 0; i < pp->primes.size(); ++i)
+        for (size_t k = i + 1; k < pp->primes.size(); ++k) if (pp->primes[i] == pp->primes[k]) { set_err(WD_EINVAL); return nullptr; }
+    wd_rns_conv* c = new (std::nothrow) wd_rns_conv();
+    if (!c) { set_err(WD_ENOMEM); return nullptr; }
+    c->pq = pq; c->pp = pp;
+    std::vector<uint4> hs, hd, pinv(pq->L);
+    std::vector<uint32_t> hw;
+    bool ok = true;
+    bconv_tables(pq->primes, pp->primes, hs, hw, hd);
+    ok = ok && upload(&c->d_up_src, hs) && upload(&c->d_up_w, hw) && upload(&c->d_up_dst, hd);
+    bconv_tables(pp->primes, pq->primes, hs, hw, hd);
+    ok = ok && upload(&c->d_dn_src, hs) && upload(&c->d_dn_w, hw) && upload(&c->d_dn_dst, hd);
+    for (uint32_t i = 0; i < pq->L; ++i) {
+        const uint32_t q = pq->primes[i];
+        uint32_t P = 1;
+        for (uint32_t pj : pp->primes) P = pm_mul(P, pj % q, q);
+        const uint32_t inv = pm_pow(P, q - 2, q);
+        pinv[i] = make_uint4(0, 0, inv, pm_shoup(inv, q));
+    }
+    ok = ok && upload(&c->d_pinv, pinv);
+    if (!ok) { cudaGetLastError(); free_conv(c); set_err(WD_ENOMEM); return nullptr; }
+    set_err(WD_OK);
+    return c;
+}
+
+void wd_rns_conv_destroy(wd_rns_conv* c) { free_conv(c); }
+
+int wd_modup(const wd_rns_conv* c, const uint32_t* in, uint32_t* out, uint32_t batch, uint32_t* work, wd_stream_t st) {
+    g_last_launches = 0;
+    if (!c || !in || !out || !work) return set_err(WD_EINVAL);
+    if (((uintptr_t)in | (uintptr_t)out | (uintptr_t)work) & 15) return set_err(WD_EINVAL);
+    if (batch == 0) return set_err(WD_OK);
+    const wd_ntt_plan *pq = c->pq, *pp = c->pp;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != pq->device) return set_err(WD_EINVAL);
+    if ((uint64_t)batch * (pq->L + pp->L) > 0x7fffffffull) return set_err(WD_EINVAL);
+    cudaStream_t s = (cudaStream_t)st;
+    const uint32_t N = pq->N, a = pq->L, k = pp->L;
+    // K1: INTT of the Q limbs -> work [batch][a][N]
+    NttArgs ai;
+    ai.in = in; ai.in2 = nullptr; ai.out = work; ai.tw = pq->d_inv; ai.lc = pq->d_lc; ai.L = a;
+    uint32_t launches = (uint32_t)launch_cuda_core(pq, false, ai, batch * a, s);
+    // the Q limbs pass through unchanged (NTT domain)
+    if (cudaMemcpy2DAsync(out, (size_t)(a + k) * N * 4, in, (size_t)a * N * 4, (size_t)a * N * 4, batch,
+                          cudaMemcpyDeviceToDevice, s) != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    // K2: BConv Q -> P into the P section of out (coefficient domain)
+    BconvTab t{c->d_up_src, c->d_up_w, c->d_up_dst, a, k};
+    if (launch_bconv(pq, work, a, out, a + k, a, t, batch, s) != WD_OK) return set_err(WD_ECUDA);
+    // K3: forward NTT of the P section in place (rows strided by a + k)
+    NttArgs af;
+    af.in = out + (size_t)a * N; af.in2 = nullptr; af.out = out + (size_t)a * N; af.tw = pp->d_fwd; af.lc = pp->d_lc;
+    af.L = k; af.in_ls = a + k; af.out_ls = a + k;
+    launch_v8_rows<0>(pp, true, af, batch * k, s);
+    launches += 2;
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    g_last_launches = launches;
+    return set_err(WD_OK);
+}
+
+int wd_moddown(const wd_rns_conv* c, const uint32_t* in, uint32_t* out, uint32_t batch, uint32_t* work, wd_stream_t st) {
+    g_last_launches = 0;
+    if (!c || !in || !out || !work) return set_err(WD_EINVAL);
+    if (((uintptr_t)in | (uintptr_t)out | (uintptr_t)work) & 15) return set_err(WD_EINVAL);
+    if (batch == 0) return set_err(WD_OK);
+    const wd_ntt_plan *pq = c->pq, *pp = c->pp;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != pq->device) return set_err(WD_EINVAL);
+    if ((uint64_t)batch * (pq->L + pp->L) > 0x7fffffffull) return set_err(WD_EINVAL);
+    cudaStream_t s = (cudaStream_t)st;
+    const uint32_t N = pq->N, a = pq->L, k = pp->L;
+    uint32_t* wp = work;                                   // [batch][k][N] P-limb coefficients
+    uint32_t* wq = work + (size_t)batch * k * N;           // [batch][a][N] BConv P -> Q
+    // K1: INTT of the P section of in (rows strided by a + k) -> wp
+    NttArgs ai;
+    ai.in = in + (size_t)a * N; ai.in2 = nullptr; ai.out = wp; ai.tw = pp->d_inv; ai.lc = pp->d_lc; ai.L = k;
+    ai.in_ls = a + k;
+    launch_v8_rows<0>(pp, false, ai, batch * k, s);
+    // K2: BConv P -> Q (coefficient domain) -> wq
+    BconvTab t{c->d_dn_src, c->d_dn_w, c->d_dn_dst, k, a};
+    if (launch_bconv(pq, wp, k, wq, a, 0, t, batch, s) != WD_OK) return set_err(WD_ECUDA);
+    // K3: forward NTT over Q with the store map out = (in_Q - NTT(wq)) * P^-1 (v8, EPI = 2)
+    NttArgs af;
+    af.in = wq; af.in2 = nullptr; af.out = out; af.tw = pq->d_fwd; af.lc = pq->d_lc; af.L = a;
+    af.aux = in; af.rs = c->d_pinv; af.Lfull = a + k;
+    launch_v8_rows<2>(pq, true, af, batch * a, s);
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    g_last_launches = 3;
     return set_err(WD_OK);
 }
 

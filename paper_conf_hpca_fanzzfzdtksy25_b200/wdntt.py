@@ -47,6 +47,10 @@ _SIGS = {
     "wd_ntt_inverse_host": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_ntt_pointwise_inverse": (_i32, [_vp, _vp, _vp, _vp, _u32, _vp]),
     "wd_rescale": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
+    "wd_rns_conv_create": (_vp, [_vp, _vp]),
+    "wd_rns_conv_destroy": (None, [_vp]),
+    "wd_modup": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
+    "wd_moddown": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_ntt_plan_n": (_u32, [_vp]),
     "wd_ntt_plan_limbs": (_u32, [_vp]),
     "wd_ntt_plan_psi": (_u32, [_vp, _u32]),
@@ -126,6 +130,25 @@ def wd_ntt_pointwise_inverse(plan: int, a, b, out, batch: int, stream=None) -> i
 
 def wd_rescale(plan: int, inp, out, batch: int, work, stream=None) -> int:
     return _check(_lib.wd_rescale(plan, _ptr(inp), _ptr(out), batch, _ptr(work), _stream(stream, inp)), "wd_rescale")
+
+
+def wd_rns_conv_create(plan_q: int, plan_p: int) -> int:
+    h = _lib.wd_rns_conv_create(plan_q, plan_p)
+    if not h:
+        raise WdNttError(_lib.wd_ntt_last_error(), "wd_rns_conv_create")
+    return h
+
+
+def wd_rns_conv_destroy(conv: int) -> None:
+    _lib.wd_rns_conv_destroy(conv)
+
+
+def wd_modup(conv: int, inp, out, batch: int, work, stream=None) -> int:
+    return _check(_lib.wd_modup(conv, _ptr(inp), _ptr(out), batch, _ptr(work), _stream(stream, inp)), "wd_modup")
+
+
+def wd_moddown(conv: int, inp, out, batch: int, work, stream=None) -> int:
+    return _check(_lib.wd_moddown(conv, _ptr(inp), _ptr(out), batch, _ptr(work), _stream(stream, inp)), "wd_moddown")
 
 
 def wd_ntt_forward_host(plan: int, h_in, h_out, batch: int, d_work, stream=None) -> int:
@@ -238,6 +261,43 @@ class Plan:
     def close(self):
         if getattr(self, "handle", None):
             wd_ntt_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class RnsConv:
+    """RAII wrapper of wd_rns_conv: ModUp / ModDown between ``plan_q`` (a limbs) and ``plan_p`` (k limbs)."""
+
+    def __init__(self, plan_q: "Plan", plan_p: "Plan"):
+        self.pq, self.pp = plan_q, plan_p              # keep the plans alive
+        self.handle = wd_rns_conv_create(plan_q.handle, plan_p.handle)
+
+    def modup(self, x, out=None, work=None, stream=None):
+        import torch
+        a, k, n = self.pq.L, self.pp.L, self.pq.N
+        b = x.numel() // (a * n)
+        out = torch.empty((b, a + k, n), dtype=x.dtype, device=x.device) if out is None else out
+        work = torch.empty((b, a, n), dtype=x.dtype, device=x.device) if work is None else work
+        wd_modup(self.handle, x, out, b, work, stream)
+        return out
+
+    def moddown(self, x, out=None, work=None, stream=None):
+        import torch
+        a, k, n = self.pq.L, self.pp.L, self.pq.N
+        b = x.numel() // ((a + k) * n)
+        out = torch.empty((b, a, n), dtype=x.dtype, device=x.device) if out is None else out
+        work = torch.empty((b, a + k, n), dtype=x.dtype, device=x.device) if work is None else work
+        wd_moddown(self.handle, x, out, b, work, stream)
+        return out
+
+    def close(self):
+        if getattr(self, "handle", None):
+            wd_rns_conv_destroy(self.handle)
             self.handle = None
 
     def __del__(self):  # pragma: no cover

@@ -106,3 +106,62 @@ def test_rescale_errors(wd):
     dup = wd.Plan(n, [P[0], P[1], P[0]])                       # q_last repeated: no inverse
     with pytest.raises(wd.WdNttError):
         wd.wd_rescale(dup.handle, to_dev(inputs.uniform_residues([P[0], P[1], P[0]], n, 1, 3)), out, 1, work)
+
+
+# ---------------------------------------------------------------- ModUp / ModDown (row f3)
+QS = [P[0], P[1], P[2], SMALL[2]]
+PS = [P[40], SMALL[3], P[41]]
+
+
+@pytest.mark.parametrize("logn,a,k,batch", [(12, 4, 3, 2), (13, 3, 1, 3), (16, 4, 3, 2), (17, 2, 2, 1)])
+def test_modup_moddown_vs_oracle(wd, logn, a, k, batch):
+    n = 1 << logn
+    qs, ps = QS[:a], PS[:k]
+    if logn == 17:                                   # q = 1 mod 2^18 needed: bench primes only
+        qs, ps = P[:a], P[40:40 + k]
+    pq, pp = wd.Plan(n, qs), wd.Plan(n, ps)
+    conv = wd.RnsConv(pq, pp)
+    x = inputs.uniform_residues(qs, n, batch, 8400 + logn)
+    up = conv.modup(to_dev(x))
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(up), rns.modup(x, qs, ps)), ("modup", logn)
+    e = inputs.uniform_residues(qs + ps, n, batch, 8500 + logn)
+    dn = conv.moddown(to_dev(e))
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(dn), rns.moddown(e, qs, ps)), ("moddown", logn)
+
+
+def test_modup_moddown_keyswitch_shape(wd):
+    # the paper's KeySwitch shape (Table III: N = 2^16, l = 34 ... 36 limbs, K = 1 special prime)
+    # with a batch of 8 polynomials: ModUp 36 -> 37 limbs, ModDown 37 -> 36
+    n, a, k, batch = 1 << 16, 36, 1, 8
+    qs, ps = P[:a], P[50:50 + k]
+    pq, pp = wd.Plan(n, qs), wd.Plan(n, ps)
+    conv = wd.RnsConv(pq, pp)
+    x = inputs.uniform_residues(qs, n, batch, 8600)
+    up = to_host(conv.modup(to_dev(x)))
+    dn = to_host(conv.moddown(to_dev(up)))
+    torch.cuda.synchronize()
+    for b in (0, 5):
+        assert np.array_equal(up[b:b + 1], rns.modup(x[b:b + 1], qs, ps)), b
+        assert np.array_equal(dn[b:b + 1], rns.moddown(up[b:b + 1], qs, ps)), b
+
+
+def test_modup_many_rows_and_wide_bases(wd):
+    n, qs, ps = 1 << 13, P[:20], P[30:46]            # 20 -> 36 limbs; more rows than resident CTAs
+    pq, pp = wd.Plan(n, qs), wd.Plan(n, ps)
+    conv = wd.RnsConv(pq, pp)
+    x = inputs.uniform_residues(qs, n, 12, 8700)
+    up = to_host(conv.modup(to_dev(x)))
+    assert np.array_equal(up, rns.modup(x, qs, ps))
+    dn = to_host(conv.moddown(to_dev(up)))
+    assert np.array_equal(dn, rns.moddown(up, qs, ps))
+
+
+def test_rns_conv_errors(wd):
+    n = 1 << 12
+    pq = wd.Plan(n, P[:3])
+    with pytest.raises(wd.WdNttError):
+        wd.RnsConv(pq, wd.Plan(n, [P[2], P[9]]))            # a prime in both bases
+    with pytest.raises(wd.WdNttError):
+        wd.RnsConv(pq, wd.Plan(1 << 13, P[10:12]))          # N mismatch
