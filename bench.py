@@ -286,7 +286,7 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="wd", choices=["wd", "reference"])
-    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused"])
+    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused", "cuda_gemm"])
     ap.add_argument("--share", type=float, default=-1.0, help="tensor share for --mode fused")
     ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
     ap.add_argument("--e2e-steps", type=int, default=3)

@@ -57,6 +57,8 @@ typedef struct CUstream_st* wd_stream_t;       /* == cudaStream_t */
 #define WD_MODE_CUDA     1   /* CUDA-core radix-2^k butterflies only (WD-BO role)       */
 #define WD_MODE_TENSOR   2   /* tcgen05 kind::i8 inner DFTs + CUDA-core epilogue        */
 #define WD_MODE_FUSED    3   /* both paths concurrently on the same SMs (WD-FUSE role)  */
+#define WD_MODE_CUDA_GEMM 4  /* inner DFTs as 32-bit GEMMs on the CUDA cores (WD-CUDA,   *
+                              * PAPER.md:322/401), N = 2^16 only     */
 
 /*
  * wd_ntt_plan_create -- PAPER.md:358 (initialisation phase: moduli, twiddles

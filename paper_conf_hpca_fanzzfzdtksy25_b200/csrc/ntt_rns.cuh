@@ -45,7 +45,7 @@ constexpr int BC_MAX = 64;                // max source / target limbs
 
 struct BconvTab {
     const uint4* src;       // [S] {q_i, (Q/q_i)^-1 mod q_i, Shoup, 0}
-    const uint32_t* w;      // [S][D] (Q/q_i) mod p_j
+    const uint2* w;         // [S][D] {(Q/q_i) mod p_j, its Shoup companion mod p_j}
     const uint4* dst;       // [D] {p_j, mu_lo, mu_hi, 0}: mu = floor((2^64 - 1) / p_j)
     uint32_t S, D;
 };
@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(BC_T) rns_bconv(const uint32_t* __restrict__ x
                                                   BconvTab tab, uint32_t N, uint32_t batch) {
     extern __shared__ uint32_t bsm[];
     uint32_t* ys = bsm;                                  // [S][BC_T]
-    uint32_t* ws = bsm + tab.S * BC_T;                   // [S][D]
+    uint2* ws = reinterpret_cast<uint2*>(bsm + tab.S * BC_T);   // [S][D]
     for (uint32_t i = threadIdx.x; i < tab.S * tab.D; i += BC_T) ws[i] = tab.w[i];
     const uint32_t per_poly = N / BC_T;
     __syncthreads();
@@ -80,14 +80,27 @@ __global__ void __launch_bounds__(BC_T) rns_bconv(const uint32_t* __restrict__ x
         for (uint32_t j = 0; j < tab.D; ++j) {
             const uint4 d = tab.dst[j];
             const uint64_t mu = ((uint64_t)d.z << 32) | d.y;
-            uint64_t acc = 0;
-            uint32_t i = 0;
-            while (i < tab.S) {
-                const uint32_t e = min(tab.S, i + 15);
-                for (; i < e; ++i) acc += (uint64_t)ys[i * BC_T + threadIdx.x] * ws[i * tab.D + j];
-                acc = reduce64(acc, d.x, mu);
+            uint32_t r;
+            if (tab.S <= 4) {                            // few terms: lazy Shoup products in [0, 2p)
+                const uint32_t p2 = 2 * d.x;
+                r = 0;
+                for (uint32_t i = 0; i < tab.S; ++i) {
+                    const uint2 w = ws[i * tab.D + j];
+                    r += shoup_mul(ys[i * BC_T + threadIdx.x], w.x, w.y, d.x);
+                    r = umin32(r, r - p2);
+                }
+                r = canon2(r, d.x);
+            } else {                                     // many terms: 64-bit MACs, Barrett every 15
+                uint64_t acc = 0;
+                uint32_t i = 0;
+                while (i < tab.S) {
+                    const uint32_t e = min(tab.S, i + 15);
+                    for (; i < e; ++i) acc += (uint64_t)ys[i * BC_T + threadIdx.x] * ws[i * tab.D + j].x;
+                    acc = reduce64(acc, d.x, mu);
+                }
+                r = (uint32_t)acc;
             }
-            __stcs(yb + (size_t)j * N, (uint32_t)acc);
+            __stcs(yb + (size_t)j * N, r);
         }
     }
 }

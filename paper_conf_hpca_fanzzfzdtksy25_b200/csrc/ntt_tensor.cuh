@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <vector>
+#include <cstring>
 #include "modarith.cuh"
 #include "ntt_cuda_core.cuh"
 #include "ntt_persist.cuh"
@@ -45,6 +46,7 @@ struct TensorTables {
     uint2* d_sg2 = nullptr;        // [L][256][16]
     uint2* d_sg3 = nullptr;        // [L][4096][16]
     uint2* d_c16 = nullptr;        // [L] Shoup companions of 2^16 and of 1
+    uint32_t* d_mat = nullptr;     // [L][4][256] u32 block matrices M0, F, MI0 (N^-1), F' (WD-CUDA, row f2)
     bool ok = false;
 };
 
@@ -635,7 +637,7 @@ __global__ void __launch_bounds__(TC_T, TC_CTAS_PER_SM) ntt_tc16(TcArgs ta, uint
 // ------------------------------------------------------------------ host side
 inline void free_tensor_tables(TensorTables& t) {
     cudaFree(t.d_G); cudaFree(t.d_B); cudaFree(t.d_tw1); cudaFree(t.d_tw2); cudaFree(t.d_tw3);
-    cudaFree(t.d_sg1); cudaFree(t.d_sg2); cudaFree(t.d_sg3); cudaFree(t.d_c16);
+    cudaFree(t.d_sg1); cudaFree(t.d_sg2); cudaFree(t.d_sg3); cudaFree(t.d_c16); cudaFree(t.d_mat);
     t = TensorTables();
 }
 
@@ -648,6 +650,7 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
     std::vector<uint2> t1((size_t)L * 256), t2((size_t)L * 4096), t3((size_t)L * 65536);
     std::vector<uint2> s1((size_t)L * 256), s2((size_t)L * 4096), s3((size_t)L * 65536);
     std::vector<uint2> c16(L);
+    std::vector<uint32_t> mat((size_t)L * 4 * 256);
     for (uint32_t l = 0; l < L; ++l) {
         const uint32_t q = primes[l], psi = psis[l], psi_inv = pm_pow(psi, q - 2, q);
         std::vector<uint32_t> pw(N), pwi(N), fb(N), ib(N);
@@ -657,9 +660,11 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
         const uint32_t ninv = pm_pow(N % q, q - 2, q);
         uint32_t M[16][16], F[16][16], Fi[16][16];
         block_fwd(M, fb, 0, 0, q);
+        std::memcpy(&mat[((size_t)l * 4 + 0) * 256], M, 1024);
         byte_planes(&B[((size_t)l * 4 + 0) * 4096], M, q);
         byte_planes(&Gi[(((size_t)l * 2 + 0) * 17 + 0) * 4096], M, q);
         block_inv(M, ib, 0, 0, q, ninv);
+        std::memcpy(&mat[((size_t)l * 4 + 2) * 256], M, 1024);
         byte_planes(&B[((size_t)l * 4 + 2) * 4096], M, q);
         byte_planes(&Gi[(((size_t)l * 2 + 1) * 17 + 0) * 4096], M, q);
         for (uint32_t g = 0; g < 16; ++g) {              // stage-1 blocks, one image per group
@@ -696,6 +701,8 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
         }
         byte_planes(&B[((size_t)l * 4 + 1) * 4096], F, q);
         byte_planes(&B[((size_t)l * 4 + 3) * 4096], Fi, q);
+        std::memcpy(&mat[((size_t)l * 4 + 1) * 256], F, 1024);
+        std::memcpy(&mat[((size_t)l * 4 + 3) * 256], Fi, 1024);
         c16[l] = make_uint2(pm_shoup(65536u % q, q), pm_shoup(1u, q));
     }
     auto up = [](void** d, const void* h, size_t n) {
@@ -705,7 +712,8 @@ inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vecto
     if (!up((void**)&tc.d_G, Gi.data(), Gi.size()) || !up((void**)&tc.d_B, B.data(), B.size()) || !up((void**)&tc.d_tw1, t1.data(), t1.size() * 8) ||
         !up((void**)&tc.d_tw2, t2.data(), t2.size() * 8) || !up((void**)&tc.d_tw3, t3.data(), t3.size() * 8) ||
         !up((void**)&tc.d_sg1, s1.data(), s1.size() * 8) || !up((void**)&tc.d_sg2, s2.data(), s2.size() * 8) ||
-        !up((void**)&tc.d_sg3, s3.data(), s3.size() * 8) || !up((void**)&tc.d_c16, c16.data(), c16.size() * 8))
+        !up((void**)&tc.d_sg3, s3.data(), s3.size() * 8) || !up((void**)&tc.d_c16, c16.data(), c16.size() * 8) ||
+        !up((void**)&tc.d_mat, mat.data(), mat.size() * 4))
         return 4;
     tc.ok = true;
     return 0;

@@ -754,4 +754,206 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v10(NttArgs a, const uint8_t* G, 
     if (t < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
 }
 
+
+// ---------------------------------------------------------------------------------------------
+// WD-CUDA ("CUDA Cores ... directly compute high-precision
+// (32-bit) GEMM"): the same 4 radix-16 stages of N = 2^16 as the tensor path, but
+// every inner 16-point DFT is a 32-bit matrix-vector product on the CUDA cores --
+//   forward stage s >= 1:  x_j <- x_j * tau_g[j];  y = F x        (stage 0: y = M0 x)
+//   inverse stage s >= 1:  y = F' x;  y_k <- y_k * sigma_g[k]      (stage 0': y = MI0 x, N^-1 in MI0)
+// with the matrices and twists of the tensor tables (ntt_tensor.cuh build_tensor_tables), each
+// output a pair of 8-term 64-bit multiply-accumulates (x < 2^31, M < 2^30: < 2^64) reduced by a
+// 64-bit Barrett step.  It is the paper's comparison variant (Fig. 6): 16 wide multiplies per
+// element per stage instead of 2 Shoup butterflies, so it is expected to be slower than WD-BO.
+// Data movement is v8's (N = 16 x 4096, 2-CTA cluster per row).
+__device__ __forceinline__ uint32_t wdc_reduce(uint64_t v, const LimbConst& lc) {
+    const uint64_t quo = __umul64hi(v, lc.mu);
+    const uint32_t r = (uint32_t)(v - quo * lc.q);       // < 3q
+    return umin32(r, r - lc.q);                          // < 2q (lazy)
+}
+// y = M x (M row-major [16][16] in shared memory, broadcast reads), x_j < 2^31 -> y_k < 4q
+__device__ __forceinline__ void wdc_gemm16(uint32_t* x, const uint32_t* M, const LimbConst& lc) {
+    uint32_t y[16];
+#pragma unroll
+    for (int k = 0; k < 16; ++k) {
+        const uint4* row = reinterpret_cast<const uint4*>(M + 16 * k);
+        uint64_t a0 = 0, a1 = 0;
+#pragma unroll
+        for (int v = 0; v < 2; ++v) {
+            const uint4 m = row[v];
+            a0 += (uint64_t)x[4 * v] * m.x + (uint64_t)x[4 * v + 1] * m.y + (uint64_t)x[4 * v + 2] * m.z +
+                  (uint64_t)x[4 * v + 3] * m.w;
+        }
+#pragma unroll
+        for (int v = 2; v < 4; ++v) {
+            const uint4 m = row[v];
+            a1 += (uint64_t)x[4 * v] * m.x + (uint64_t)x[4 * v + 1] * m.y + (uint64_t)x[4 * v + 2] * m.z +
+                  (uint64_t)x[4 * v + 3] * m.w;
+        }
+        y[k] = wdc_reduce(a0, lc) + wdc_reduce(a1, lc);
+    }
+#pragma unroll
+    for (int k = 0; k < 16; ++k) x[k] = y[k];
+}
+// x_j <- x_j * t[j] (Shoup, result < 2q); t = 16 consecutive (w, w') pairs of one group
+__device__ __forceinline__ void wdc_twist(uint32_t* x, const uint2* __restrict__ t, uint32_t q) {
+#pragma unroll
+    for (int j = 0; j < 16; j += 2) {
+        const uint4 w = __ldg(reinterpret_cast<const uint4*>(t + j));
+        x[j] = shoup_mul(x[j], w.x, w.y, q);
+        x[j + 1] = shoup_mul(x[j + 1], w.z, w.w, q);
+    }
+}
+__device__ __forceinline__ uint32_t wdc_canon(uint32_t v, uint32_t q, uint32_t q2) { return canon4(v, q, q2); }
+
+struct WdcArgs {
+    NttArgs a;
+    const uint32_t* mat;     // [L][4][256]: M0, F, MI0 (with N^-1), F'
+    const uint2 *t1, *t2, *t3;   // twists of this direction: tau (forward) / sigma (inverse)
+};
+
+template <bool FWD>
+__global__ void __launch_bounds__(V8_T, 3) ntt_wdcuda16(WdcArgs wa, uint32_t rows) {
+    constexpr int LOGN = 16, CL = 2;
+    constexpr int NP = V8_SUBW / V8_T / CL, NS = 16 / CL;
+    const NttArgs& a = wa.a;
+    const int rank = (int)(blockIdx.x % CL);
+    const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
+    extern __shared__ __align__(16) uint32_t smem[];
+    uint32_t* Mst = smem + 2 * V8_SUBW;                 // [2][256]: stage-0 matrix, fixed DFT
+    const int t = threadIdx.x, hi4 = t >> 4, lo4 = t & 15;
+#pragma unroll 1
+    for (uint32_t row = blockIdx.x / CL; row < rows; row += gridDim.x / CL) {
+        const uint32_t limb = row % a.L;
+        const LimbConst lc = a.lc[limb];
+        const uint32_t q = lc.q, q2 = lc.q2;
+        const uint32_t* in = a.in + ((size_t)row << LOGN);
+        uint32_t* out = a.out + ((size_t)row << LOGN);
+        const uint32_t* mats = wa.mat + ((size_t)limb * 4 + (FWD ? 0 : 2)) * 256;
+        for (int i = t; i < 512; i += V8_T) Mst[i] = mats[i];
+        const uint2* T1 = wa.t1 + (size_t)limb * 256;
+        const uint2* T2 = wa.t2 + (size_t)limb * 4096;
+        const uint2* T3 = wa.t3 + (size_t)limb * 65536;
+        __syncthreads();
+        if constexpr (FWD) {
+#pragma unroll 1
+            for (int pass = p0; pass < p0 + NP; ++pass) {          // stage 0 on columns: y = M0 x
+                const int c = pass * V8_T + t;
+                uint32_t x[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) x[k] = __ldcs(in + k * V8_SUBW + c);
+                wdc_gemm16(x, Mst, lc);
+#pragma unroll
+                for (int k = 0; k < 16; ++k) out[k * V8_SUBW + c] = x[k];
+            }
+            cluster_sync();
+            v8_load_fwd_slice(smem, out + s0 * V8_SUBW);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
+                cp_async_wait<0>();
+                __syncwarp();
+                uint32_t x[16];
+                {   // stage 1, group s
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    wdc_twist(x, T1 + s * 16, q);
+                    wdc_gemm16(x, Mst + 256, lc);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
+                }
+                __syncthreads();
+                if (s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, out + (s + 1) * V8_SUBW);
+                {   // stage 2, group s * 16 + aa
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    wdc_twist(x, T2 + (s * 16 + aa) * 16, q);
+                    wdc_gemm16(x, Mst + 256, lc);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncwarp();
+                {   // stage 3, group s * 256 + t
+                    const int aa = hi4, b = lo4;
+                    const uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    wdc_twist(x, T3 + ((size_t)s * 256 + t) * 16, q);
+                    wdc_gemm16(x, Mst + 256, lc);
+                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        __stcs(o + v, make_uint4(wdc_canon(x[4 * v], q, q2), wdc_canon(x[4 * v + 1], q, q2),
+                                                 wdc_canon(x[4 * v + 2], q, q2), wdc_canon(x[4 * v + 3], q, q2)));
+                }
+            }
+        } else {
+            v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
+                cp_async_wait<0>();
+                __syncwarp();
+                uint32_t x[16];
+                {   // stage 3', group s * 256 + t: y = F' x, then sigma
+                    const int aa = hi4, b = lo4;
+                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    wdc_gemm16(x, Mst + 256, lc);
+                    wdc_twist(x, T3 + ((size_t)s * 256 + t) * 16, q);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                }
+                __syncwarp();
+                {   // stage 2', group s * 16 + aa
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    wdc_gemm16(x, Mst + 256, lc);
+                    wdc_twist(x, T2 + (s * 16 + aa) * 16, q);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncthreads();
+                if (s + 1 < s1) v8_load_inv_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, in + (s + 1) * V8_SUBW);
+                {   // stage 1', group s
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    wdc_gemm16(x, Mst + 256, lc);
+                    wdc_twist(x, T1 + s * 16, q);
+                    uint32_t* o = out + s * V8_SUBW + b * 16 + c;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) o[i * 256] = x[i];
+                }
+            }
+            cluster_sync();
+#pragma unroll 1
+            for (int pass = p0; pass < p0 + NP; ++pass) {          // stage 0' on columns: y = MI0 x
+                const int c = pass * V8_T + t;
+                uint32_t x[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) x[k] = out[k * V8_SUBW + c];
+                wdc_gemm16(x, Mst, lc);
+#pragma unroll
+                for (int k = 0; k < 16; ++k) __stcs(out + k * V8_SUBW + c, wdc_canon(x[k], q, q2));
+            }
+        }
+        __syncthreads();
+    }
+}
+
 }  // namespace wd

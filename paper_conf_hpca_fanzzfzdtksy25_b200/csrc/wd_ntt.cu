@@ -100,6 +100,7 @@ int prep_cc() {
             return WD_ECUDA;
     }
     if constexpr (LOGN == 16) {
+        if (set_smem(ntt_wdcuda16<true>, V8_SMEM + 2048) || set_smem(ntt_wdcuda16<false>, V8_SMEM + 2048)) return WD_ECUDA;
         if (set_smem(ntt_v10<true, false, 1>, V10_SMEM) || set_smem(ntt_v10<false, false, 1>, V10_SMEM) ||
             set_smem(ntt_v10<false, true, 1>, V10_SMEM) || set_smem(ntt_v10<true, false, 2>, V10_SMEM) ||
             set_smem(ntt_v10<false, false, 2>, V10_SMEM) || set_smem(ntt_v10<false, true, 2>, V10_SMEM))
@@ -418,7 +419,21 @@ int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2,
     a.in = in; a.in2 = in2; a.out = out; a.tw = fwd ? p->d_fwd : p->d_inv; a.lc = p->d_lc; a.L = p->L;
     const int mode = effective_mode(p);
     int launches = 0;
-    if (mode == WD_MODE_CUDA || in2 != nullptr || !tensor_supported(p->logN)) {
+    if (mode == WD_MODE_CUDA_GEMM && in2 == nullptr && p->logN == 16 && p->tc.ok) {
+        WdcArgs wa;
+        wa.a = a; wa.mat = p->tc.d_mat;
+        wa.t1 = fwd ? p->tc.d_tw1 : p->tc.d_sg1; wa.t2 = fwd ? p->tc.d_tw2 : p->tc.d_sg2; wa.t3 = fwd ? p->tc.d_tw3 : p->tc.d_sg3;
+        cudaLaunchConfig_t cfg = {};
+        cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM + 2048; cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+        cfg.attrs = at; cfg.numAttrs = 1;
+        cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)(p->sm_count * 3 / 2)) * 2);
+        if (fwd) cudaLaunchKernelEx(&cfg, ntt_wdcuda16<true>, wa, rows);
+        else cudaLaunchKernelEx(&cfg, ntt_wdcuda16<false>, wa, rows);
+        launches = 1;
+    } else if (mode == WD_MODE_CUDA || mode == WD_MODE_CUDA_GEMM || in2 != nullptr || !tensor_supported(p->logN)) {
         if (mode != WD_MODE_CUDA && in2 == nullptr && mode != WD_MODE_AUTO) return set_err(WD_EUNSUPPORTED);
         launches = launch_cuda_core(p, fwd, a, rows, s);
     } else {
@@ -488,8 +503,8 @@ void free_plan(wd_ntt_plan* p) {
 struct wd_rns_conv {
     const wd_ntt_plan* pq = nullptr;   // Q basis (a limbs)
     const wd_ntt_plan* pp = nullptr;   // P basis (k special limbs)
-    uint4* d_up_src = nullptr; uint32_t* d_up_w = nullptr; uint4* d_up_dst = nullptr;   // BConv Q -> P
-    uint4* d_dn_src = nullptr; uint32_t* d_dn_w = nullptr; uint4* d_dn_dst = nullptr;   // BConv P -> Q
+    uint4* d_up_src = nullptr; uint2* d_up_w = nullptr; uint4* d_up_dst = nullptr;      // BConv Q -> P
+    uint4* d_dn_src = nullptr; uint2* d_dn_w = nullptr; uint4* d_dn_dst = nullptr;      // BConv P -> Q
     uint4* d_pinv = nullptr;           // [a] {0, 0, P^-1 mod q_i, Shoup} (EPI = 2 store map)
 };
 
@@ -504,7 +519,7 @@ void free_conv(wd_rns_conv* c) {
 
 // host tables of BConv src -> dst: {q_i, (Q/q_i)^-1, Shoup}, (Q/q_i) mod p_j, {p_j, mu}
 void bconv_tables(const std::vector<uint32_t>& src, const std::vector<uint32_t>& dst, std::vector<uint4>& hs,
-                  std::vector<uint32_t>& hw, std::vector<uint4>& hd) {
+                  std::vector<uint2>& hw, std::vector<uint4>& hd) {
     const size_t S = src.size(), D = dst.size();
     hs.resize(S); hw.resize(S * D); hd.resize(D);
     for (size_t i = 0; i < S; ++i) {
@@ -515,7 +530,7 @@ void bconv_tables(const std::vector<uint32_t>& src, const std::vector<uint32_t>&
         for (size_t j = 0; j < D; ++j) {
             uint32_t v = 1;
             for (size_t k = 0; k < S; ++k) if (k != i) v = pm_mul(v, src[k] % dst[j], dst[j]);
-            hw[i * D + j] = v;
+            hw[i * D + j] = make_uint2(v, pm_shoup(v, dst[j]));
         }
     }
     for (size_t j = 0; j < D; ++j) {
@@ -548,7 +563,7 @@ void launch_v8_rows(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t r
 
 int launch_bconv(const wd_ntt_plan* p, const uint32_t* x, uint32_t x_ls, uint32_t* y, uint32_t y_ls, uint32_t y_off,
                  const BconvTab& t, uint32_t batch, cudaStream_t s) {
-    const size_t smem = sizeof(uint32_t) * (t.S * BC_T + t.S * t.D);
+    const size_t smem = sizeof(uint32_t) * t.S * BC_T + sizeof(uint2) * t.S * t.D;
     if (smem > 48 * 1024 && cudaFuncSetAttribute(rns_bconv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
         return WD_ECUDA;
     const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)batch * (p->N / BC_T), (uint64_t)p->sm_count * 8);
@@ -718,7 +733,7 @@ wd_rns_conv* wd_rns_conv_create(const wd_ntt_plan* pq, const wd_ntt_plan* pp) {
     if (!c) { set_err(WD_ENOMEM); return nullptr; }
     c->pq = pq; c->pp = pp;
     std::vector<uint4> hs, hd, pinv(pq->L);
-    std::vector<uint32_t> hw;
+    std::vector<uint2> hw;
     bool ok = true;
     bconv_tables(pq->primes, pp->primes, hs, hw, hd);
     ok = ok && upload(&c->d_up_src, hs) && upload(&c->d_up_w, hw) && upload(&c->d_up_dst, hd);
@@ -825,8 +840,9 @@ int wd_ntt_check_prime(uint32_t q, uint32_t N) {
 }
 
 int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
-    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_FUSED) return set_err(WD_EINVAL);
-    if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED) && !tensor_supported(p->logN)) return set_err(WD_EUNSUPPORTED);
+    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_CUDA_GEMM) return set_err(WD_EINVAL);
+    if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED || mode == WD_MODE_CUDA_GEMM) && !tensor_supported(p->logN))
+        return set_err(WD_EUNSUPPORTED);
     if (tensor_share > 1.0f) return set_err(WD_EINVAL);
     p->mode = mode;
     if (tensor_share >= 0.0f) p->tensor_share = tensor_share;

@@ -308,3 +308,20 @@ def test_prime_sizes_n16(wd, ver, monkeypatch):
     q = np.repeat(inputs.structured("qm1", primes, n), 3, axis=0)
     assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes)), ver
     assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes)), ver
+
+
+# -------------------------------------------------------------- WD-CUDA (row f2): 32-bit GEMM inner DFTs
+def test_wd_cuda_gemm_mode(wd):
+    n = 1 << 16
+    primes = [P[0], P[33], 786433, 269221889, 805961729]
+    x = inputs.uniform_residues(primes, n, 3, 5300)
+    plan = wd.Plan(n, primes, mode="cuda_gemm")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes))
+    assert np.array_equal(gpu_inv(wd, plan, y), x)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes))
+    q = np.repeat(inputs.structured("qm1", primes, n), 3, axis=0)
+    assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes))
+    assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes))
+    with pytest.raises(wd.WdNttError):
+        wd.Plan(1 << 15, P[:2], mode="cuda_gemm")          # N = 2^16 only
