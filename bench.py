@@ -44,6 +44,7 @@ CONFIG_NAMES = {"c1": "config1 (BASELINE configs[0])", "c2": "config2 (one ciphe
 CONFIG_NAMES.update({"s%d" % _lg: "config5 sweep point N=2^%d, L=16, 128 polynomials" % _lg for _lg in range(12, 18)})
 METRIC = "NTT KOPS (N=2^16, L=36) at 1/2/4/8 B200; % of HBM / int8 tensor roofline"
 FALLBACK_HBM_GBS = 6650.0
+BFLY_PER_CLK_SM = 13.57       # measured: scripts/int_probe.cu ct_bfly_hi, 4 CTAs/SM (profiles/r01/int_probe.jsonl)
 
 
 def peaks():
@@ -224,7 +225,19 @@ def run_rescale(args):
             "roofline": {"bound": "hbm", "kernel": "whole op (3 launches)", "achieved": alg / (ms / 1e3) / 1e9,
                          "peak": hbm, "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None,
                          "peak_kind": pk_kind, "algorithmic_bytes_per_step": alg},
-            "gpu_launches": launches, "clocks": clk.summary()}
+            # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
+        # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
+        # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
+        # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
+        "roofline_alu": {"bound": "alu", "kernel": dom_name,
+                         "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
+                         "peak": BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3,
+                         "unit": "G butterflies/s",
+                         "frac": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9
+                                 / (BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3),
+                         "note": "algorithmic butterflies (N/2 log2 N per transform); the WD-CUDA and tensor "
+                                 "modes do other work per element, for them this is a normalised rate"},
+        "gpu_launches": launches, "clocks": clk.summary()}
     print(json.dumps(line), flush=True)
 
 
@@ -276,7 +289,19 @@ def run_modupdown(args):
             "roofline": {"bound": "hbm", "kernel": "whole op", "achieved": alg / (ms / 1e3) / 1e9, "peak": hbm,
                          "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None, "peak_kind": pk_kind,
                          "algorithmic_bytes_per_step": alg},
-            "gpu_launches": launches, "clocks": clk.summary()}
+            # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
+        # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
+        # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
+        # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
+        "roofline_alu": {"bound": "alu", "kernel": dom_name,
+                         "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
+                         "peak": BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3,
+                         "unit": "G butterflies/s",
+                         "frac": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9
+                                 / (BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3),
+                         "note": "algorithmic butterflies (N/2 log2 N per transform); the WD-CUDA and tensor "
+                                 "modes do other work per element, for them this is a normalised rate"},
+        "gpu_launches": launches, "clocks": clk.summary()}
     print(json.dumps(line), flush=True)
 
 
@@ -439,6 +464,18 @@ def main():
                      "frac": achieved / hbm, "traffic": traffic,
                      "peak_kind": "%s (MEASURED_PEAKS.json hbm_gbs copy bandwidth)" % pk_kind,
                      "algorithmic_bytes_per_launch": alg_bytes},
+        # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
+        # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
+        # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
+        # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
+        "roofline_alu": {"bound": "alu", "kernel": dom_name,
+                         "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
+                         "peak": BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3,
+                         "unit": "G butterflies/s",
+                         "frac": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9
+                                 / (BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3),
+                         "note": "algorithmic butterflies (N/2 log2 N per transform); the WD-CUDA and tensor "
+                                 "modes do other work per element, for them this is a normalised rate"},
         "gpu_launches": launches,
         "occupancy_ctas_per_sm": {"cuda_fwd": wdntt.wd_ntt_occupancy(plan.handle, "cuda", True),
                                   "cuda_inv": wdntt.wd_ntt_occupancy(plan.handle, "cuda", False),

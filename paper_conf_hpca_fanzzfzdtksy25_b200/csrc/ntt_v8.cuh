@@ -956,4 +956,326 @@ __global__ void __launch_bounds__(V8_T, 3) ntt_wdcuda16(WdcArgs wa, uint32_t row
     }
 }
 
+
+// ---------------------------------------------------------------------------------------------
+// v11 (N = 2^16): v8's data movement with the ROW-phase radix-16 stages on the tensor cores.
+// Within a 4096-word sub-row s (elements a*256 + b*16 + c) the three stages are
+//   stage 1 (layers 4..7,  group s):            folded matrix M1_s (twist inside, no extra work)
+//   stage 2 (layers 8..11, group s*16 + a):      M = F diag(tau2_g)  -> Shoup twist, then fixed F
+//   stage 3 (layers 12..15, group s*256 + a*16 + b): M = F diag(tau3_g)
+// (inverse: MI1_s, and F' followed by the sigma twist), i.e. the tensor tables' factorisation,
+// over 256 instances = 2 MMA tiles of 128 per stage.  TMASK selects which of the three stages run
+// on the tensor cores (bit st-1); the others keep v8's butterflies, and the column phase (layers
+// 0..3) is always v8's register-only butterflies, so the tensor pipe of one CTA's row phase
+// overlaps the CUDA-core butterflies of the other CTAs on the SM.  Per
+// tile: every warp moves 32 instances x 8 coefficients smem -> registers (conflict-free in v8's
+// layout) -> TMEM (tcgen05.st), one thread issues 2 MMAs, every warp reads back its 8 outputs x
+// 4 planes (tcgen05.ld), recombines and writes them in place (or to global, forward stage 3).
+constexpr int V11_SMEM = V8_SMEM + 3 * 4096 + 64;    // sub-rows, B: F/F' + 2 x M1_s/MI1_s, mbarrier
+
+struct V11Args {
+    NttArgs a;
+    const uint8_t* G;        // [L][2][17][4096] byte planes: [0] M0/MI0, [1+g] M1_g/MI1_g
+    const uint8_t* B;        // [L][4][4096]: M0, F, MI0, F'
+    const uint2 *t2, *t3;    // twists of this direction (tau forward / sigma inverse), stages 2, 3
+    const uint2* c16;
+};
+
+template <bool FWD, int ST>
+__device__ __forceinline__ void v11_stage(uint32_t* S, uint32_t* gout, uint32_t tmem, uint32_t bimg,
+                                          uint64_t* bar, uint32_t& ph, const uint2* __restrict__ tws,
+                                          uint32_t q, uint32_t q2, uint32_t c16s, uint32_t one_s) {
+    const int t = threadIdx.x, w = t >> 5, lane = t & 31;
+    const int lq = w & 3, h = w >> 2;
+    const uint32_t tl = tmem + ((uint32_t)(32 * lq) << 16);
+#pragma unroll 1
+    for (int tt = 0; tt < 2; ++tt) {
+        const int i = tt * 128 + lq * 32 + lane;          // instance (u, v) = (i >> 4, i & 15)
+        const int u = i >> 4, v = i & 15;
+        uint32_t x[8];
+        if constexpr (ST == 1) {
+#pragma unroll
+            for (int jj = 0; jj < 8; ++jj) x[jj] = S[v8_phys(8 * h + jj, u, v)];
+        } else if constexpr (ST == 2) {
+#pragma unroll
+            for (int jj = 0; jj < 8; ++jj) x[jj] = S[v8_phys(u, 8 * h + jj, v)];
+        } else {
+            const uint32_t* base = S + u * 256 + ((v ^ (u & 1)) << 4);
+            const int sw = (v >> 1) & 3;
+#pragma unroll
+            for (int vv = 0; vv < 2; ++vv) {
+                const uint4 g = *reinterpret_cast<const uint4*>(base + (((2 * h + vv) ^ sw) << 2));
+                x[4 * vv] = g.x; x[4 * vv + 1] = g.y; x[4 * vv + 2] = g.z; x[4 * vv + 3] = g.w;
+            }
+        }
+        if constexpr (FWD && ST >= 2) {                    // x_j <- x_j * tau_g[j]
+            const uint4* tp = reinterpret_cast<const uint4*>(tws + (size_t)(ST == 2 ? u : i) * 16 + 8 * h);
+#pragma unroll
+            for (int jj = 0; jj < 8; jj += 2) {
+                const uint4 tw = __ldg(tp + jj / 2);
+                x[jj] = shoup_mul(x[jj], tw.x, tw.y, q);
+                x[jj + 1] = shoup_mul(x[jj + 1], tw.z, tw.w, q);
+            }
+        }
+        tmem_st8(tl + 8 * h, x);
+        tmem_wait_st();
+        tc_fence_before();
+        __syncthreads();                                   // A complete; previous tile's D read
+        if (t == 0) {
+            tc_fence_after();
+            tc_mma_ts(tmem + 64, tmem, umma_desc(bimg), 0);
+            tc_mma_ts(tmem + 64, tmem + 8, umma_desc(bimg + 256), 1);
+            tc_commit(bar);
+        }
+        uint4 sg[4];
+        if constexpr (!FWD && ST >= 2) {                   // sigma_g[k], k = 8h .. 8h+7, in flight
+            const uint4* sp = reinterpret_cast<const uint4*>(tws + (size_t)(ST == 2 ? u : i) * 16 + 8 * h);
+#pragma unroll
+            for (int k2 = 0; k2 < 4; ++k2) sg[k2] = __ldg(sp + k2);
+        }
+        mbar_wait(bar, ph);
+        ph ^= 1;
+        tc_fence_after();
+        uint32_t d[32];
+        tmem_ld32(tl + 64 + 32 * h, d);
+        tmem_wait_ld();
+        tc_fence_before();
+        uint32_t y[8];
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk) {
+            y[kk] = v10_combine(d + 4 * kk, q, q2, c16s, one_s);        // [0, 4q)
+            if constexpr (!FWD && ST >= 2)
+                y[kk] = shoup_mul(y[kk], (kk & 1) ? sg[kk / 2].z : sg[kk / 2].x, (kk & 1) ? sg[kk / 2].w : sg[kk / 2].y, q);
+            if constexpr (!FWD && ST == 1) y[kk] = umin32(y[kk], y[kk] - q2);   // GS column phase wants [0, 2q)
+        }
+        if constexpr (ST == 1) {
+#pragma unroll
+            for (int kk = 0; kk < 8; ++kk) S[v8_phys(8 * h + kk, u, v)] = y[kk];
+        } else if constexpr (ST == 2) {
+#pragma unroll
+            for (int kk = 0; kk < 8; ++kk) S[v8_phys(u, 8 * h + kk, v)] = y[kk];
+        } else if (FWD) {
+            uint4* o = reinterpret_cast<uint4*>(gout + i * 16 + 8 * h);
+#pragma unroll
+            for (int vv = 0; vv < 2; ++vv)
+                __stcs(o + vv, make_uint4(canon4(y[4 * vv], q, q2), canon4(y[4 * vv + 1], q, q2),
+                                          canon4(y[4 * vv + 2], q, q2), canon4(y[4 * vv + 3], q, q2)));
+        } else {
+            uint32_t* base = S + u * 256 + ((v ^ (u & 1)) << 4);
+            const int sw = (v >> 1) & 3;
+#pragma unroll
+            for (int vv = 0; vv < 2; ++vv)
+                *reinterpret_cast<uint4*>(base + (((2 * h + vv) ^ sw) << 2)) =
+                    make_uint4(y[4 * vv], y[4 * vv + 1], y[4 * vv + 2], y[4 * vv + 3]);
+        }
+    }
+    __syncthreads();                                       // the stage's results visible to every warp
+}
+
+template <bool FWD, int TMASK, int CL = 2>
+__global__ void __launch_bounds__(V8_T, 4) ntt_v11(V11Args va, uint32_t rows) {
+    constexpr int LOGN = 16, A = 4;
+    constexpr int NP = V8_SUBW / V8_T / CL, NS = 16 / CL;
+    constexpr bool T1 = TMASK & 1, T2 = TMASK & 2, T3 = TMASK & 4;
+    const NttArgs& a = va.a;
+    const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
+    const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
+    extern __shared__ __align__(1024) uint32_t smem_v11[];
+    uint32_t* const smem = smem_v11;
+    uint8_t* Bf = reinterpret_cast<uint8_t*>(smem + 2 * V8_SUBW);       // F / F'
+    uint8_t* B1 = Bf + 4096;                                            // [2] M1_s / MI1_s
+    uint64_t* bar = reinterpret_cast<uint64_t*>(Bf + 3 * 4096);
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(bar + 1);
+    const int t = threadIdx.x, hi4 = t >> 4, lo4 = t & 15;
+    if (t == 0) {
+        mbar_init(bar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (t < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tslot;
+    uint32_t ph = 0;
+#pragma unroll 1
+    for (uint32_t row = blockIdx.x / CL; row < rows; row += gridDim.x / CL) {
+        const uint32_t limb = row % a.L;
+        const LimbConst lc = a.lc[limb];
+        const uint32_t q = lc.q, q2 = lc.q2;
+        const uint2 cc = va.c16[limb];
+        const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+        const uint32_t* in = a.in + ((size_t)row << LOGN);
+        uint32_t* out = a.out + ((size_t)row << LOGN);
+        const uint8_t* Gl = va.G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096;
+        const uint2* tw2 = va.t2 + (size_t)limb * 4096;
+        const uint2* tw3 = va.t3 + (size_t)limb * 65536;
+        if constexpr (TMASK != 0) {                                       // F / F' of this limb
+            cp_async16(Bf + 16 * t, va.B + ((size_t)limb * 4 + (FWD ? 1 : 3)) * 4096 + 16 * t);
+            cp_async_commit();
+        }
+        auto load_b1 = [&](int s) {                                      // M1_s / MI1_s
+            if constexpr (T1) {
+                cp_async16(B1 + ((s - s0) & 1) * 4096 + 16 * t, Gl + (1 + s) * 4096 + 16 * t);
+                cp_async_commit();
+            }
+        };
+        if constexpr (FWD) {
+#pragma unroll 1
+            for (int pass = p0; pass < p0 + NP; ++pass) {                   // phase 1 (v8)
+                const int c = pass * V8_T + t;
+                uint32_t x[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) x[k] = __ldcs(in + k * V8_SUBW + c);
+                fwd_radix<A>(x, tw, 0, 0, q, q2);
+#pragma unroll
+                for (int k = 0; k < 16; ++k) out[k * V8_SUBW + c] = x[k];
+            }
+            if constexpr (CL > 1) cluster_sync(); else __syncthreads();
+            v8_load_fwd_slice(smem, out + s0 * V8_SUBW);
+            load_b1(s0);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
+                cp_async_wait<0>();
+                if constexpr (TMASK != 0) fence_async_smem();
+                if constexpr (T1) __syncthreads(); else __syncwarp();
+                uint32_t x[16];
+                if constexpr (T1) {
+                    v11_stage<true, 1>(S, nullptr, tmem, smem_addr(B1 + ((s - s0) & 1) * 4096), bar, ph, nullptr,
+                                       q, q2, cc.x, cc.y);
+                } else {
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    fwd_radix<4>(x, tw, A, (uint32_t)s, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
+                    __syncthreads();
+                }
+                if (s + 1 < s1) {
+                    v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, out + (s + 1) * V8_SUBW);
+                    load_b1(s + 1);
+                }
+                if constexpr (T2) {
+                    v11_stage<true, 2>(S, nullptr, tmem, smem_addr(Bf), bar, ph, tw2 + (size_t)s * 16 * 16,
+                                       q, q2, cc.x, cc.y);
+                } else {
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    fwd_radix<4>(x, tw, A + 4, (uint32_t)s * 16 + aa, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                    if constexpr (T3) __syncthreads(); else __syncwarp();
+                }
+                if constexpr (T3) {
+                    v11_stage<true, 3>(S, out + s * V8_SUBW, tmem, smem_addr(Bf), bar, ph, tw3 + (size_t)s * 256 * 16,
+                                       q, q2, cc.x, cc.y);
+                } else {
+                    uint2 w3[15];
+                    load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                    const int aa = hi4, b = lo4;
+                    const uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    fwd16_tw(x, w3, q, q2);
+                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
+                                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                }
+            }
+        } else {
+            v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+            load_b1(s0);
+#pragma unroll 1
+            for (int s = s0; s < s1; ++s) {
+                uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
+                cp_async_wait<0>();
+                if constexpr (TMASK != 0) fence_async_smem();
+                if constexpr (T3) __syncthreads(); else __syncwarp();
+                uint32_t x[16];
+                if constexpr (T3) {
+                    v11_stage<false, 3>(S, nullptr, tmem, smem_addr(Bf), bar, ph, tw3 + (size_t)s * 256 * 16,
+                                        q, q2, cc.x, cc.y);
+                } else {
+                    uint2 w3[15];
+                    load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                    const int aa = hi4, b = lo4;
+                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
+                    }
+                    inv16_tw(x, w3, q, q2);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                    if constexpr (T2) __syncthreads(); else __syncwarp();
+                }
+                if constexpr (T2) {
+                    v11_stage<false, 2>(S, nullptr, tmem, smem_addr(Bf), bar, ph, tw2 + (size_t)s * 16 * 16,
+                                        q, q2, cc.x, cc.y);
+                } else {
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    inv_radix<4, false>(x, tw, A + 4, (uint32_t)s * 16 + aa, lc);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                    __syncthreads();
+                }
+                if (s + 1 < s1) {
+                    v8_load_inv_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, in + (s + 1) * V8_SUBW);
+                    load_b1(s + 1);
+                }
+                if constexpr (T1) {
+                    // MI1_s of THIS sub-row: its group was committed with sub-row s (waited above)
+                    v11_stage<false, 1>(S, nullptr, tmem, smem_addr(B1 + ((s - s0) & 1) * 4096), bar, ph, nullptr,
+                                        q, q2, cc.x, cc.y);
+                    const int b = hi4, c = lo4;
+                    uint32_t* o = out + s * V8_SUBW + b * 16 + c;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) o[i * 256] = S[v8_phys(i, b, c)];
+                } else {
+                    const int b = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
+                    inv_radix<4, false>(x, tw, A, (uint32_t)s, lc);
+                    uint32_t* o = out + s * V8_SUBW + b * 16 + c;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) o[i * 256] = x[i];
+                }
+            }
+            if constexpr (CL > 1) cluster_sync(); else __syncthreads();
+#pragma unroll 1
+            for (int pass = p0; pass < p0 + NP; ++pass) {                   // phase 1' (v8)
+                const int c = pass * V8_T + t;
+                uint32_t x[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) x[k] = out[k * V8_SUBW + c];
+                inv_radix<A, true>(x, tw, 0, 0, lc);
+#pragma unroll
+                for (int k = 0; k < 16; ++k) __stcs(out + k * V8_SUBW + c, canon2(x[k], q));
+            }
+        }
+        __syncthreads();
+    }
+    cp_async_wait<0>();
+    tc_fence_before();
+    __syncthreads();
+    if (t < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
+}
+
 }  // namespace wd

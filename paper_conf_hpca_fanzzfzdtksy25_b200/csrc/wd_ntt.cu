@@ -101,6 +101,11 @@ int prep_cc() {
     }
     if constexpr (LOGN == 16) {
         if (set_smem(ntt_wdcuda16<true>, V8_SMEM + 2048) || set_smem(ntt_wdcuda16<false>, V8_SMEM + 2048)) return WD_ECUDA;
+        if (set_smem(ntt_v11<true, 1>, V11_SMEM) || set_smem(ntt_v11<false, 1>, V11_SMEM) ||
+            set_smem(ntt_v11<true, 3>, V11_SMEM) || set_smem(ntt_v11<false, 3>, V11_SMEM) ||
+            set_smem(ntt_v11<true, 6>, V11_SMEM) || set_smem(ntt_v11<false, 6>, V11_SMEM) ||
+            set_smem(ntt_v11<true, 7>, V11_SMEM) || set_smem(ntt_v11<false, 7>, V11_SMEM))
+            return WD_ECUDA;
         if (set_smem(ntt_v10<true, false, 1>, V10_SMEM) || set_smem(ntt_v10<false, false, 1>, V10_SMEM) ||
             set_smem(ntt_v10<false, true, 1>, V10_SMEM) || set_smem(ntt_v10<true, false, 2>, V10_SMEM) ||
             set_smem(ntt_v10<false, false, 2>, V10_SMEM) || set_smem(ntt_v10<false, true, 2>, V10_SMEM))
@@ -217,6 +222,7 @@ void launch_v9(bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
 // v10 (ntt_v8.cuh, N = 2^16): v8 with the column phase on the tensor cores; 2-CTA cluster per row
 template <int CL>
 void launch_v10(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s);
+void launch_v11(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s);
 
 // v8 forward with an epilogue variant (EPI, ntt_rns.cuh), one CTA per row (N = 2^12)
 template <int LOGN, int EPI>
@@ -273,6 +279,10 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         // AUTO at or above the SM count: v8 (see DESIGN.md 5.1 for the measured (CTAs/SM,
         // cluster) choice; WD_NTT_MINB / WD_NTT_CL override it for A/B runs)
         if constexpr (LOGN == 16) {
+            if (p->kernel_ver == 11 && p->tc.ok && a.in2 == nullptr) {
+                launch_v11(p, fwd, a, rows, s);
+                return;
+            }
             if (p->kernel_ver == 10 && p->tc.ok) {
                 if ((p->v8_cl ? p->v8_cl : V8_DEFAULT_CL) >= 2) launch_v10<2>(p, fwd, a, rows, s);
                 else launch_v10<1>(p, fwd, a, rows, s);
@@ -379,6 +389,33 @@ void launch_v10(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows,
     }
     cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)ncl) * CL);
     cudaLaunchKernelEx(&cfg, k, a, (const uint8_t*)p->tc.d_G, (const uint2*)p->tc.d_c16, rows);
+}
+
+// v11: which row-phase stages run on the tensor cores (bit st-1); WD_NTT_TMASK overrides
+template <int TM>
+void launch_v11_tm(const wd_ntt_plan* p, bool fwd, const V11Args& va, uint32_t rows, cudaStream_t s) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V11_SMEM; cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+    cfg.attrs = at; cfg.numAttrs = 1;
+    cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)(p->sm_count * 2)) * 2);   // 4 CTAs / SM (TMEM: 4 x 128)
+    if (fwd) cudaLaunchKernelEx(&cfg, ntt_v11<true, TM>, va, rows);
+    else cudaLaunchKernelEx(&cfg, ntt_v11<false, TM>, va, rows);
+}
+void launch_v11(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    V11Args va;
+    va.a = a; va.G = p->tc.d_G; va.B = p->tc.d_B; va.c16 = p->tc.d_c16;
+    va.t2 = fwd ? p->tc.d_tw2 : p->tc.d_sg2; va.t3 = fwd ? p->tc.d_tw3 : p->tc.d_sg3;
+    int tm = 7;
+    if (const char* ev = getenv("WD_NTT_TMASK")) tm = atoi(ev);
+    switch (tm) {
+        case 1: launch_v11_tm<1>(p, fwd, va, rows, s); break;
+        case 3: launch_v11_tm<3>(p, fwd, va, rows, s); break;
+        case 6: launch_v11_tm<6>(p, fwd, va, rows, s); break;
+        default: launch_v11_tm<7>(p, fwd, va, rows, s); break;
+    }
 }
 
 int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {

@@ -249,7 +249,7 @@ def test_modes_headline_config(wd, mode, share):
 
 
 # -------------------------------------------------------------- every CUDA-core kernel generation
-@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8", "v9", "v10"])
+@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8", "v9", "v10", "v11"])
 @pytest.mark.parametrize("logn", [12, 13, 14, 15, 16, 17])
 def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
@@ -276,7 +276,7 @@ def test_cuda_core_generations(wd, ver, logn, monkeypatch):
 # More rows than resident CTAs (clusters), so every CTA walks several rows and the cross-row
 # prefetches (v9: next row's first unit staged during the current row) are exercised; the row
 # count is ragged with respect to the grid.
-@pytest.mark.parametrize("ver", ["v8", "v9", "v10"])
+@pytest.mark.parametrize("ver", ["v8", "v9", "v10", "v11"])
 @pytest.mark.parametrize("logn,batch", [(14, 161), (16, 83)])
 def test_persistent_many_rows(wd, ver, logn, batch, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
@@ -293,7 +293,7 @@ def test_persistent_many_rows(wd, ver, logn, batch, monkeypatch):
 # Primes across the range the ABI accepts: the tensor column phase (v10) recombines its byte
 # planes with a cheaper reduction when q > 2^29 and a general one below; both must be exact.
 # 786433 = 3 * 2^18 + 1; the others are the first primes = 1 (mod 2^17) above 2^28, 2^29, 1.5*2^29.
-@pytest.mark.parametrize("ver", ["v8", "v10"])
+@pytest.mark.parametrize("ver", ["v8", "v10", "v11"])
 def test_prime_sizes_n16(wd, ver, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
     n = 1 << 16
@@ -325,3 +325,19 @@ def test_wd_cuda_gemm_mode(wd):
     assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes))
     with pytest.raises(wd.WdNttError):
         wd.Plan(1 << 15, P[:2], mode="cuda_gemm")          # N = 2^16 only
+
+
+# v11: every tensor / butterfly split of the row phase (bit st-1 of WD_NTT_TMASK = stage st on the
+# tensor cores), over more rows than resident CTAs
+@pytest.mark.parametrize("tmask", ["1", "3", "6", "7"])
+def test_v11_stage_splits(wd, tmask, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", "v11")
+    monkeypatch.setenv("WD_NTT_TMASK", tmask)
+    n = 1 << 16
+    primes = [P[2], P[31], 786433, 537133057]
+    x = inputs.uniform_residues(primes, n, 80, 5400 + int(tmask))
+    plan = wd.Plan(n, primes, mode="cuda")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), tmask
+    assert np.array_equal(gpu_inv(wd, plan, y), x), tmask
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), tmask
