@@ -250,9 +250,10 @@ template <int LOGN>
 void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     using S = CcShape<LOGN>;
     if constexpr (LOGN >= 14) {
-        // measured: a row split over a CTA cluster wins when there are fewer rows than SMs
-        // (config 2: one ciphertext = 72 rows -> 1648 vs 1010 KOPS); one row per CTA wins above
-        const bool small = p->kernel_ver == 0 && rows < (uint32_t)p->sm_count && (LOGN == 15 || LOGN == 16);
+        // measured: a row split over a 4-CTA cluster (v5) wins only for a handful of rows; from
+        // a quarter of the SM count up v8's 2-CTA clusters win (config 2, one ciphertext = 72
+        // rows at N = 2^16: v8 2006 vs v5 1681 KOPS, profiles/r01/ab/)
+        const bool small = p->kernel_ver == 0 && rows < (uint32_t)p->sm_count / 4 && (LOGN == 15 || LOGN == 16);
         if (p->kernel_ver == 5 || small) {
             constexpr int CLN = 1 << (LOGN - 14);
             const uint32_t units = std::max<uint32_t>(1, std::min<uint32_t>(rows, (uint32_t)(2 * p->sm_count / CLN)));
@@ -295,7 +296,8 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             else launch_v9<LOGN, 1>(fwd, a, rows, s);
             return;
         }
-        const bool autov8 = p->kernel_ver == 0 && rows >= (uint32_t)p->sm_count;
+        const bool autov8 = p->kernel_ver == 0 && (rows >= (uint32_t)p->sm_count ||
+                                                   ((LOGN == 15 || LOGN == 16) && rows >= (uint32_t)p->sm_count / 4));
         if (p->kernel_ver == 8 || autov8) {
             int minb = p->v8_minb ? p->v8_minb : V8_DEFAULT_MINB;
             int cl = p->v8_cl ? p->v8_cl : V8_DEFAULT_CL;
