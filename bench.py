@@ -225,19 +225,7 @@ def run_rescale(args):
             "roofline": {"bound": "hbm", "kernel": "whole op (3 launches)", "achieved": alg / (ms / 1e3) / 1e9,
                          "peak": hbm, "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None,
                          "peak_kind": pk_kind, "algorithmic_bytes_per_step": alg},
-            # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
-        # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
-        # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
-        # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
-        "roofline_alu": {"bound": "alu", "kernel": dom_name,
-                         "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
-                         "peak": BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3,
-                         "unit": "G butterflies/s",
-                         "frac": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9
-                                 / (BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3),
-                         "note": "algorithmic butterflies (N/2 log2 N per transform); the WD-CUDA and tensor "
-                                 "modes do other work per element, for them this is a normalised rate"},
-        "gpu_launches": launches, "clocks": clk.summary()}
+            "gpu_launches": launches, "clocks": clk.summary()}
     print(json.dumps(line), flush=True)
 
 
@@ -289,19 +277,7 @@ def run_modupdown(args):
             "roofline": {"bound": "hbm", "kernel": "whole op", "achieved": alg / (ms / 1e3) / 1e9, "peak": hbm,
                          "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None, "peak_kind": pk_kind,
                          "algorithmic_bytes_per_step": alg},
-            # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
-        # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
-        # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
-        # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
-        "roofline_alu": {"bound": "alu", "kernel": dom_name,
-                         "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
-                         "peak": BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3,
-                         "unit": "G butterflies/s",
-                         "frac": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9
-                                 / (BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3),
-                         "note": "algorithmic butterflies (N/2 log2 N per transform); the WD-CUDA and tensor "
-                                 "modes do other work per element, for them this is a normalised rate"},
-        "gpu_launches": launches, "clocks": clk.summary()}
+            "gpu_launches": launches, "clocks": clk.summary()}
     print(json.dumps(line), flush=True)
 
 

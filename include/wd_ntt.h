@@ -167,6 +167,24 @@ int wd_rescale(const wd_ntt_plan* plan, const uint32_t* in, uint32_t* out, uint3
  * before them.
  */
 typedef struct wd_rns_conv wd_rns_conv;
+/*
+ * Limb-sharded ModUp (SURVEY.md 8 rows e + f3: the one step of the path with a real exchange).
+ * Rank g holds a shard of the Q limbs; plan_q covers that shard and q_all (a_all primes,
+ * host array, read during the call) is the whole basis Q.  wd_modup_partial INTTs the local
+ * limbs and writes this shard's share of BConv_{Q->P} with the whole-Q constants as
+ * canonical residues in 64-bit words, partial [batch][k][N] (device).  The caller sums the
+ * shards' partials (an integer all-reduce, e.g. NCCL ncclSum on int64), then
+ * wd_modup_finish reduces the sums mod p_j into out_p [batch][k][N] and NTTs them: the P
+ * limbs of ModUp, identical on every rank.  ModDown needs no exchange when the P limbs are
+ * replicated: wd_moddown on a shard conversion object produces the local Q limbs.
+ * wd_modup itself refuses a shard object (WD_EINVAL).  work >= batch*a_local*N words.
+ */
+wd_rns_conv* wd_rns_conv_create_shard(const wd_ntt_plan* plan_q_local, const wd_ntt_plan* plan_p,
+                                      const uint32_t* q_all, uint32_t a_all);
+int wd_modup_partial(const wd_rns_conv* conv, const uint32_t* in_local, uint64_t* partial,
+                     uint32_t batch, uint32_t* work, wd_stream_t stream);
+int wd_modup_finish(const wd_rns_conv* conv, const uint64_t* sum, uint32_t* out_p,
+                    uint32_t batch, wd_stream_t stream);
 wd_rns_conv* wd_rns_conv_create(const wd_ntt_plan* plan_q, const wd_ntt_plan* plan_p);
 void wd_rns_conv_destroy(wd_rns_conv* conv);
 int wd_modup(const wd_rns_conv* conv, const uint32_t* in, uint32_t* out, uint32_t batch,

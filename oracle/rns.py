@@ -147,3 +147,26 @@ def moddown(a: np.ndarray, qs, ps) -> np.ndarray:
         t = (a[:, i, :].astype(np.uint64) + q - corr[:, i, :].astype(np.uint64)) % q
         out[:, i, :] = (t * pow(P % q, -1, q) % q).astype(np.uint32)
     return out
+
+
+def bconv_partial(x: np.ndarray, local_src, all_src, dst) -> np.ndarray:
+    """One limb shard's share of BConv_{Q->P} (limb-sharded ModUp, SURVEY.md 8 rows e/f3):
+    the terms of ``bconv`` for the source limbs this shard holds, with Q the product of ALL
+    source primes; returns [B][len(dst)][N] residues mod p_j (uint64).  Summing the shards'
+    results mod p_j gives ``bconv(x_all, all_src, dst)``."""
+    x = np.ascontiguousarray(x, dtype=np.uint32)
+    B, a, N = x.shape
+    assert a == len(local_src)
+    Q = 1
+    for q in all_src:
+        Q *= int(q)
+    out = np.zeros((B, len(dst), N), dtype=np.uint64)
+    for j, p in enumerate(dst):
+        p = int(p)
+        acc = np.zeros((B, N), dtype=object)
+        for i, q in enumerate(local_src):
+            q = int(q)
+            y = (x[:, i, :].astype(object) * pow((Q // q) % q, -1, q)) % q
+            acc = acc + y * ((Q // q) % p)
+        out[:, j, :] = (acc % p).astype(np.uint64)
+    return out

@@ -58,39 +58,66 @@ __device__ __forceinline__ uint32_t reduce64(uint64_t v, uint32_t p, uint64_t mu
 }
 
 // x: [batch][x_ls][N] (source limbs start at row 0 of each polynomial's block);
-// y: [batch][y_ls][N], targets written at rows y_off .. y_off + D - 1 of each block
+// y: [batch][y_ls][N], targets written at rows y_off .. y_off + D - 1 of each block.
+// The tables live in shared memory; the source loads are issued 8 at a time and the target
+// loop is unrolled by 4 so each thread keeps several independent memory operations in flight.
+// y64 != nullptr (limb-sharded ModUp): the canonical residues go to y64 [batch][D][N] as 64-bit
+// words instead, so the shards' partial sums can be added by an integer all-reduce.
 __global__ void __launch_bounds__(BC_T) rns_bconv(const uint32_t* __restrict__ x, uint32_t x_ls,
                                                   uint32_t* __restrict__ y, uint32_t y_ls, uint32_t y_off,
-                                                  BconvTab tab, uint32_t N, uint32_t batch) {
-    extern __shared__ uint32_t bsm[];
-    uint32_t* ys = bsm;                                  // [S][BC_T]
-    uint2* ws = reinterpret_cast<uint2*>(bsm + tab.S * BC_T);   // [S][D]
+                                                  BconvTab tab, uint32_t N, uint32_t batch,
+                                                  unsigned long long* __restrict__ y64 = nullptr) {
+    extern __shared__ uint4 bsm4[];
+    uint4* src = bsm4;                                   // [S]
+    uint4* dst = bsm4 + tab.S;                           // [D]
+    uint2* ws = reinterpret_cast<uint2*>(bsm4 + tab.S + tab.D);              // [S][D]
+    uint32_t* ys = reinterpret_cast<uint32_t*>(ws + tab.S * tab.D);          // [S][BC_T]
+    for (uint32_t i = threadIdx.x; i < tab.S; i += BC_T) src[i] = tab.src[i];
+    for (uint32_t i = threadIdx.x; i < tab.D; i += BC_T) dst[i] = tab.dst[i];
     for (uint32_t i = threadIdx.x; i < tab.S * tab.D; i += BC_T) ws[i] = tab.w[i];
     const uint32_t per_poly = N / BC_T;
     __syncthreads();
     for (uint32_t blk = blockIdx.x; blk < batch * per_poly; blk += gridDim.x) {
         const uint32_t b = blk / per_poly, n = (blk % per_poly) * BC_T + threadIdx.x;
         const uint32_t* xb = x + (size_t)b * x_ls * N + n;
-        for (uint32_t i = 0; i < tab.S; ++i) {
-            const uint4 s = tab.src[i];
-            const uint32_t v = shoup_mul(__ldcs(xb + (size_t)i * N), s.y, s.z, s.x);
-            ys[i * BC_T + threadIdx.x] = canon2(v, s.x);
+        for (uint32_t i0 = 0; i0 < tab.S; i0 += 8) {
+            uint32_t v[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) v[u] = i0 + u < tab.S ? __ldcs(xb + (size_t)(i0 + u) * N) : 0u;
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+                if (i0 + u < tab.S) {
+                    const uint4 sc = src[i0 + u];
+                    ys[(i0 + u) * BC_T + threadIdx.x] = canon2(shoup_mul(v[u], sc.y, sc.z, sc.x), sc.x);
+                }
         }
         uint32_t* yb = y + ((size_t)b * y_ls + y_off) * N + n;
-        for (uint32_t j = 0; j < tab.D; ++j) {
-            const uint4 d = tab.dst[j];
-            const uint64_t mu = ((uint64_t)d.z << 32) | d.y;
-            uint32_t r;
-            if (tab.S <= 4) {                            // few terms: lazy Shoup products in [0, 2p)
-                const uint32_t p2 = 2 * d.x;
-                r = 0;
+        if (tab.S <= 4) {                                // few terms: lazy Shoup products in [0, 2p)
+            for (uint32_t j0 = 0; j0 < tab.D; j0 += 4) {
+                uint32_t r[4] = {0, 0, 0, 0};
                 for (uint32_t i = 0; i < tab.S; ++i) {
-                    const uint2 w = ws[i * tab.D + j];
-                    r += shoup_mul(ys[i * BC_T + threadIdx.x], w.x, w.y, d.x);
-                    r = umin32(r, r - p2);
+                    const uint32_t yi = ys[i * BC_T + threadIdx.x];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        if (j0 + u < tab.D) {
+                            const uint32_t p = dst[j0 + u].x;
+                            const uint2 w = ws[i * tab.D + j0 + u];
+                            r[u] += shoup_mul(yi, w.x, w.y, p);
+                            r[u] = umin32(r[u], r[u] - 2 * p);
+                        }
                 }
-                r = canon2(r, d.x);
-            } else {                                     // many terms: 64-bit MACs, Barrett every 15
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (j0 + u < tab.D) {
+                        const uint32_t res = canon2(r[u], dst[j0 + u].x);
+                        if (y64) y64[((size_t)b * tab.D + j0 + u) * N + n] = res;
+                        else __stcs(yb + (size_t)(j0 + u) * N, res);
+                    }
+            }
+        } else {                                         // many terms: 64-bit MACs, Barrett every 15
+            for (uint32_t j = 0; j < tab.D; ++j) {
+                const uint4 d = dst[j];
+                const uint64_t mu = ((uint64_t)d.z << 32) | d.y;
                 uint64_t acc = 0;
                 uint32_t i = 0;
                 while (i < tab.S) {
@@ -98,10 +125,20 @@ __global__ void __launch_bounds__(BC_T) rns_bconv(const uint32_t* __restrict__ x
                     for (; i < e; ++i) acc += (uint64_t)ys[i * BC_T + threadIdx.x] * ws[i * tab.D + j].x;
                     acc = reduce64(acc, d.x, mu);
                 }
-                r = (uint32_t)acc;
+                if (y64) y64[((size_t)b * tab.D + j) * N + n] = acc;
+                else __stcs(yb + (size_t)j * N, (uint32_t)acc);
             }
-            __stcs(yb + (size_t)j * N, r);
         }
+    }
+}
+
+// sum [rows][N] 64-bit (the all-reduced shard partials) -> canonical residue mod p_{row % D}
+__global__ void __launch_bounds__(256) rns_reduce64(const unsigned long long* __restrict__ sum, uint32_t* __restrict__ out,
+                                                    const uint4* __restrict__ dst, uint32_t D, uint32_t N, uint32_t rows) {
+    const size_t total = (size_t)rows * N;
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < total; i += (size_t)gridDim.x * blockDim.x) {
+        const uint4 d = dst[(i / N) % D];
+        out[i] = reduce64(sum[i], d.x, ((uint64_t)d.z << 32) | d.y);
     }
 }
 

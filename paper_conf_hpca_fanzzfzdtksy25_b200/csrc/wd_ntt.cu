@@ -545,6 +545,7 @@ struct wd_rns_conv {
     uint4* d_up_src = nullptr; uint2* d_up_w = nullptr; uint4* d_up_dst = nullptr;      // BConv Q -> P
     uint4* d_dn_src = nullptr; uint2* d_dn_w = nullptr; uint4* d_dn_dst = nullptr;      // BConv P -> Q
     uint4* d_pinv = nullptr;           // [a] {0, 0, P^-1 mod q_i, Shoup} (EPI = 2 store map)
+    bool sharded = false;              // Q-limb shard: Q -> P tables use the whole Q (wd_modup_partial)
 };
 
 namespace {
@@ -557,18 +558,21 @@ void free_conv(wd_rns_conv* c) {
 }
 
 // host tables of BConv src -> dst: {q_i, (Q/q_i)^-1, Shoup}, (Q/q_i) mod p_j, {p_j, mu}
+// Q = product of `all` (the whole source basis; `src` is the subset this table converts --
+// all of it, or one limb shard of it for the sharded ModUp)
 void bconv_tables(const std::vector<uint32_t>& src, const std::vector<uint32_t>& dst, std::vector<uint4>& hs,
-                  std::vector<uint2>& hw, std::vector<uint4>& hd) {
+                  std::vector<uint2>& hw, std::vector<uint4>& hd, const std::vector<uint32_t>* all_src = nullptr) {
+    const std::vector<uint32_t>& all = all_src ? *all_src : src;
     const size_t S = src.size(), D = dst.size();
     hs.resize(S); hw.resize(S * D); hd.resize(D);
     for (size_t i = 0; i < S; ++i) {
         uint32_t qh = 1;                                   // (Q/q_i) mod q_i
-        for (size_t k = 0; k < S; ++k) if (k != i) qh = pm_mul(qh, src[k] % src[i], src[i]);
+        for (uint32_t qk : all) if (qk != src[i]) qh = pm_mul(qh, qk % src[i], src[i]);
         const uint32_t inv = pm_pow(qh, src[i] - 2, src[i]);
         hs[i] = make_uint4(src[i], inv, pm_shoup(inv, src[i]), 0);
         for (size_t j = 0; j < D; ++j) {
             uint32_t v = 1;
-            for (size_t k = 0; k < S; ++k) if (k != i) v = pm_mul(v, src[k] % dst[j], dst[j]);
+            for (uint32_t qk : all) if (qk != src[i]) v = pm_mul(v, qk % dst[j], dst[j]);
             hw[i * D + j] = make_uint2(v, pm_shoup(v, dst[j]));
         }
     }
@@ -602,7 +606,7 @@ void launch_v8_rows(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t r
 
 int launch_bconv(const wd_ntt_plan* p, const uint32_t* x, uint32_t x_ls, uint32_t* y, uint32_t y_ls, uint32_t y_off,
                  const BconvTab& t, uint32_t batch, cudaStream_t s) {
-    const size_t smem = sizeof(uint32_t) * t.S * BC_T + sizeof(uint2) * t.S * t.D;
+    const size_t smem = sizeof(uint4) * (t.S + t.D) + sizeof(uint2) * t.S * t.D + sizeof(uint32_t) * t.S * BC_T;
     if (smem > 48 * 1024 && cudaFuncSetAttribute(rns_bconv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
         return WD_ECUDA;
     const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)batch * (p->N / BC_T), (uint64_t)p->sm_count * 8);
@@ -756,11 +760,28 @@ int wd_rescale(const wd_ntt_plan* p, const uint32_t* in, uint32_t* out, uint32_t
     return set_err(WD_OK);
 }
 
+wd_rns_conv* wd_rns_conv_create_shard(const wd_ntt_plan* pq, const wd_ntt_plan* pp, const uint32_t* q_all,
+                                      uint32_t a_all);
+
 wd_rns_conv* wd_rns_conv_create(const wd_ntt_plan* pq, const wd_ntt_plan* pp) {
+    if (!pq) { set_err(WD_EINVAL); return nullptr; }
+    return wd_rns_conv_create_shard(pq, pp, pq->primes.data(), pq->L);
+}
+
+wd_rns_conv* wd_rns_conv_create_shard(const wd_ntt_plan* pq, const wd_ntt_plan* pp, const uint32_t* q_all,
+                                      uint32_t a_all) {
     if (!pq || !pp) { set_err(WD_EINVAL); return nullptr; }
+    if (!q_all || a_all < pq->L || a_all > 4096) { set_err(WD_EINVAL); return nullptr; }
     if (pq->N != pp->N || pq->device != pp->device || pq->logN < 12 || pq->L > BC_MAX || pp->L > BC_MAX) {
         set_err(WD_EUNSUPPORTED); return nullptr;
     }
+    std::vector<uint32_t> all(q_all, q_all + a_all);
+    for (uint32_t a : pq->primes)                          // the local limbs must be part of Q
+        if (std::find(all.begin(), all.end(), a) == all.end()) { set_err(WD_EINVAL); return nullptr; }
+    for (size_t i = 0; i < all.size(); ++i)
+        for (size_t k = i + 1; k < all.size(); ++k) if (all[i] == all[k]) { set_err(WD_EINVAL); return nullptr; }
+    for (uint32_t a : all)
+        for (uint32_t b : pp->primes) if (a == b) { set_err(WD_EINVAL); return nullptr; }
     for (uint32_t a : pq->primes) {
         for (uint32_t b : pp->primes) if (a == b) { set_err(WD_EINVAL); return nullptr; }
     }
@@ -774,8 +795,9 @@ wd_rns_conv* wd_rns_conv_create(const wd_ntt_plan* pq, const wd_ntt_plan* pp) {
     std::vector<uint4> hs, hd, pinv(pq->L);
     std::vector<uint2> hw;
     bool ok = true;
-    bconv_tables(pq->primes, pp->primes, hs, hw, hd);
+    bconv_tables(pq->primes, pp->primes, hs, hw, hd, &all);
     ok = ok && upload(&c->d_up_src, hs) && upload(&c->d_up_w, hw) && upload(&c->d_up_dst, hd);
+    c->sharded = a_all != pq->L;
     bconv_tables(pp->primes, pq->primes, hs, hw, hd);
     ok = ok && upload(&c->d_dn_src, hs) && upload(&c->d_dn_w, hw) && upload(&c->d_dn_dst, hd);
     for (uint32_t i = 0; i < pq->L; ++i) {
@@ -799,6 +821,7 @@ int wd_modup(const wd_rns_conv* c, const uint32_t* in, uint32_t* out, uint32_t b
     if (((uintptr_t)in | (uintptr_t)out | (uintptr_t)work) & 15) return set_err(WD_EINVAL);
     if (batch == 0) return set_err(WD_OK);
     const wd_ntt_plan *pq = c->pq, *pp = c->pp;
+    if (c->sharded) return set_err(WD_EINVAL);             // a shard needs wd_modup_partial + all-reduce
     int dev = -1;
     if (cudaGetDevice(&dev) != cudaSuccess || dev != pq->device) return set_err(WD_EINVAL);
     if ((uint64_t)batch * (pq->L + pp->L) > 0x7fffffffull) return set_err(WD_EINVAL);
@@ -820,6 +843,55 @@ int wd_modup(const wd_rns_conv* c, const uint32_t* in, uint32_t* out, uint32_t b
     af.L = k; af.in_ls = a + k; af.out_ls = a + k;
     launch_v8_rows<0>(pp, true, af, batch * k, s);
     launches += 2;
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    g_last_launches = launches;
+    return set_err(WD_OK);
+}
+
+int wd_modup_partial(const wd_rns_conv* c, const uint32_t* in, uint64_t* partial, uint32_t batch,
+                     uint32_t* work, wd_stream_t st) {
+    g_last_launches = 0;
+    if (!c || !in || !partial || !work) return set_err(WD_EINVAL);
+    if (((uintptr_t)in | (uintptr_t)partial | (uintptr_t)work) & 15) return set_err(WD_EINVAL);
+    if (batch == 0) return set_err(WD_OK);
+    const wd_ntt_plan *pq = c->pq, *pp = c->pp;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != pq->device) return set_err(WD_EINVAL);
+    if ((uint64_t)batch * (pq->L + pp->L) > 0x7fffffffull) return set_err(WD_EINVAL);
+    cudaStream_t s = (cudaStream_t)st;
+    const uint32_t a = pq->L, k = pp->L;
+    NttArgs ai;
+    ai.in = in; ai.in2 = nullptr; ai.out = work; ai.tw = pq->d_inv; ai.lc = pq->d_lc; ai.L = a;
+    uint32_t launches = (uint32_t)launch_cuda_core(pq, false, ai, batch * a, s);
+    BconvTab t{c->d_up_src, c->d_up_w, c->d_up_dst, a, k};
+    const size_t smem = sizeof(uint4) * (t.S + t.D) + sizeof(uint2) * t.S * t.D + sizeof(uint32_t) * t.S * BC_T;
+    if (smem > 48 * 1024 && cudaFuncSetAttribute(rns_bconv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+        return set_err(WD_ECUDA);
+    const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)batch * (pq->N / BC_T), (uint64_t)pq->sm_count * 8);
+    rns_bconv<<<blocks, BC_T, smem, s>>>(work, a, nullptr, k, 0, t, pq->N, batch,
+                                         reinterpret_cast<unsigned long long*>(partial));
+    if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    g_last_launches = launches + 1;
+    return set_err(WD_OK);
+}
+
+int wd_modup_finish(const wd_rns_conv* c, const uint64_t* sum, uint32_t* out_p, uint32_t batch,
+                    wd_stream_t st) {
+    g_last_launches = 0;
+    if (!c || !sum || !out_p) return set_err(WD_EINVAL);
+    if (((uintptr_t)sum | (uintptr_t)out_p) & 15) return set_err(WD_EINVAL);
+    if (batch == 0) return set_err(WD_OK);
+    const wd_ntt_plan* pp = c->pp;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != pp->device) return set_err(WD_EINVAL);
+    cudaStream_t s = (cudaStream_t)st;
+    const uint32_t rows = batch * pp->L;
+    const uint32_t blocks = (uint32_t)std::min<uint64_t>(((uint64_t)rows * pp->N + 255) / 256, (uint64_t)pp->sm_count * 8);
+    rns_reduce64<<<blocks, 256, 0, s>>>(reinterpret_cast<const unsigned long long*>(sum), out_p, c->d_up_dst, pp->L,
+                                        pp->N, rows);
+    NttArgs af;
+    af.in = out_p; af.in2 = nullptr; af.out = out_p; af.tw = pp->d_fwd; af.lc = pp->d_lc; af.L = pp->L;
+    const uint32_t launches = 1 + (uint32_t)launch_cuda_core(pp, true, af, rows, s);
     if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
     g_last_launches = launches;
     return set_err(WD_OK);

@@ -85,3 +85,20 @@ def sharded_transform(x_full: torch.Tensor | None, primes: list[int], N: int, ba
 def _device():
     return torch.device("cuda", torch.cuda.current_device()) if torch.cuda.is_available() and \
         dist.get_backend() == "nccl" else torch.device("cpu")
+
+
+def sharded_modup(x_local: torch.Tensor, partial_fn: Callable[[torch.Tensor], torch.Tensor],
+                  finish_fn: Callable[[torch.Tensor], torch.Tensor]) -> torch.Tensor:
+    """Limb-sharded ModUp (SURVEY.md 8 rows e + f3): the one exchange step of the path.
+
+    Every rank holds its shard of the Q limbs ``x_local`` [B][a_g][N] (NTT domain).
+    ``partial_fn`` returns this shard's share of BConv_{Q->P} as int64 [B][k][N]
+    (on the GPU: ``RnsConv.modup_partial`` of a shard conversion object); the shares are
+    summed by ONE all-reduce, then ``finish_fn`` reduces mod p_j and NTTs
+    (``RnsConv.modup_finish``).  Returns the P limbs [B][k][N], identical on every rank.
+    The all-reduce moves B*k*N*8 bytes per rank: k = 1 special prime (Table III)
+    makes it 1/a of the input.
+    """
+    part = partial_fn(x_local)
+    dist.all_reduce(part, op=dist.ReduceOp.SUM)
+    return finish_fn(part)

@@ -49,6 +49,9 @@ _SIGS = {
     "wd_ntt_pointwise_inverse": (_i32, [_vp, _vp, _vp, _vp, _u32, _vp]),
     "wd_rescale": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_rns_conv_create": (_vp, [_vp, _vp]),
+    "wd_rns_conv_create_shard": (_vp, [_vp, _vp, _P32, _u32]),
+    "wd_modup_partial": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
+    "wd_modup_finish": (_i32, [_vp, _vp, _vp, _u32, _vp]),
     "wd_rns_conv_destroy": (None, [_vp]),
     "wd_modup": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
     "wd_moddown": (_i32, [_vp, _vp, _vp, _u32, _vp, _vp]),
@@ -138,6 +141,25 @@ def wd_rns_conv_create(plan_q: int, plan_p: int) -> int:
     if not h:
         raise WdNttError(_lib.wd_ntt_last_error(), "wd_rns_conv_create")
     return h
+
+
+def wd_rns_conv_create_shard(plan_q_local: int, plan_p: int, q_all) -> int:
+    q_all = [int(q) for q in q_all]
+    arr = (ctypes.c_uint32 * len(q_all))(*q_all)
+    h = _lib.wd_rns_conv_create_shard(plan_q_local, plan_p, arr, len(q_all))
+    if not h:
+        raise WdNttError(_lib.wd_ntt_last_error(), "wd_rns_conv_create_shard")
+    return h
+
+
+def wd_modup_partial(conv: int, inp, partial, batch: int, work, stream=None) -> int:
+    return _check(_lib.wd_modup_partial(conv, _ptr(inp), _ptr(partial), batch, _ptr(work), _stream(stream, inp)),
+                  "wd_modup_partial")
+
+
+def wd_modup_finish(conv: int, total, out_p, batch: int, stream=None) -> int:
+    return _check(_lib.wd_modup_finish(conv, _ptr(total), _ptr(out_p), batch, _stream(stream, total)),
+                  "wd_modup_finish")
 
 
 def wd_rns_conv_destroy(conv: int) -> None:
@@ -274,9 +296,31 @@ class Plan:
 class RnsConv:
     """RAII wrapper of wd_rns_conv: ModUp / ModDown between ``plan_q`` (a limbs) and ``plan_p`` (k limbs)."""
 
-    def __init__(self, plan_q: "Plan", plan_p: "Plan"):
+    def __init__(self, plan_q: "Plan", plan_p: "Plan", q_all=None):
         self.pq, self.pp = plan_q, plan_p              # keep the plans alive
-        self.handle = wd_rns_conv_create(plan_q.handle, plan_p.handle)
+        if q_all is None:
+            self.handle = wd_rns_conv_create(plan_q.handle, plan_p.handle)
+        else:                                          # plan_q is one limb shard of q_all
+            self.handle = wd_rns_conv_create_shard(plan_q.handle, plan_p.handle, q_all)
+
+    def modup_partial(self, x, partial=None, work=None, stream=None):
+        """This shard's 64-bit share of BConv_{Q->P}: [B][k][N] int64 (sum over shards, then finish)."""
+        import torch
+        a, k, n = self.pq.L, self.pp.L, self.pq.N
+        b = x.numel() // (a * n)
+        partial = torch.empty((b, k, n), dtype=torch.int64, device=x.device) if partial is None else partial
+        work = torch.empty((b, a, n), dtype=x.dtype, device=x.device) if work is None else work
+        wd_modup_partial(self.handle, x, partial, b, work, stream)
+        return partial
+
+    def modup_finish(self, total, out=None, stream=None):
+        """Summed partials -> the P limbs of ModUp, NTT domain [B][k][N]."""
+        import torch
+        k, n = self.pp.L, self.pp.N
+        b = total.numel() // (k * n)
+        out = torch.empty((b, k, n), dtype=torch.int32, device=total.device) if out is None else out
+        wd_modup_finish(self.handle, total, out, b, stream)
+        return out
 
     def modup(self, x, out=None, work=None, stream=None):
         import torch

@@ -67,3 +67,47 @@ def test_sharded_equals_unsharded_gloo(L):
         p.join(120)
         assert p.exitcode == 0
     assert q.get(timeout=5) is True
+
+
+# -------------------------------------------------- limb-sharded ModUp: the all-reduce exchange
+def _modup_worker(rank, world, port, n, out_q):
+    import oracle
+    from oracle import rns
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    qs = inputs.bench_primes(5)
+    ps = [786433, 805961729]
+    x = inputs.uniform_residues(qs, n, 2, 123)                  # every rank can build the same input
+    l0, l1 = wdist.limb_range(len(qs), world, rank)
+    x_local = torch.from_numpy(np.ascontiguousarray(x[:, l0:l1]).view(np.int32))
+
+    def partial_fn(xl):
+        coeff = oracle.ntt_inverse(xl.numpy().view(np.uint32), qs[l0:l1], threads=1)
+        return torch.from_numpy(rns.bconv_partial(coeff, qs[l0:l1], qs, ps).astype(np.int64))
+
+    def finish_fn(total):
+        t = total.numpy().astype(np.uint64)
+        for j, p in enumerate(ps):
+            t[:, j] %= p
+        return torch.from_numpy(oracle.ntt_forward(t.astype(np.uint32), ps, threads=1).view(np.int32))
+
+    up_p = wdist.sharded_modup(x_local, partial_fn, finish_fn)
+    ref = rns.modup(x, qs, ps)[:, len(qs):]
+    out_q.put((rank, bool(np.array_equal(up_p.numpy().view(np.uint32), ref))))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_sharded_modup_allreduce_gloo():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_modup_worker, args=(r, 2, port, 128, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(120)
+        assert p.exitcode == 0
+    res = sorted(q.get(timeout=5) for _ in range(2))
+    assert res == [(0, True), (1, True)]

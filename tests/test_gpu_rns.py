@@ -165,3 +165,30 @@ def test_rns_conv_errors(wd):
         wd.RnsConv(pq, wd.Plan(n, [P[2], P[9]]))            # a prime in both bases
     with pytest.raises(wd.WdNttError):
         wd.RnsConv(pq, wd.Plan(1 << 13, P[10:12]))          # N mismatch
+
+
+def test_sharded_modup_partials(wd):
+    # two Q-limb shards on one GPU: partial shares summed (the all-reduce's job) and finished
+    # equal the unsharded ModUp's P limbs; ModDown on a shard gives that shard's Q limbs
+    n, qs, ps = 1 << 16, P[:6], P[40:42]
+    x = inputs.uniform_residues(qs, n, 3, 8800)
+    pp = wd.Plan(n, ps)
+    total, convs = None, []
+    for a0, a1 in [(0, 4), (4, 6)]:
+        pq = wd.Plan(n, qs[a0:a1])
+        conv = wd.RnsConv(pq, pp, q_all=qs)
+        convs.append((a0, a1, conv, pq))
+        part = conv.modup_partial(to_dev(np.ascontiguousarray(x[:, a0:a1])))
+        total = part if total is None else total + part
+    up_p = convs[0][2].modup_finish(total)
+    torch.cuda.synchronize()
+    full = rns.modup(x, qs, ps)
+    assert np.array_equal(to_host(up_p), full[:, len(qs):])
+    with pytest.raises(wd.WdNttError):
+        convs[0][2].modup(to_dev(np.ascontiguousarray(x[:, 0:4])))   # a shard cannot run the whole ModUp
+    ext = inputs.uniform_residues(qs + ps, n, 2, 8900)
+    down = rns.moddown(ext, qs, ps)
+    for a0, a1, conv, pq in convs:
+        loc = np.ascontiguousarray(np.concatenate([ext[:, a0:a1], ext[:, len(qs):]], axis=1))
+        got = to_host(conv.moddown(to_dev(loc)))
+        assert np.array_equal(got, down[:, a0:a1]), (a0, a1)

@@ -160,3 +160,17 @@ def test_moddown_exact_multiple_of_p():
     a = oracle.ntt_forward(coeff[None], allp)
     down = oracle.ntt_inverse(rns.moddown(a, QS, PS), QS)[0]
     assert np.array_equal(down, np.array([[x % int(q) for x in X] for q in QS], dtype=np.uint32))
+
+
+@pytest.mark.parametrize("split", [1, 2, 3])
+def test_bconv_partial_shards_sum_to_full(split):
+    # limb-sharded ModUp: the shards' partial BConv sums add up (mod p_j) to the full BConv
+    n = 32
+    x = inputs.uniform_residues(QS, n, 2, 7900 + split)
+    full = rns.bconv(x, QS, PS).astype(np.uint64)
+    acc = np.zeros_like(full)
+    for a0, a1 in [(0, split), (split, len(QS))]:
+        acc += rns.bconv_partial(np.ascontiguousarray(x[:, a0:a1]), QS[a0:a1], QS, PS)
+    for j, p in enumerate(PS):
+        acc[:, j] %= int(p)
+    assert np.array_equal(acc, full)
