@@ -42,6 +42,7 @@ struct NttArgs {
     // v8 only: rows between consecutive polynomials in `in` / `out` (0 = L, contiguous); lets a
     // launch cover a limb SECTION of a wider [batch][Lfull][N] tensor (ModUp / ModDown, ntt_rns.cuh)
     uint32_t in_ls = 0, out_ls = 0;
+    uint32_t stagger_ns = 0;         // v8 experiment knob (WD_NTT_STAGGER): grid quarters start k * this apart
 };
 
 __device__ __forceinline__ uint32_t row_map(uint32_t row, uint32_t L, uint32_t ls) {

@@ -107,6 +107,10 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
     extern __shared__ __align__(16) uint32_t smem[];
     const int t = threadIdx.x;
     const int hi4 = t >> 4, lo4 = t & 15;
+    if (a.stagger_ns) {                          // experiment: start the grid's quarters staggered
+        const uint32_t k = blockIdx.x * 4 / gridDim.x;
+        for (uint32_t i = 0; i < k * a.stagger_ns / 1000; ++i) __nanosleep(1000);
+    }
 
 #pragma unroll 1
     for (uint32_t row = blockIdx.x / CL; row < rows; row += gridDim.x / CL) {
@@ -125,7 +129,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
 
         if constexpr (FWD) {
             // ---- phase 1: layers 0..A-1 on columns c (elements c + 4096 k) ----
-            if constexpr (A > 0 && ONLY != 2) {
+            if constexpr (A > 0 && ONLY != 2 && (ONLY < 3 || ONLY == 7)) {
 #pragma unroll 1
                 for (int pass = p0; pass < p0 + NP; ++pass) {
                     const int c = pass * V8_T + t;
@@ -145,12 +149,15 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
             // ---- phase 2: layers A..A+11 on sub-rows s ----
             if constexpr (ONLY != 1) {
             const uint32_t* src = A > 0 ? out : in;
-            v8_load_fwd_slice(smem, src + s0 * V8_SUBW);
+            if constexpr (ONLY < 3 || ONLY == 7) v8_load_fwd_slice(smem, src + s0 * V8_SUBW);
 #pragma unroll 1
             for (int s = s0; s < s1; ++s) {
                 uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
-                cp_async_wait<0>();
+                if constexpr (ONLY < 3 || ONLY == 7) cp_async_wait<0>();
                 __syncwarp();                            // this warp's stage-1 slice of sub-row s landed
+                // ONLY 3..5 (timing experiments): 3 = no sub-row loads, 4 = no loads and no stores,
+                // 5 = as 4 with every sub-row's twiddles taken from sub-row 0 (L1-resident)
+                const uint32_t st = ONLY == 5 ? 0u : (uint32_t)s;
                 uint32_t x[16];
                 {   // stage 1: layers A..A+3, thread (b, c), elements a (stride 256)
                     const int b = hi4, c = lo4;
@@ -159,19 +166,19 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                         x[i] = S[v8_phys(i, b, c)];
                         if constexpr (EPI == 1 && A == 0) x[i] = rs_in(x[i], a.rs_thr, rsc, q);
                     }
-                    fwd_radix<4>(x, tw, A, (uint32_t)s, q, q2);
+                    fwd_radix<4>(x, tw, A, st, q, q2);
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
                 }
                 __syncthreads();                         // stage 1 done everywhere; sub-row s-1 fully consumed
-                if (s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
+                if ((ONLY < 3 || ONLY == 7) && s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
                 uint2 w3[JIT3 ? 1 : 15];
-                if constexpr (!JIT3) load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);   // stage-3 twiddles, in flight
+                if constexpr (!JIT3) load_tw16(w3, tw, A + 8, st * 256 + t);   // stage-3 twiddles, in flight
                 {   // stage 2: layers A+4..A+7, thread (a, c), elements b (stride 16)
                     const int aa = hi4, c = lo4;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
-                    fwd_radix<4>(x, tw, A + 4, (uint32_t)s * 16 + aa, q, q2);
+                    fwd_radix<4>(x, tw, A + 4, st * 16 + aa, q, q2);
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
                 }
@@ -185,10 +192,50 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                         const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
                         x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
                     }
-                    if constexpr (JIT3) fwd_radix<4>(x, tw, A + 8, (uint32_t)s * 256 + t, q, q2);
+                    if constexpr (JIT3) fwd_radix<4>(x, tw, A + 8, st * 256 + t, q, q2);
                     else fwd16_tw(x, w3, q, q2);
                     uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
-                    if constexpr (EPI) {
+                    if constexpr (ONLY == 6 || ONLY == 7) {   // coalesced stores in the wrong order (timing only)
+                        uint4* o2 = reinterpret_cast<uint4*>(out + s * V8_SUBW);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v)
+                            __stcs(o2 + v * V8_T + t, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
+                                                     canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                    } else if constexpr (ONLY >= 4) {
+                        uint32_t z = 0;
+#pragma unroll
+                        for (int i = 0; i < 16; ++i) z ^= x[i];
+                        if (z == 0xFFFFFFFFu && x[0] == 0xFFFFFFFFu) o[0] = make_uint4(z, z, z, z);
+                    } else if constexpr (ONLY != 8) {
+                        // Coalesced store through the warp's own 2 KB of S: stage 3 of warp w covers
+                        // words 512w .. 512w+511 of the sub-row, so after writing them back (the same
+                        // conflict-free 16-byte slots it read) each lane re-reads granules 128v + 4*lane
+                        // and every STG.128 of the warp writes 512 contiguous bytes (the direct
+                        // per-thread 64-byte stores cost 4x the L1 wavefronts: v86 vs v83, DESIGN 5.1).
+                        uint32_t* wb = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v)
+                            *reinterpret_cast<uint4*>(wb + ((v ^ sw) << 2)) =
+                                make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                        __syncwarp();
+                        const int wbase = (t >> 5) * 512 + 4 * (t & 31);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            const int e = wbase + 128 * v;
+                            const uint4 u = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
+                            uint4* og = reinterpret_cast<uint4*>(out + s * V8_SUBW + e);
+                            if constexpr (EPI) {
+                                const uint4 av = __ldcs(reinterpret_cast<const uint4*>(ain + s * V8_SUBW + e));
+                                __stcs(og, make_uint4(rs_out(av.x, umin32(u.x, u.x - q2), rsc, q),
+                                                      rs_out(av.y, umin32(u.y, u.y - q2), rsc, q),
+                                                      rs_out(av.z, umin32(u.z, u.z - q2), rsc, q),
+                                                      rs_out(av.w, umin32(u.w, u.w - q2), rsc, q)));
+                            } else {
+                                __stcs(og, make_uint4(canon4(u.x, q, q2), canon4(u.y, q, q2),
+                                                      canon4(u.z, q, q2), canon4(u.w, q, q2)));
+                            }
+                        }
+                    } else if constexpr (EPI) {
                         const uint4* ai = reinterpret_cast<const uint4*>(ain + s * V8_SUBW + t * 16);
 #pragma unroll
                         for (int v = 0; v < 4; ++v) {

@@ -41,6 +41,7 @@ struct wd_ntt_plan {
     int v6_ctas = 4;               // resident 256-thread CTAs per SM for v6 (WD_NTT_CTAS: 2..4, A/B runs)
     int v8_minb = 0;               // v8 CTAs per SM (WD_NTT_MINB: 4..6; 0 = measured default)
     int v8_cl = 0;                 // v8 CTAs per row cluster (WD_NTT_CL: 1, 2, 4; 0 = measured default)
+    uint32_t stagger_ns = 0;       // WD_NTT_STAGGER (v8 experiment)
     int kernel_ver = 0;            // 0 = AUTO, the measured default per N and row count (launch_cc);
                                    // WD_NTT_KERNEL=v1|v2|v3|v5|v6 forces a generation (A/B runs)
     std::vector<uint32_t> primes, psi;
@@ -270,6 +271,24 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         }
     }
     if constexpr (LOGN >= 12) {
+        if (fwd && p->kernel_ver == 86) { ntt_v8<LOGN, true, false, 6><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows); return; }
+        if (fwd && p->kernel_ver == 88) {   // v8 (2-CTA cluster) with the old per-thread 64-byte stores
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(p->sm_count * 4); cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM; cfg.stream = s;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+            cfg.attrs = at; cfg.numAttrs = 1;
+            if constexpr (LOGN >= 13) cudaLaunchKernelEx(&cfg, ntt_v8<LOGN, true, false, 8, 4, 2>, a, rows);
+            return;
+        }
+        if (fwd && p->kernel_ver == 87) { ntt_v8<LOGN, true, false, 7><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows); return; }
+        if (fwd && p->kernel_ver >= 83 && p->kernel_ver <= 85) {   // timing experiments (ntt_v8 ONLY 3..5)
+            if (p->kernel_ver == 83) ntt_v8<LOGN, true, false, 3><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            else if (p->kernel_ver == 84) ntt_v8<LOGN, true, false, 4><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            else ntt_v8<LOGN, true, false, 5><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
+            return;
+        }
         if (p->kernel_ver == 81 || p->kernel_ver == 82) {   // timing experiment: one phase of v8 only
             if (fwd && p->kernel_ver == 81) ntt_v8<LOGN, true, false, 1><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
             else if (fwd) ntt_v8<LOGN, true, false, 2><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
@@ -456,6 +475,7 @@ int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2,
     const uint32_t rows = (uint32_t)rows64;
     NttArgs a;
     a.in = in; a.in2 = in2; a.out = out; a.tw = fwd ? p->d_fwd : p->d_inv; a.lc = p->d_lc; a.L = p->L;
+    a.stagger_ns = p->stagger_ns;
     const int mode = effective_mode(p);
     int launches = 0;
     if (mode == WD_MODE_CUDA_GEMM && in2 == nullptr && p->logN == 16 && p->tc.ok) {
@@ -661,6 +681,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (const char* ev = getenv("WD_NTT_CTAS")) p->v6_ctas = std::max(1, std::min(4, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_MINB")) p->v8_minb = std::max(4, std::min(6, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
+    if (const char* ev = getenv("WD_NTT_STAGGER")) p->stagger_ns = (uint32_t)atoi(ev);
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
