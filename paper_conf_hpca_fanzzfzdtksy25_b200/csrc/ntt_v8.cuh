@@ -74,7 +74,8 @@ __device__ __forceinline__ void v8_load_sub(uint32_t* S, const uint32_t* src) {
 
 // MINB: resident CTAs per SM the register budget is cut for (4 -> 64 registers; 5, 6 -> 48, 40
 // with per-layer just-in-time stage-3 twiddles instead of 15 preloaded pairs).
-// ONLY: 1 = phase 1 only, 2 = phase 2 only (timing experiments; results are wrong).
+// ONLY: 1 = phase 1 only, 2 = phase 2 only, 3..8 other timing experiments (results are wrong); 9 = v8
+// without the column-pass prefetch (correct; A/B runs).
 // CL > 1: a cluster of CL CTAs shares each row -- CTA rank r takes column passes and sub-rows
 // [r, r+1) * (16|R)/CL, with ONE cluster barrier (release/acquire) between the phases.  Rows
 // in flight, hence the L2 footprint of the intermediate, shrink by CL.
@@ -102,6 +103,9 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
     static_assert(R % CL == 0 && (V8_SUBW / V8_T) % CL == 0, "cluster splits passes and sub-rows evenly");
     constexpr int NP = V8_SUBW / V8_T / CL;  // phase-1 column passes per CTA
     constexpr int NS = R / CL;               // phase-2 sub-rows per CTA
+    // PF: column passes pipelined two deep (needs 2 x 2^A data registers: A <= 4; ONLY = 9 turns
+    // it off for A/B runs)
+    constexpr bool PF = R <= 16 && NP % 2 == 0 && NP >= 2 && ONLY != 9;
     const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
     const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
     extern __shared__ __align__(16) uint32_t smem[];
@@ -129,7 +133,37 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
 
         if constexpr (FWD) {
             // ---- phase 1: layers 0..A-1 on columns c (elements c + 4096 k) ----
-            if constexpr (A > 0 && ONLY != 2 && (ONLY < 3 || ONLY == 7)) {
+            if constexpr (A > 0 && ONLY != 2 && (ONLY < 3 || ONLY >= 7) && PF) {
+                // column passes software-pipelined by two register sets: pass p+1's 2^A loads are
+                // in flight while pass p computes (ncu: the first use of the column loads was the
+                // top stall site, long scoreboard, with one pass in flight per thread)
+                uint32_t xa[R], xb[R];
+                auto ldp = [&](uint32_t (&v)[R], int pass) {
+                    const int c = pass * V8_T + t;
+#pragma unroll
+                    for (int k = 0; k < R; ++k) v[k] = EPI == 1 ? __ldg(in + k * V8_SUBW + c) : __ldcs(in + k * V8_SUBW + c);
+                };
+                auto cmp = [&](uint32_t (&v)[R], int pass) {
+                    const int c = pass * V8_T + t;
+                    if constexpr (EPI == 1) {
+#pragma unroll
+                        for (int k = 0; k < R; ++k) v[k] = rs_in(v[k], a.rs_thr, rsc, q);
+                    }
+                    fwd_radix<A>(v, tw, 0, 0, q, q2);
+#pragma unroll
+                    for (int k = 0; k < R; ++k) out[k * V8_SUBW + c] = v[k];
+                };
+                ldp(xa, p0);
+#pragma unroll 1
+                for (int pass = p0; pass < p0 + NP; pass += 2) {
+                    ldp(xb, pass + 1);
+                    cmp(xa, pass);
+                    if (pass + 2 < p0 + NP) ldp(xa, pass + 2);
+                    cmp(xb, pass + 1);
+                }
+                if constexpr (CL > 1) cluster_sync();    // the whole intermediate is written
+                else __syncthreads();
+            } else if constexpr (A > 0 && ONLY != 2 && (ONLY < 3 || ONLY >= 7)) {
 #pragma unroll 1
                 for (int pass = p0; pass < p0 + NP; ++pass) {
                     const int c = pass * V8_T + t;
@@ -149,11 +183,11 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
             // ---- phase 2: layers A..A+11 on sub-rows s ----
             if constexpr (ONLY != 1) {
             const uint32_t* src = A > 0 ? out : in;
-            if constexpr (ONLY < 3 || ONLY == 7) v8_load_fwd_slice(smem, src + s0 * V8_SUBW);
+            if constexpr (ONLY < 3 || ONLY >= 7) v8_load_fwd_slice(smem, src + s0 * V8_SUBW);
 #pragma unroll 1
             for (int s = s0; s < s1; ++s) {
                 uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
-                if constexpr (ONLY < 3 || ONLY == 7) cp_async_wait<0>();
+                if constexpr (ONLY < 3 || ONLY >= 7) cp_async_wait<0>();
                 __syncwarp();                            // this warp's stage-1 slice of sub-row s landed
                 // ONLY 3..5 (timing experiments): 3 = no sub-row loads, 4 = no loads and no stores,
                 // 5 = as 4 with every sub-row's twiddles taken from sub-row 0 (L1-resident)
@@ -171,7 +205,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
                 }
                 __syncthreads();                         // stage 1 done everywhere; sub-row s-1 fully consumed
-                if ((ONLY < 3 || ONLY == 7) && s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
+                if ((ONLY < 3 || ONLY >= 7) && s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
                 uint2 w3[JIT3 ? 1 : 15];
                 if constexpr (!JIT3) load_tw16(w3, tw, A + 8, st * 256 + t);   // stage-3 twiddles, in flight
                 {   // stage 2: layers A+4..A+7, thread (a, c), elements b (stride 16)
@@ -201,7 +235,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                         for (int v = 0; v < 4; ++v)
                             __stcs(o2 + v * V8_T + t, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
                                                      canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
-                    } else if constexpr (ONLY >= 4) {
+                    } else if constexpr (ONLY == 4 || ONLY == 5) {
                         uint32_t z = 0;
 #pragma unroll
                         for (int i = 0; i < 16; ++i) z ^= x[i];
@@ -321,6 +355,28 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
             if constexpr (A > 0 && ONLY != 2) {
                 if constexpr (CL > 1) cluster_sync();    // the whole intermediate is written
                 else __syncthreads();
+                if constexpr (PF) {                       // two register sets, as in phase 1
+                    uint32_t xa[R], xb[R];
+                    auto ldp = [&](uint32_t (&v)[R], int pass) {
+                        const int c = pass * V8_T + t;
+#pragma unroll
+                        for (int k = 0; k < R; ++k) v[k] = out[k * V8_SUBW + c];
+                    };
+                    auto cmp = [&](uint32_t (&v)[R], int pass) {
+                        const int c = pass * V8_T + t;
+                        inv_radix<A, true>(v, tw, 0, 0, lc);
+#pragma unroll
+                        for (int k = 0; k < R; ++k) __stcs(out + k * V8_SUBW + c, canon2(v[k], q));
+                    };
+                    ldp(xa, p0);
+#pragma unroll 1
+                    for (int pass = p0; pass < p0 + NP; pass += 2) {
+                        ldp(xb, pass + 1);
+                        cmp(xa, pass);
+                        if (pass + 2 < p0 + NP) ldp(xa, pass + 2);
+                        cmp(xb, pass + 1);
+                    }
+                } else
 #pragma unroll 1
                 for (int pass = p0; pass < p0 + NP; ++pass) {
                     const int c = pass * V8_T + t;

@@ -282,6 +282,16 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             if constexpr (LOGN >= 13) cudaLaunchKernelEx(&cfg, ntt_v8<LOGN, true, false, 8, 4, 2>, a, rows);
             return;
         }
+        if (p->kernel_ver == 89) {   // v8 (2-CTA cluster) without the column-pass prefetch
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(p->sm_count * 4); cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM; cfg.stream = s;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+            cfg.attrs = at; cfg.numAttrs = 1;
+            if constexpr (LOGN >= 13) cudaLaunchKernelEx(&cfg, fwd ? ntt_v8<LOGN, true, false, 9, 4, 2> : ntt_v8<LOGN, false, false, 9, 4, 2>, a, rows);
+            return;
+        }
         if (fwd && p->kernel_ver == 87) { ntt_v8<LOGN, true, false, 7><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows); return; }
         if (fwd && p->kernel_ver >= 83 && p->kernel_ver <= 85) {   // timing experiments (ntt_v8 ONLY 3..5)
             if (p->kernel_ver == 83) ntt_v8<LOGN, true, false, 3><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows);
