@@ -37,6 +37,21 @@ __device__ __forceinline__ int v8_phys(int a, int b, int c) {
     return a * 256 + ((b ^ (a & 1)) << 4) + (c ^ (((b >> 1) & 3) << 2));
 }
 
+// Sub-row loads read data for the LAST time (the input, or the L2-resident intermediate); an L2
+// evict-first hint would keep them from pushing other rows' intermediates out of L2 (see below).
+__device__ __forceinline__ uint64_t l2_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ void cp_async16_ef(void* smem_dst, const void* gsrc, uint64_t pol) {
+    // NOTE: the .L2::cache_hint form of cp.async (createpolicy evict_first) faulted with an
+    // illegal instruction on B200 (ptxas packs the policy into the odd UR of the memory
+    // descriptor), so the hint is dropped here; pol is unused.
+    (void)pol;
+    cp_async16(smem_dst, gsrc);
+}
+
 // Per-warp slices: in phase 2 each warp cp.asyncs exactly the words its own FIRST stage reads,
 // so the first stage needs only the warp's own wait + __syncwarp, and the stage pair that stays
 // inside a half-warp (forward 2->3, inverse 3'->2') needs only __syncwarp: one CTA barrier per
@@ -44,30 +59,33 @@ __device__ __forceinline__ int v8_phys(int a, int b, int c) {
 // forward (stage 1, thread (b,c) loops a): warp w reads words a*256 + 32w .. +31, a = 0..15
 __device__ __forceinline__ void v8_load_fwd_slice(uint32_t* S, const uint32_t* src) {
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    const uint64_t pol = l2_evict_first();
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
         const int a = 4 * k + (l >> 3), g = l & 7;           // 128-byte segment a, granule g
-        cp_async16(S + v8_phys(a, 2 * w + (g >> 2), (g & 3) << 2), src + a * 256 + 32 * w + 4 * g);
+        cp_async16_ef(S + v8_phys(a, 2 * w + (g >> 2), (g & 3) << 2), src + a * 256 + 32 * w + 4 * g, pol);
     }
     cp_async_commit();
 }
 // inverse (stage 3', thread (a,b) reads 16 contiguous c): warp w reads words 512w .. 512w + 511
 __device__ __forceinline__ void v8_load_inv_slice(uint32_t* S, const uint32_t* src) {
     const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+    const uint64_t pol = l2_evict_first();
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
         const int e = 512 * w + 4 * (32 * k + l);
-        cp_async16(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15), src + e);
+        cp_async16_ef(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15), src + e, pol);
     }
     cp_async_commit();
 }
 
 // cp.async one 4096-word sub-row (contiguous in global) into the swizzled layout
 __device__ __forceinline__ void v8_load_sub(uint32_t* S, const uint32_t* src) {
+    const uint64_t pol = l2_evict_first();
 #pragma unroll
     for (int k = 0; k < V8_SUBW / 4 / V8_T; ++k) {
         const int G = threadIdx.x + k * V8_T;               // 16-byte granule: words 4G..4G+3
-        cp_async16(S + v8_phys(G >> 6, (G >> 2) & 15, (G & 3) << 2), src + 4 * G);
+        cp_async16_ef(S + v8_phys(G >> 6, (G >> 2) & 15, (G & 3) << 2), src + 4 * G, pol);
     }
     cp_async_commit();
 }
@@ -360,7 +378,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     auto ldp = [&](uint32_t (&v)[R], int pass) {
                         const int c = pass * V8_T + t;
 #pragma unroll
-                        for (int k = 0; k < R; ++k) v[k] = out[k * V8_SUBW + c];
+                        for (int k = 0; k < R; ++k) v[k] = __ldcs(out + k * V8_SUBW + c);   // last use
                     };
                     auto cmp = [&](uint32_t (&v)[R], int pass) {
                         const int c = pass * V8_T + t;
@@ -382,7 +400,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     const int c = pass * V8_T + t;
                     uint32_t x[R];
 #pragma unroll
-                    for (int k = 0; k < R; ++k) x[k] = out[k * V8_SUBW + c];
+                    for (int k = 0; k < R; ++k) x[k] = __ldcs(out + k * V8_SUBW + c);
                     inv_radix<A, true>(x, tw, 0, 0, lc);
 #pragma unroll
                     for (int k = 0; k < R; ++k) __stcs(out + k * V8_SUBW + c, canon2(x[k], q));
