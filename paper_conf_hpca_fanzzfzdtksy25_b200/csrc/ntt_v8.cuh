@@ -90,6 +90,28 @@ __device__ __forceinline__ void v8_load_sub(uint32_t* S, const uint32_t* src) {
     cp_async_commit();
 }
 
+// Coalesced forward store of a sub-row's stage-3 results (v8 and the kernels sharing its layout):
+// stage 3 of warp w holds words 512w .. 512w+511 (thread (aa, b): 16 contiguous words), the same
+// words its stages 2 and 3 read, so the warp writes them back to its own slots of S, syncs, and
+// each lane re-reads granules 128v + 4*lane: every STG.128 writes 512 contiguous bytes instead of
+// 32 scattered 16-byte pieces (4x fewer L1 wavefronts).
+template <typename F>
+__device__ __forceinline__ void v8_store_sub(uint32_t* S, int aa, int b, const uint32_t* x, uint32_t* osub, F fin) {
+    uint32_t* wb = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+    const int sw = (b >> 1) & 3;
+#pragma unroll
+    for (int v = 0; v < 4; ++v)
+        *reinterpret_cast<uint4*>(wb + ((v ^ sw) << 2)) = make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+    __syncwarp();
+    const int wbase = (threadIdx.x >> 5) * 512 + 4 * (threadIdx.x & 31);
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+        const int e = wbase + 128 * v;
+        const uint4 u = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
+        __stcs(reinterpret_cast<uint4*>(osub + e), make_uint4(fin(u.x), fin(u.y), fin(u.z), fin(u.w)));
+    }
+}
+
 // MINB: resident CTAs per SM the register budget is cut for (4 -> 64 registers; 5, 6 -> 48, 40
 // with per-layer just-in-time stage-3 twiddles instead of 15 preloaded pairs).
 // ONLY: 1 = phase 1 only, 2 = phase 2 only, 3..8 other timing experiments (results are wrong); 9 = v8
@@ -533,11 +555,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v9(NttArgs a, uint32_t rows) {
                         x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
                     }
                     fwd16_tw(x, w3, q, q2);
-                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
-                                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                    v8_store_sub(S, aa, b, x, out + s * V8_SUBW, [&](uint32_t y) { return canon4(y, q, q2); });
                 }
             }
         } else {
@@ -798,11 +816,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v10(NttArgs a, const uint8_t* G, 
                         x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
                     }
                     fwd16_tw(x, w3, q, q2);
-                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
-                                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                    v8_store_sub(S, aa, b, x, out + s * V8_SUBW, [&](uint32_t y) { return canon4(y, q, q2); });
                 }
             }
         } else {
@@ -1007,11 +1021,7 @@ __global__ void __launch_bounds__(V8_T, 3) ntt_wdcuda16(WdcArgs wa, uint32_t row
                     }
                     wdc_twist(x, T3 + ((size_t)s * 256 + t) * 16, q);
                     wdc_gemm16(x, Mst + 256, lc);
-                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        __stcs(o + v, make_uint4(wdc_canon(x[4 * v], q, q2), wdc_canon(x[4 * v + 1], q, q2),
-                                                 wdc_canon(x[4 * v + 2], q, q2), wdc_canon(x[4 * v + 3], q, q2)));
+                    v8_store_sub(S, aa, b, x, out + s * V8_SUBW, [&](uint32_t y) { return wdc_canon(y, q, q2); });
                 }
             }
         } else {
@@ -1307,11 +1317,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v11(V11Args va, uint32_t rows) {
                         x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
                     }
                     fwd16_tw(x, w3, q, q2);
-                    uint4* o = reinterpret_cast<uint4*>(out + s * V8_SUBW + t * 16);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        __stcs(o + v, make_uint4(canon4(x[4 * v], q, q2), canon4(x[4 * v + 1], q, q2),
-                                                 canon4(x[4 * v + 2], q, q2), canon4(x[4 * v + 3], q, q2)));
+                    v8_store_sub(S, aa, b, x, out + s * V8_SUBW, [&](uint32_t y) { return canon4(y, q, q2); });
                 }
             }
         } else {
