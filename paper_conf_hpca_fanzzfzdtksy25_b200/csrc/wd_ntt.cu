@@ -331,12 +331,17 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             int minb = p->v8_minb ? p->v8_minb : V8_DEFAULT_MINB;
             int cl = p->v8_cl ? p->v8_cl : V8_DEFAULT_CL;
             if (LOGN == 17 && fwd && !p->v8_minb) minb = 4;     // radix-32 column phase spills at 48 regs
-            if ((1 << (LOGN - 12)) < cl) cl = 1;
+            // few rows (<= half the SM count, e.g. one ciphertext at L = 36): 8-CTA clusters put
+            // ~4 CTAs per SM to work on them (config 2: 2105 -> 2485 KOPS, profiles/r01/f4)
+            if (!p->v8_cl && (LOGN == 15 || LOGN == 16) && rows * 8 <= (uint32_t)p->sm_count * 4) cl = 8;
+            if ((1 << (LOGN - 12)) < cl || (cl == 8 && (LOGN < 15 || LOGN > 16))) cl = 1;
             if (cl == 1) launch_v8<LOGN>(minb, fwd, a, rows, p->sm_count, s);
             else if (cl == 2) {
                 if (minb == 4) launch_v8_cluster<LOGN, 4, 2>(fwd, a, rows, s);
                 else if (LOGN == 16 && minb == 3) { if constexpr (LOGN == 16) launch_v8_cluster<LOGN, 3, 2>(fwd, a, rows, s); }
                 else launch_v8_cluster<LOGN, 5, 2>(fwd, a, rows, s);
+            } else if (cl == 8) {
+                if constexpr (LOGN >= 15 && LOGN <= 16) launch_v8_cluster<LOGN, 4, 8>(fwd, a, rows, s);
             } else {
                 if (minb == 4) launch_v8_cluster<LOGN, 4, 4>(fwd, a, rows, s);
                 else launch_v8_cluster<LOGN, 5, 4>(fwd, a, rows, s);
@@ -691,7 +696,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     p->kernel_ver = 0;   // AUTO: v8 at >= SM-count rows; below: v5 (2^15, 2^16), v6 (2^17), v1 (<= 2^14)
     if (const char* ev = getenv("WD_NTT_CTAS")) p->v6_ctas = std::max(1, std::min(4, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_MINB")) p->v8_minb = std::max(3, std::min(6, atoi(ev)));
-    if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
+    if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 8 ? 8 : atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
     if (const char* ev = getenv("WD_NTT_STAGGER")) p->stagger_ns = (uint32_t)atoi(ev);
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
