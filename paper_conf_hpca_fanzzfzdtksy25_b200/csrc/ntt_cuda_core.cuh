@@ -42,6 +42,10 @@ struct NttArgs {
     // v8 only: rows between consecutive polynomials in `in` / `out` (0 = L, contiguous); lets a
     // launch cover a limb SECTION of a wider [batch][Lfull][N] tensor (ModUp / ModDown, ntt_rns.cuh)
     uint32_t in_ls = 0, out_ls = 0;
+    // v8 inverse only: if set, every input row is also copied unchanged to cpy (rows between
+    // polynomials: cpy_ls) as it is staged -- ModUp's pass-through of the Q limbs (ntt_rns.cuh)
+    uint32_t* cpy = nullptr;
+    uint32_t cpy_ls = 0;
     uint32_t stagger_ns = 0;         // v8 experiment knob (WD_NTT_STAGGER): grid quarters start k * this apart
 };
 

@@ -132,6 +132,121 @@ __global__ void __launch_bounds__(BC_T) rns_bconv(const uint32_t* __restrict__ x
     }
 }
 
+// Few targets (D <= 4: ModUp with k <= 4 special primes) and many sources: each thread takes 4
+// consecutive coefficients (16-byte loads: a CTA reads 2 KB contiguous per source row, where
+// rns_bconv reads 512 B with scalar loads), the per-source terms [x_i (Q/q_i)^-1]_{q_i} go
+// straight from registers into 64-bit accumulators -- no shared-memory staging of the S terms --
+// and BCF_U source rows are loaded per batch.  Same arithmetic and the same result as
+// rns_bconv's 64-bit MAC path: a Barrett reduction after every BCF_U (< 15) products.
+constexpr int BCF_U = 8;
+constexpr int BCF_C = 4 * BC_T;                  // coefficients per CTA
+template <int D>
+__global__ void __launch_bounds__(BC_T) rns_bconv_few(const uint32_t* __restrict__ x, uint32_t x_ls,
+                                                      uint32_t* __restrict__ y, uint32_t y_ls, uint32_t y_off,
+                                                      BconvTab tab, uint32_t N, uint32_t batch) {
+    extern __shared__ uint4 bsm4[];
+    uint4* src = bsm4;                                   // [S]
+    uint4* dst = bsm4 + tab.S;                           // [D]
+    uint2* ws = reinterpret_cast<uint2*>(bsm4 + tab.S + D);                  // [S][D]
+    for (uint32_t i = threadIdx.x; i < tab.S; i += BC_T) src[i] = tab.src[i];
+    for (uint32_t i = threadIdx.x; i < D; i += BC_T) dst[i] = tab.dst[i];
+    for (uint32_t i = threadIdx.x; i < tab.S * D; i += BC_T) ws[i] = tab.w[i];
+    __syncthreads();
+    const uint32_t per_poly = N / BCF_C;
+    for (uint32_t blk = blockIdx.x; blk < batch * per_poly; blk += gridDim.x) {
+        const uint32_t b = blk / per_poly, n = (blk % per_poly) * BCF_C + 4 * threadIdx.x;
+        const uint4* xb = reinterpret_cast<const uint4*>(x + (size_t)b * x_ls * N + n);
+        const uint32_t n4 = N / 4;
+        uint64_t acc[4][D];
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+            for (int j = 0; j < D; ++j) acc[c][j] = 0;
+        for (uint32_t i0 = 0; i0 < tab.S; i0 += BCF_U) {
+            uint4 v[BCF_U];
+#pragma unroll
+            for (int u = 0; u < BCF_U; ++u) v[u] = i0 + u < tab.S ? __ldcs(xb + (size_t)(i0 + u) * n4) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+            for (int u = 0; u < BCF_U; ++u)
+                if (i0 + u < tab.S) {
+                    const uint4 sc = src[i0 + u];
+                    const uint32_t yv[4] = {canon2(shoup_mul(v[u].x, sc.y, sc.z, sc.x), sc.x),
+                                            canon2(shoup_mul(v[u].y, sc.y, sc.z, sc.x), sc.x),
+                                            canon2(shoup_mul(v[u].z, sc.y, sc.z, sc.x), sc.x),
+                                            canon2(shoup_mul(v[u].w, sc.y, sc.z, sc.x), sc.x)};
+#pragma unroll
+                    for (int j = 0; j < D; ++j) {
+                        const uint32_t w = ws[(i0 + u) * D + j].x;
+#pragma unroll
+                        for (int c = 0; c < 4; ++c) acc[c][j] += (uint64_t)yv[c] * w;
+                    }
+                }
+#pragma unroll
+            for (int j = 0; j < D; ++j) {
+                const uint4 d = dst[j];
+                const uint64_t mu = ((uint64_t)d.z << 32) | d.y;
+#pragma unroll
+                for (int c = 0; c < 4; ++c) acc[c][j] = reduce64(acc[c][j], d.x, mu);
+            }
+        }
+        uint32_t* yb = y + ((size_t)b * y_ls + y_off) * N + n;
+#pragma unroll
+        for (int j = 0; j < D; ++j)
+            __stcs(reinterpret_cast<uint4*>(yb + (size_t)j * N),
+                   make_uint4((uint32_t)acc[0][j], (uint32_t)acc[1][j], (uint32_t)acc[2][j], (uint32_t)acc[3][j]));
+    }
+}
+
+// Few sources (S <= 4: ModDown with k <= 4 special primes) and many targets: 4 consecutive
+// coefficients per thread, the S terms in registers, and one 16-byte streaming store per target
+// row (a CTA writes 2 KB contiguous per target row; rns_bconv writes 512 B with scalar stores).
+// Same lazy Shoup sum in [0, 2p) and the same canonical result as rns_bconv's few-terms path.
+template <int S>
+__global__ void __launch_bounds__(BC_T) rns_bconv_fewsrc(const uint32_t* __restrict__ x, uint32_t x_ls,
+                                                         uint32_t* __restrict__ y, uint32_t y_ls, uint32_t y_off,
+                                                         BconvTab tab, uint32_t N, uint32_t batch) {
+    extern __shared__ uint4 bsm4[];
+    uint4* src = bsm4;                                   // [S]
+    uint4* dst = bsm4 + S;                               // [D]
+    uint2* ws = reinterpret_cast<uint2*>(bsm4 + S + tab.D);                  // [S][D]
+    for (uint32_t i = threadIdx.x; i < S; i += BC_T) src[i] = tab.src[i];
+    for (uint32_t i = threadIdx.x; i < tab.D; i += BC_T) dst[i] = tab.dst[i];
+    for (uint32_t i = threadIdx.x; i < S * tab.D; i += BC_T) ws[i] = tab.w[i];
+    __syncthreads();
+    const uint32_t per_poly = N / BCF_C;
+    for (uint32_t blk = blockIdx.x; blk < batch * per_poly; blk += gridDim.x) {
+        const uint32_t b = blk / per_poly, n = (blk % per_poly) * BCF_C + 4 * threadIdx.x;
+        const uint4* xb = reinterpret_cast<const uint4*>(x + (size_t)b * x_ls * N + n);
+        uint32_t yv[S][4];
+#pragma unroll
+        for (int i = 0; i < S; ++i) {
+            const uint4 v = __ldcs(xb + (size_t)i * (N / 4));
+            const uint4 sc = src[i];
+            yv[i][0] = canon2(shoup_mul(v.x, sc.y, sc.z, sc.x), sc.x);
+            yv[i][1] = canon2(shoup_mul(v.y, sc.y, sc.z, sc.x), sc.x);
+            yv[i][2] = canon2(shoup_mul(v.z, sc.y, sc.z, sc.x), sc.x);
+            yv[i][3] = canon2(shoup_mul(v.w, sc.y, sc.z, sc.x), sc.x);
+        }
+        uint32_t* yb = y + ((size_t)b * y_ls + y_off) * N + n;
+#pragma unroll 2
+        for (uint32_t j = 0; j < tab.D; ++j) {
+            const uint32_t p = dst[j].x;
+            uint32_t r[4] = {0, 0, 0, 0};
+#pragma unroll
+            for (int i = 0; i < S; ++i) {
+                const uint2 w = ws[i * tab.D + j];
+#pragma unroll
+                for (int c = 0; c < 4; ++c) {
+                    r[c] += shoup_mul(yv[i][c], w.x, w.y, p);
+                    r[c] = umin32(r[c], r[c] - 2 * p);
+                }
+            }
+            __stcs(reinterpret_cast<uint4*>(yb + (size_t)j * N),
+                   make_uint4(canon2(r[0], p), canon2(r[1], p), canon2(r[2], p), canon2(r[3], p)));
+        }
+    }
+}
+
 // sum [rows][N] 64-bit (the all-reduced shard partials) -> canonical residue mod p_{row % D}
 __global__ void __launch_bounds__(256) rns_reduce64(const unsigned long long* __restrict__ sum, uint32_t* __restrict__ out,
                                                     const uint4* __restrict__ dst, uint32_t D, uint32_t N, uint32_t rows) {

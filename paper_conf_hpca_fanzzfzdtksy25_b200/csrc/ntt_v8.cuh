@@ -340,6 +340,16 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                 if constexpr (!JIT3) load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);   // in flight across the wait
                 cp_async_wait<0>();
                 __syncwarp();                            // this warp's rows of sub-row s landed
+                if (a.cpy) {                             // ModUp: pass the NTT-domain input through
+                    const int wbase = (t >> 5) * 512 + 4 * (t & 31);
+                    uint32_t* cp = a.cpy + ((size_t)row_map(row, a.L, a.cpy_ls) << LOGN) + s * V8_SUBW;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {        // the warp's own 2 KB slice, 512 B per store
+                        const int e = wbase + 128 * v;
+                        __stcs(reinterpret_cast<uint4*>(cp + e),
+                               *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15)));
+                    }
+                }
                 uint32_t x[16];
                 {   // stage 3': layers A+11..A+8, thread (a, b), 16 contiguous elements
                     const int aa = hi4, b = lo4;

@@ -642,6 +642,28 @@ void launch_v8_rows(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t r
 
 int launch_bconv(const wd_ntt_plan* p, const uint32_t* x, uint32_t x_ls, uint32_t* y, uint32_t y_ls, uint32_t y_off,
                  const BconvTab& t, uint32_t batch, cudaStream_t s) {
+    if (t.D <= 4 && t.S > 4 && p->N >= (uint32_t)BCF_C) {   // few targets: register accumulation
+        const size_t sm = sizeof(uint4) * (t.S + t.D) + sizeof(uint2) * t.S * t.D;
+        const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)batch * (p->N / BCF_C), (uint64_t)p->sm_count * 8);
+        switch (t.D) {
+            case 1: rns_bconv_few<1><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+            case 2: rns_bconv_few<2><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+            case 3: rns_bconv_few<3><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+            default: rns_bconv_few<4><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+        }
+        return WD_OK;
+    }
+    if (t.S <= 4 && p->N >= (uint32_t)BCF_C) {         // few sources: terms in registers, 16-B stores
+        const size_t sm = sizeof(uint4) * (t.S + t.D) + sizeof(uint2) * t.S * t.D;
+        const uint32_t blocks = (uint32_t)std::min<uint64_t>((uint64_t)batch * (p->N / BCF_C), (uint64_t)p->sm_count * 8);
+        switch (t.S) {
+            case 1: rns_bconv_fewsrc<1><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+            case 2: rns_bconv_fewsrc<2><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+            case 3: rns_bconv_fewsrc<3><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+            default: rns_bconv_fewsrc<4><<<blocks, BC_T, sm, s>>>(x, x_ls, y, y_ls, y_off, t, p->N, batch); break;
+        }
+        return WD_OK;
+    }
     const size_t smem = sizeof(uint4) * (t.S + t.D) + sizeof(uint2) * t.S * t.D + sizeof(uint32_t) * t.S * BC_T;
     if (smem > 48 * 1024 && cudaFuncSetAttribute(rns_bconv, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
         return WD_ECUDA;
@@ -867,10 +889,19 @@ int wd_modup(const wd_rns_conv* c, const uint32_t* in, uint32_t* out, uint32_t b
     // K1: INTT of the Q limbs -> work [batch][a][N]
     NttArgs ai;
     ai.in = in; ai.in2 = nullptr; ai.out = work; ai.tw = pq->d_inv; ai.lc = pq->d_lc; ai.L = a;
-    uint32_t launches = (uint32_t)launch_cuda_core(pq, false, ai, batch * a, s);
-    // the Q limbs pass through unchanged (NTT domain)
-    if (cudaMemcpy2DAsync(out, (size_t)(a + k) * N * 4, in, (size_t)a * N * 4, (size_t)a * N * 4, batch,
-                          cudaMemcpyDeviceToDevice, s) != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    uint32_t launches;
+    if (pq->logN >= 12 && pq->kernel_ver == 0) {
+        // v8 copies the Q limbs (NTT domain, unchanged) into out as it stages them: one read of
+        // the input instead of two (the separate 2-D copy cost ~0.4 ms at config 3)
+        ai.cpy = out; ai.cpy_ls = a + k;
+        launch_v8_rows<0>(pq, false, ai, batch * a, s);
+        launches = 1;
+    } else {
+        launches = (uint32_t)launch_cuda_core(pq, false, ai, batch * a, s);
+        // the Q limbs pass through unchanged (NTT domain)
+        if (cudaMemcpy2DAsync(out, (size_t)(a + k) * N * 4, in, (size_t)a * N * 4, (size_t)a * N * 4, batch,
+                              cudaMemcpyDeviceToDevice, s) != cudaSuccess) { cudaGetLastError(); return set_err(WD_ECUDA); }
+    }
     // K2: BConv Q -> P into the P section of out (coefficient domain)
     BconvTab t{c->d_up_src, c->d_up_w, c->d_up_dst, a, k};
     if (launch_bconv(pq, work, a, out, a + k, a, t, batch, s) != WD_OK) return set_err(WD_ECUDA);

@@ -14,7 +14,7 @@ import oracle  # noqa: E402
 from oracle import rns  # noqa: E402
 from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs  # noqa: E402
 
-P = inputs.bench_primes(60)
+P = inputs.bench_primes(110)
 SMALL = [786433, 269221889, 537133057, 805961729]
 
 
@@ -145,6 +145,18 @@ def test_modup_moddown_keyswitch_shape(wd):
     for b in (0, 5):
         assert np.array_equal(up[b:b + 1], rns.modup(x[b:b + 1], qs, ps)), b
         assert np.array_equal(dn[b:b + 1], rns.moddown(up[b:b + 1], qs, ps)), b
+
+
+@pytest.mark.parametrize("logn,a,k,batch", [(13, 6, 4, 3), (14, 9, 2, 2), (12, 37, 1, 2)])
+def test_modup_few_targets_many_sources(wd, logn, a, k, batch):
+    # rns_bconv_few (S > 4 sources, D <= 4 targets: register accumulation, Barrett every 12
+    # terms) and ModUp's Q-limb pass-through fused into the v8 INTT
+    n, qs, ps = 1 << logn, P[:a], P[100:100 + k]
+    pq, pp = wd.Plan(n, qs), wd.Plan(n, ps)
+    conv = wd.RnsConv(pq, pp)
+    x = inputs.uniform_residues(qs, n, batch, 8800 + logn)
+    up = to_host(conv.modup(to_dev(x)))
+    assert np.array_equal(up, rns.modup(x, qs, ps))
 
 
 def test_modup_many_rows_and_wide_bases(wd):
