@@ -19,6 +19,7 @@
 #include "ntt_cuda_core.cuh"
 #include "ntt_persist.cuh"
 #include "ntt_v8.cuh"
+#include "ntt_v12.cuh"
 #include "ntt_smem.cuh"
 #include "ntt_cluster.cuh"
 #include "ntt_tensor.cuh"
@@ -271,6 +272,22 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         }
     }
     if constexpr (LOGN >= 12) {
+        if constexpr (LOGN == 15 || LOGN == 16) {
+            if (fwd && p->kernel_ver == 12) {            // v12: phases of consecutive rows interleaved
+                cudaLaunchConfig_t cfg = {};
+                cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V12_SMEM; cfg.stream = s;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+                cfg.attrs = at; cfg.numAttrs = 1;
+                int ncl = 0;
+                cfg.gridDim = dim3(148 * 4);
+                if (cudaOccupancyMaxActiveClusters(&ncl, ntt_v12f<LOGN>, &cfg) != cudaSuccess || ncl < 1) { cudaGetLastError(); ncl = 1; }
+                cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)ncl) * 2);
+                cudaLaunchKernelEx(&cfg, ntt_v12f<LOGN>, a, rows);
+                return;
+            }
+        }
         if (fwd && p->kernel_ver == 86) { ntt_v8<LOGN, true, false, 6><<<p->sm_count * 4, V8_T, V8_SMEM, s>>>(a, rows); return; }
         if (fwd && p->kernel_ver == 88) {   // v8 (2-CTA cluster) with the old per-thread 64-byte stores
             cudaLaunchConfig_t cfg = {};
@@ -327,7 +344,7 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
         }
         const bool autov8 = p->kernel_ver == 0 && (rows >= (uint32_t)p->sm_count ||
                                                    ((LOGN == 15 || LOGN == 16) && rows >= (uint32_t)p->sm_count / 4));
-        if (p->kernel_ver == 8 || autov8) {
+        if (p->kernel_ver == 8 || p->kernel_ver == 12 || autov8) {
             int minb = p->v8_minb ? p->v8_minb : V8_DEFAULT_MINB;
             int cl = p->v8_cl ? p->v8_cl : V8_DEFAULT_CL;
             if (LOGN == 17 && fwd && !p->v8_minb) minb = 4;     // radix-32 column phase spills at 48 regs

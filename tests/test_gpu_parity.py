@@ -249,7 +249,7 @@ def test_modes_headline_config(wd, mode, share):
 
 
 # -------------------------------------------------------------- every CUDA-core kernel generation
-@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8", "v9", "v10", "v11"])
+@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8", "v9", "v10", "v11", "v12"])
 @pytest.mark.parametrize("logn", [12, 13, 14, 15, 16, 17])
 def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
@@ -276,8 +276,8 @@ def test_cuda_core_generations(wd, ver, logn, monkeypatch):
 # More rows than resident CTAs (clusters), so every CTA walks several rows and the cross-row
 # prefetches (v9: next row's first unit staged during the current row) are exercised; the row
 # count is ragged with respect to the grid.
-@pytest.mark.parametrize("ver", ["v8", "v9", "v10", "v11"])
-@pytest.mark.parametrize("logn,batch", [(14, 161), (16, 83)])
+@pytest.mark.parametrize("ver", ["v8", "v9", "v10", "v11", "v12"])
+@pytest.mark.parametrize("logn,batch", [(14, 161), (15, 97), (16, 83)])
 def test_persistent_many_rows(wd, ver, logn, batch, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
     n = 1 << logn
@@ -293,7 +293,7 @@ def test_persistent_many_rows(wd, ver, logn, batch, monkeypatch):
 # Primes across the range the ABI accepts: the tensor column phase (v10) recombines its byte
 # planes with a cheaper reduction when q > 2^29 and a general one below; both must be exact.
 # 786433 = 3 * 2^18 + 1; the others are the first primes = 1 (mod 2^17) above 2^28, 2^29, 1.5*2^29.
-@pytest.mark.parametrize("ver", ["v8", "v10", "v11"])
+@pytest.mark.parametrize("ver", ["v8", "v10", "v11", "v12"])
 def test_prime_sizes_n16(wd, ver, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
     n = 1 << 16
