@@ -285,6 +285,62 @@ def run_modupdown(args):
     print(json.dumps(line), flush=True)
 
 
+def run_polymul(args):
+    """--op polymul: the negacyclic polynomial product c = INTT(NTT(a) o NTT(b)) mod (X^N + 1, q_l)
+    of SURVEY.md 8 row f1 (the HMULT tensor-product step), at the config shape (default c3:
+    N=2^16, L=36, 128 polynomial pairs).  One step = two forward launches and one fused
+    pointwise-product + inverse launch over every pair; value = polynomial products per second.
+    Roofline: HBM, algorithmic bytes = read a and b, write c (12*N bytes per row); the three
+    launches move 28*N bytes per row (the NTT-domain operands round-trip through HBM)."""
+    import torch
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt
+    torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+    logn, L, nct = CONFIGS[args.config]
+    n = 1 << logn
+    batch = 1 if nct is None else 2 * nct
+    primes = inputs.bench_primes(L)
+    plan = wdntt.Plan(n, primes)
+    xa = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 2, device="cuda")
+    xb = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 3, device="cuda")
+    ya, yb, c = torch.empty_like(xa), torch.empty_like(xa), torch.empty_like(xa)
+    sp = torch.cuda.current_stream().cuda_stream
+
+    def step():
+        wdntt.wd_ntt_forward(plan.handle, xa, ya, batch, sp)
+        n0 = wdntt.wd_ntt_last_launches()
+        wdntt.wd_ntt_forward(plan.handle, xb, yb, batch, sp)
+        n1 = wdntt.wd_ntt_last_launches()
+        wdntt.wd_ntt_pointwise_inverse(plan.handle, ya, yb, c, batch, sp)
+        return n0 + n1 + wdntt.wd_ntt_last_launches()
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    launches = 0
+    with ClockSampler(0) as clk:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(args.steps):
+            launches += step()
+        e1.record()
+        torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    pk, pk_kind = peaks()
+    hbm = float(pk.get("hbm_gbs", FALLBACK_HBM_GBS))
+    alg = batch * L * n * 12.0
+    line = {"metric": "negacyclic polynomial multiply throughput (N=2^%d, L=%d)" % (logn, L),
+            "value": batch / (ms / 1e3), "unit": "polynomial products/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic (splitmix64 uniform residues)",
+            "config": {"workload": "%s: %d polynomial pairs, NTT(a), NTT(b), fused pointwise product + INTT"
+                                   % (CONFIG_NAMES[args.config], batch), "N": n, "L": L, "polys": batch},
+            "roofline": {"bound": "hbm", "kernel": "whole op (3 launches)", "achieved": alg / (ms / 1e3) / 1e9,
+                         "peak": hbm, "unit": "GB/s", "frac": alg / (ms / 1e3) / 1e9 / hbm, "traffic": None,
+                         "peak_kind": pk_kind, "algorithmic_bytes_per_step": alg},
+            "gpu_launches": launches, "clocks": clk.summary()}
+    print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -297,9 +353,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
-    ap.add_argument("--op", default="ntt", choices=["ntt", "rescale", "modup", "moddown"],
+    ap.add_argument("--op", default="ntt", choices=["ntt", "rescale", "modup", "moddown", "polymul"],
                     help="ntt: the headline forward+inverse step; rescale: SURVEY.md 8 row f4; "
-                         "modup / moddown: row f3 (KeySwitch basis changes)")
+                         "modup / moddown: row f3 (KeySwitch basis changes); polymul: row f1")
     ap.add_argument("--k", type=int, default=1, help="special primes for --op modup/moddown (PAPER.md Table III: K=1)")
     args = ap.parse_args()
     if args.op == "rescale":
@@ -307,6 +363,9 @@ def main():
         return
     if args.op in ("modup", "moddown"):
         run_modupdown(args)
+        return
+    if args.op == "polymul":
+        run_polymul(args)
         return
 
     if args.impl == "reference":

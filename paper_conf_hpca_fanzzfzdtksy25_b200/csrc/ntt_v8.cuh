@@ -350,6 +350,21 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                                *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15)));
                     }
                 }
+                if constexpr (PW) {                      // row f1: pointwise product, coalesced
+                    // the warp's own 2 KB slice: in2 read 512 B per instruction, the product
+                    // written back to the same shared-memory slots before stage 3' reads them
+                    const int wbase = (t >> 5) * 512 + 4 * (t & 31);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const int e = wbase + 128 * v;
+                        uint4* sp = reinterpret_cast<uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
+                        const uint4 u = *sp;
+                        const uint4 m = __ldcs(reinterpret_cast<const uint4*>(in2 + s * V8_SUBW + e));
+                        *sp = make_uint4(mul_mod(u.x, m.x, lc), mul_mod(u.y, m.y, lc), mul_mod(u.z, m.z, lc),
+                                         mul_mod(u.w, m.w, lc));
+                    }
+                    __syncwarp();
+                }
                 uint32_t x[16];
                 {   // stage 3': layers A+11..A+8, thread (a, b), 16 contiguous elements
                     const int aa = hi4, b = lo4;
@@ -359,15 +374,6 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     for (int v = 0; v < 4; ++v) {
                         const uint4 u = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
                         x[4 * v] = u.x; x[4 * v + 1] = u.y; x[4 * v + 2] = u.z; x[4 * v + 3] = u.w;
-                    }
-                    if constexpr (PW) {
-                        const uint4* ip2 = reinterpret_cast<const uint4*>(in2 + s * V8_SUBW + t * 16);
-#pragma unroll
-                        for (int v = 0; v < 4; ++v) {
-                            const uint4 u = __ldcs(ip2 + v);
-                            x[4 * v] = mul_mod(x[4 * v], u.x, lc); x[4 * v + 1] = mul_mod(x[4 * v + 1], u.y, lc);
-                            x[4 * v + 2] = mul_mod(x[4 * v + 2], u.z, lc); x[4 * v + 3] = mul_mod(x[4 * v + 3], u.w, lc);
-                        }
                     }
                     if constexpr (JIT3) inv_radix<4, false>(x, tw, A + 8, (uint32_t)s * 256 + t, lc);
                     else inv16_tw(x, w3, q, q2);
