@@ -214,6 +214,18 @@ int      wd_ntt_check_prime(uint32_t q, uint32_t N);
 int wd_ntt_plan_set_mode(wd_ntt_plan* plan, int mode, float tensor_share);
 int wd_ntt_plan_get_mode(const wd_ntt_plan* plan);
 
+/* Row a9's split "chosen from measurement" (the WD-FUSE ratio follows
+ * the units' measured throughput): times one forward + inverse over `batch` polynomials of
+ * scratch data (allocated and freed inside the call, zero residues) for every execution path
+ * available at this N -- WD_MODE_CUDA, and for N = 2^16 also WD_MODE_FUSED (phase-split
+ * pipeline and row splits with tensor_share 0.25 / 0.5 / 0.75), WD_MODE_TENSOR and
+ * WD_MODE_CUDA_GEMM -- with CUDA events on `stream`, and sets the plan to the fastest.
+ * Writes that path's milliseconds per forward + inverse to *best_ms if best_ms != NULL.
+ * Synchronises `stream`.  Returns WD_OK, WD_EINVAL (NULL plan, batch == 0, wrong device) or
+ * WD_ECUDA (allocation or launch failure; the plan's mode is then unchanged).  Not
+ * thread-safe against concurrent calls using the same plan. */
+int wd_ntt_plan_autotune(wd_ntt_plan* plan, uint32_t batch, wd_stream_t stream, float* best_ms);
+
 /* Kernel launches issued by the last forward/inverse call on this thread. */
 uint32_t wd_ntt_last_launches(void);
 

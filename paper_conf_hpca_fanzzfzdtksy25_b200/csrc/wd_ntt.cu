@@ -1046,6 +1046,66 @@ int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
 }
 int wd_ntt_plan_get_mode(const wd_ntt_plan* p) { return p ? effective_mode(p) : -1; }
 
+int wd_ntt_plan_autotune(wd_ntt_plan* p, uint32_t batch, wd_stream_t st, float* best_ms) {
+    if (!p || batch == 0) return set_err(WD_EINVAL);
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) return set_err(WD_EINVAL);
+    if ((uint64_t)batch * p->L > 0x7fffffffull) return set_err(WD_EINVAL);
+    cudaStream_t s = (cudaStream_t)st;
+    const size_t bytes = sizeof(uint32_t) * (size_t)batch * p->L * p->N;
+    uint32_t *x = nullptr, *y = nullptr;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    auto cleanup = [&]() {
+        if (x) cudaFree(x);
+        if (y) cudaFree(y);
+        if (e0) cudaEventDestroy(e0);
+        if (e1) cudaEventDestroy(e1);
+    };
+    if (cudaMalloc(&x, bytes) != cudaSuccess || cudaMalloc(&y, bytes) != cudaSuccess ||
+        cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess ||
+        cudaMemsetAsync(x, 0, bytes, s) != cudaSuccess) {
+        cudaGetLastError(); cleanup(); return set_err(WD_ECUDA);
+    }
+    struct Cand { int mode; float share; };
+    std::vector<Cand> cands = {{WD_MODE_CUDA, p->tensor_share}};
+    if (tensor_supported(p->logN) && p->tc.ok) {
+        cands.push_back({WD_MODE_FUSED, default_tensor_share(p->logN)});
+        for (float sh : {0.25f, 0.5f, 0.75f}) cands.push_back({WD_MODE_FUSED, sh});
+        cands.push_back({WD_MODE_TENSOR, p->tensor_share});
+        if (p->logN == 16) cands.push_back({WD_MODE_CUDA_GEMM, p->tensor_share});
+    }
+    const int mode0 = p->mode;
+    const float share0 = p->tensor_share;
+    int best = -1;
+    float best_t = 0.0f;
+    for (size_t i = 0; i < cands.size(); ++i) {
+        p->mode = cands[i].mode;
+        p->tensor_share = cands[i].share;
+        bool ok = run(p, true, x, nullptr, y, batch, s) == WD_OK && run(p, false, y, nullptr, x, batch, s) == WD_OK;
+        float t = 0.0f;
+        if (ok) {                                        // one warm-up pair, then 3 timed pairs
+            cudaEventRecord(e0, s);
+            for (int k = 0; k < 3 && ok; ++k)
+                ok = run(p, true, x, nullptr, y, batch, s) == WD_OK && run(p, false, y, nullptr, x, batch, s) == WD_OK;
+            cudaEventRecord(e1, s);
+            ok = ok && cudaEventSynchronize(e1) == cudaSuccess && cudaEventElapsedTime(&t, e0, e1) == cudaSuccess;
+        }
+        if (!ok) {
+            if (cudaGetLastError() != cudaSuccess || cands[i].mode == WD_MODE_CUDA) {
+                p->mode = mode0; p->tensor_share = share0; cleanup(); return set_err(WD_ECUDA);
+            }
+            continue;                                    // this path is unsupported here: skip it
+        }
+        t /= 3.0f;
+        if (best < 0 || t < best_t) { best = (int)i; best_t = t; }
+    }
+    cleanup();
+    p->mode = cands[best].mode;
+    p->tensor_share = cands[best].share;
+    if (best_ms) *best_ms = best_t;
+    return set_err(WD_OK);
+}
+
 uint32_t wd_ntt_last_launches(void) { return g_last_launches; }
 
 int wd_ntt_occupancy(const wd_ntt_plan* p, int mode, int fwd) {

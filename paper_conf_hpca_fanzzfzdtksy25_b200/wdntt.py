@@ -61,6 +61,7 @@ _SIGS = {
     "wd_ntt_root": (_u32, [_u32, _u32]),
     "wd_ntt_check_prime": (_i32, [_u32, _u32]),
     "wd_ntt_plan_set_mode": (_i32, [_vp, _i32, _f32]),
+    "wd_ntt_plan_autotune": (_i32, [_vp, _u32, _vp, ctypes.POINTER(ctypes.c_float)]),
     "wd_ntt_plan_get_mode": (_i32, [_vp]),
     "wd_ntt_last_launches": (_u32, []),
     "wd_ntt_occupancy": (_i32, [_vp, _i32, _i32]),
@@ -246,6 +247,15 @@ class Plan:
 
     def set_mode(self, mode, tensor_share: float = -1.0):
         wd_ntt_plan_set_mode(self.handle, mode, tensor_share)
+
+    def autotune(self, batch: int, stream=None):
+        """Time every execution path on ``batch`` scratch polynomials and keep the fastest
+        (wd_ntt_plan_autotune).  Returns (mode, ms per forward + inverse)."""
+        import torch
+        ms = ctypes.c_float(0.0)
+        st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        _check(_lib.wd_ntt_plan_autotune(self.handle, int(batch), st, ctypes.byref(ms)), "wd_ntt_plan_autotune")
+        return _lib.wd_ntt_plan_get_mode(self.handle), ms.value
 
     def psi(self, limb: int) -> int:
         return wd_ntt_plan_psi(self.handle, limb)

@@ -63,6 +63,7 @@ def test_calls_reject_null_plan():
     assert wdntt._lib.wd_ntt_forward(None, 16, 16, 1, None) == wdntt.WD_EINVAL
     assert wdntt._lib.wd_ntt_inverse(None, 16, 16, 1, None) == wdntt.WD_EINVAL
     assert wdntt._lib.wd_ntt_forward_host(None, 16, 16, 1, 16, None) == wdntt.WD_EINVAL
+    assert wdntt._lib.wd_ntt_plan_autotune(None, 1, None, None) == wdntt.WD_EINVAL
     assert wdntt.wd_ntt_strerror(wdntt.WD_EPRIME).startswith("modulus")
 
 

@@ -341,3 +341,21 @@ def test_v11_stage_splits(wd, tmask, monkeypatch):
     assert np.array_equal(y, oracle.ntt_forward(x, primes)), tmask
     assert np.array_equal(gpu_inv(wd, plan, y), x), tmask
     assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), tmask
+
+
+# -------------------------------------------------------------- row a9: split chosen from measurement
+@pytest.mark.parametrize("logn,batch", [(16, 16), (14, 8)])
+def test_autotune_picks_a_path_and_stays_exact(wd, logn, batch):
+    n = 1 << logn
+    primes = [P[3], P[17], P[40]]
+    plan = wd.Plan(n, primes)
+    mode, ms = plan.autotune(batch)
+    assert ms > 0
+    if logn == 16:
+        assert mode in (1, 2, 3, 4)
+    else:
+        assert mode == 1                                   # only the CUDA-core path below 2^16
+    x = inputs.uniform_residues(primes, n, batch, 6100 + logn)
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (mode, logn)
+    assert np.array_equal(gpu_inv(wd, plan, y), x), (mode, logn)
