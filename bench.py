@@ -37,6 +37,7 @@ CONFIGS = {
     # batch-1 small cases (config 5's "batch 1" end): kernel-selection data, not bench lines
     "t15": (15, 36, 1),
     "t16": (16, 16, 1),
+    "t17": (17, 36, 1),
 }
 # config 5 (the N sweep, BASELINE configs[4]) at batch 128 polynomials, 16 limbs: parity cases
 # and kernel-selection data, not bench lines
@@ -44,7 +45,8 @@ for _lg in range(12, 18):
     CONFIGS["s%d" % _lg] = (_lg, 16, 64)
 CONFIG_NAMES = {"c1": "config1 (BASELINE configs[0])", "c2": "config2 (one ciphertext)",
                 "c3": "config3 (BASELINE configs[2], headline)", "c4": "config4 per-GPU shard"}
-CONFIG_NAMES.update({"t15": "config5 point N=2^15, L=36, one ciphertext", "t16": "config5 point N=2^16, L=16, one ciphertext"})
+CONFIG_NAMES.update({"t15": "config5 point N=2^15, L=36, one ciphertext", "t16": "config5 point N=2^16, L=16, one ciphertext",
+                    "t17": "config5 point N=2^17, L=36, one ciphertext"})
 CONFIG_NAMES.update({"s%d" % _lg: "config5 sweep point N=2^%d, L=16, 128 polynomials" % _lg for _lg in range(12, 18)})
 METRIC = "NTT KOPS (N=2^16, L=36) at 1/2/4/8 B200; % of HBM / int8 tensor roofline"
 FALLBACK_HBM_GBS = 6650.0

@@ -343,22 +343,25 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             return;
         }
         const bool autov8 = p->kernel_ver == 0 && (rows >= (uint32_t)p->sm_count ||
-                                                   ((LOGN == 15 || LOGN == 16) && rows >= (uint32_t)p->sm_count / 4));
+                                                   ((LOGN == 15 || LOGN == 16) && rows >= (uint32_t)p->sm_count / 4) ||
+                                                   LOGN == 17);
         if (p->kernel_ver == 8 || p->kernel_ver == 12 || autov8) {
             int minb = p->v8_minb ? p->v8_minb : V8_DEFAULT_MINB;
             int cl = p->v8_cl ? p->v8_cl : V8_DEFAULT_CL;
             if (LOGN == 17 && fwd && !p->v8_minb) minb = 4;     // radix-32 column phase spills at 48 regs
             // few rows (<= half the SM count, e.g. one ciphertext at L = 36): 8-CTA clusters put
             // ~4 CTAs per SM to work on them (config 2: 2105 -> 2485 KOPS, profiles/r01/f4)
-            if (!p->v8_cl && (LOGN == 15 || LOGN == 16) && rows * 8 <= (uint32_t)p->sm_count * 4) cl = 8;
-            if ((1 << (LOGN - 12)) < cl || (cl == 8 && (LOGN < 15 || LOGN > 16))) cl = 1;
+            if (!p->v8_cl && LOGN >= 15 && rows * 8 <= (uint32_t)p->sm_count * 4) cl = 8;
+            // N = 2^17 between half and one SM count of rows: 4-CTA clusters (config 5 sweep)
+            else if (!p->v8_cl && LOGN == 17 && rows <= (uint32_t)p->sm_count) cl = 4;
+            if ((1 << (LOGN - 12)) < cl || (cl == 8 && LOGN < 15)) cl = 1;
             if (cl == 1) launch_v8<LOGN>(minb, fwd, a, rows, p->sm_count, s);
             else if (cl == 2) {
                 if (minb == 4) launch_v8_cluster<LOGN, 4, 2>(fwd, a, rows, s);
                 else if (LOGN == 16 && minb == 3) { if constexpr (LOGN == 16) launch_v8_cluster<LOGN, 3, 2>(fwd, a, rows, s); }
                 else launch_v8_cluster<LOGN, 5, 2>(fwd, a, rows, s);
             } else if (cl == 8) {
-                if constexpr (LOGN >= 15 && LOGN <= 16) launch_v8_cluster<LOGN, 4, 8>(fwd, a, rows, s);
+                if constexpr (LOGN >= 15) launch_v8_cluster<LOGN, 4, 8>(fwd, a, rows, s);
             } else {
                 if (minb == 4) launch_v8_cluster<LOGN, 4, 4>(fwd, a, rows, s);
                 else launch_v8_cluster<LOGN, 5, 4>(fwd, a, rows, s);
