@@ -352,8 +352,8 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             // few rows (<= half the SM count, e.g. one ciphertext at L = 36): 8-CTA clusters put
             // ~4 CTAs per SM to work on them (config 2: 2105 -> 2485 KOPS, profiles/r01/f4)
             if (!p->v8_cl && LOGN >= 15 && rows * 8 <= (uint32_t)p->sm_count * 4) cl = 8;
-            // N = 2^17 between half and one SM count of rows: 4-CTA clusters (config 5 sweep)
-            else if (!p->v8_cl && LOGN == 17 && rows <= (uint32_t)p->sm_count) cl = 4;
+            // between half and one SM count of rows: 4-CTA clusters (config 5 sweep)
+            else if (!p->v8_cl && LOGN >= 15 && rows <= (uint32_t)p->sm_count) cl = 4;
             if ((1 << (LOGN - 12)) < cl || (cl == 8 && LOGN < 15)) cl = 1;
             if (cl == 1) launch_v8<LOGN>(minb, fwd, a, rows, p->sm_count, s);
             else if (cl == 2) {
