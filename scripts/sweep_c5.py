@@ -4,7 +4,7 @@ point: KOPS (single-prime N-point transforms per second, reading C-9) for each d
 HBM fraction of the algorithmic 8N bytes per transform (inputs resident; no L2 flush, so the
 small points are L2-resident and latency-bound, as flagged in SURVEY.md 8.d).
 
-usage: python scripts/sweep_c5.py [--reps 5] > gpurun_out/sweep_c5.jsonl
+usage: python scripts/sweep_c5.py [--reps 10] > gpurun_out/sweep_c5.jsonl
 """
 import argparse
 import json
@@ -16,7 +16,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--reps", type=int, default=10)
     args = ap.parse_args()
     import torch
     from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt
@@ -37,15 +37,27 @@ def main():
                     wdntt.wd_ntt_inverse(plan.handle, y, z, b, sp)
                 torch.cuda.synchronize()
                 assert torch.equal(z, x), (logn, L, nct)
+                # each direction's reps captured in one CUDA graph (the batch-1 points are
+                # launch-bound; as bench.py --graph auto)
+                cs = torch.cuda.Stream()
+                cs.wait_stream(torch.cuda.current_stream())
+                gf, gi = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+                with torch.cuda.graph(gf, stream=cs):
+                    for _ in range(args.reps):
+                        wdntt.wd_ntt_forward(plan.handle, x, y, b, cs.cuda_stream)
+                with torch.cuda.graph(gi, stream=cs):
+                    for _ in range(args.reps):
+                        wdntt.wd_ntt_inverse(plan.handle, y, z, b, cs.cuda_stream)
+                gf.replay(); gi.replay()
+                torch.cuda.synchronize()
                 ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
                 ev[0].record()
-                for _ in range(args.reps):
-                    wdntt.wd_ntt_forward(plan.handle, x, y, b, sp)
+                gf.replay()
                 ev[1].record()
-                for _ in range(args.reps):
-                    wdntt.wd_ntt_inverse(plan.handle, y, z, b, sp)
+                gi.replay()
                 ev[2].record()
                 torch.cuda.synchronize()
+                assert torch.equal(z, x), (logn, L, nct, "graph")
                 fms = ev[0].elapsed_time(ev[1]) / args.reps
                 ims = ev[1].elapsed_time(ev[2]) / args.reps
                 rows = b * L
@@ -54,7 +66,7 @@ def main():
                                   "fwd_kops": rows / fms, "inv_kops": rows / ims,
                                   "hbm_frac_fwd": rows * 8.0 * n / (fms * 1e-3) / 1e9 / peak,
                                   "bytes_in": rows * 4 * n}), flush=True)
-                del x, y, z
+                del x, y, z, gf, gi
             del plan
             torch.cuda.empty_cache()
 
