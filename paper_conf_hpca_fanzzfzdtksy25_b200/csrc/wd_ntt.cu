@@ -352,6 +352,10 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             // few rows (<= half the SM count, e.g. one ciphertext at L = 36): 8-CTA clusters put
             // ~4 CTAs per SM to work on them (config 2: 2105 -> 2485 KOPS, profiles/r01/f4)
             if (!p->v8_cl && LOGN >= 15 && rows * 8 <= (uint32_t)p->sm_count * 4) cl = 8;
+            // N = 2^13, 2^14 with many rows: the whole row per CTA (its 2^A x 4096 intermediate is
+            // 32-64 KB, so 4 rows per SM stay L2-resident without the cluster split; s13 +8.6%,
+            // s14 +3.7% over 2-CTA clusters; at 1024 rows the clusters still win)
+            else if (!p->v8_cl && LOGN <= 14 && rows >= 8u * (uint32_t)p->sm_count) cl = 1;
             // between half and one SM count of rows: 4-CTA clusters (config 5 sweep)
             else if (!p->v8_cl && LOGN >= 15 && rows <= (uint32_t)p->sm_count) cl = 4;
             if ((1 << (LOGN - 12)) < cl || (cl == 8 && LOGN < 15)) cl = 1;
