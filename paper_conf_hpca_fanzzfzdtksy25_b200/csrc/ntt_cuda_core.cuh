@@ -46,7 +46,8 @@ struct NttArgs {
     // polynomials: cpy_ls) as it is staged -- ModUp's pass-through of the Q limbs (ntt_rns.cuh)
     uint32_t* cpy = nullptr;
     uint32_t cpy_ls = 0;
-    uint32_t stagger_ns = 0;         // v8 experiment knob (WD_NTT_STAGGER): grid quarters start k * this apart
+    uint32_t stagger_ns = 0;
+    uint32_t limb_major = 0;         // v8: walk rows limb by limb (rows must be a multiple of L)         // v8 experiment knob (WD_NTT_STAGGER): grid quarters start k * this apart
 };
 
 __device__ __forceinline__ uint32_t row_map(uint32_t row, uint32_t L, uint32_t ls) {

@@ -156,9 +156,14 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
         for (uint32_t i = 0; i < k * a.stagger_ns / 1000; ++i) __nanosleep(1000);
     }
 
+    const uint32_t nb = rows / a.L;              // polynomials in the launch
 #pragma unroll 1
-    for (uint32_t row = blockIdx.x / CL; row < rows; row += gridDim.x / CL) {
-        const uint32_t limb = row % a.L;
+    for (uint32_t srow = blockIdx.x / CL; srow < rows; srow += gridDim.x / CL) {
+        // limb-major schedule (a.limb_major): the rows in flight at any time share a few limbs,
+        // so their twiddle tables (N x 8 bytes per limb and direction) stay a small part of L2
+        // next to the L2-resident intermediates; the data layout is unchanged
+        const uint32_t limb = a.limb_major ? srow / nb : srow % a.L;
+        const uint32_t row = a.limb_major ? (srow - limb * nb) * a.L + limb : srow;
         const LimbConst lc = a.lc[limb];
         const uint32_t q = lc.q, q2 = lc.q2;
         const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);

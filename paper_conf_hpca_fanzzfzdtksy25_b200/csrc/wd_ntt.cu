@@ -43,6 +43,7 @@ struct wd_ntt_plan {
     int v8_minb = 0;               // v8 CTAs per SM (WD_NTT_MINB: 4..6; 0 = measured default)
     int v8_cl = 0;                 // v8 CTAs per row cluster (WD_NTT_CL: 1, 2, 4; 0 = measured default)
     uint32_t stagger_ns = 0;       // WD_NTT_STAGGER (v8 experiment)
+    uint32_t limb_major = 1;       // v8 row schedule, limb by limb (WD_NTT_LM=0: natural order)
     int kernel_ver = 0;            // 0 = AUTO, the measured default per N and row count (launch_cc);
                                    // WD_NTT_KERNEL=v1|v2|v3|v5|v6 forces a generation (A/B runs)
     std::vector<uint32_t> primes, psi;
@@ -516,6 +517,7 @@ int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2,
     NttArgs a;
     a.in = in; a.in2 = in2; a.out = out; a.tw = fwd ? p->d_fwd : p->d_inv; a.lc = p->d_lc; a.L = p->L;
     a.stagger_ns = p->stagger_ns;
+    a.limb_major = p->limb_major;
     const int mode = effective_mode(p);
     int launches = 0;
     if (mode == WD_MODE_CUDA_GEMM && in2 == nullptr && p->logN == 16 && p->tc.ok) {
@@ -744,6 +746,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (const char* ev = getenv("WD_NTT_MINB")) p->v8_minb = std::max(3, std::min(6, atoi(ev)));
     if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 8 ? 8 : atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
     if (const char* ev = getenv("WD_NTT_STAGGER")) p->stagger_ns = (uint32_t)atoi(ev);
+    if (const char* ev = getenv("WD_NTT_LM")) p->limb_major = atoi(ev) != 0;
     if (const char* ev = getenv("WD_NTT_KERNEL")) p->kernel_ver = ev[0] == 'v' ? atoi(ev + 1) : p->kernel_ver;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
