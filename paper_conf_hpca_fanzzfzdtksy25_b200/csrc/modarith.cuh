@@ -21,7 +21,20 @@ struct __align__(32) LimbConst {
     uint32_t ninv, ninv_sh;  // N^-1 mod q and its Shoup companion
     uint32_t wn, wn_sh;      // psi^-brv(1) * N^-1 (last inverse layer) + Shoup
     uint64_t mu;             // floor((2^64-1)/q): Barrett constant for a*b mod q (pointwise)
+    uint32_t qinv;           // q^-1 mod 2^32 (Montgomery product of the v8 pointwise inverse)
+    uint32_t ninv_r, ninv_r_sh;  // N^-1 * 2^32 mod q + Shoup: the last layer undoes 2^-32
+    uint32_t wn_r, wn_r_sh;      // wn * 2^32 mod q + Shoup
+    uint32_t pad_[3];
 };
+
+// a * b * 2^-32 mod q in (0, 2q) for a, b < q (Montgomery, R = 2^32): t = a*b < q^2 < q*2^32,
+// m = t * q^-1 mod 2^32, so t - m*q = 0 (mod 2^32) and (t - m*q) / 2^32 = hi(t) - hi(m*q) lies in
+// (-q, q); + q.  One IMAD.WIDE, one IMAD, one IMAD.HI, one IADD3 (Barrett's mul_mod: ~12 ops).
+__device__ __forceinline__ uint32_t mont_mul(uint32_t a, uint32_t b, const LimbConst& c) {
+    const uint64_t t = (uint64_t)a * b;
+    const uint32_t m = (uint32_t)t * c.qinv;
+    return (uint32_t)(t >> 32) - __umulhi(m, c.q) + c.q;
+}
 
 // a * b mod q for two variable residues (< 2^32 each, product < 2^62 for q < 2^30): Barrett
 __device__ __forceinline__ uint32_t mul_mod(uint32_t a, uint32_t b, const LimbConst& c) {

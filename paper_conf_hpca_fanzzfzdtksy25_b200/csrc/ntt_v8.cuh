@@ -165,6 +165,10 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
         const uint32_t limb = a.limb_major ? srow / nb : srow % a.L;
         const uint32_t row = a.limb_major ? (srow - limb * nb) * a.L + limb : srow;
         const LimbConst lc = a.lc[limb];
+        // the last inverse layer's constants: with the pointwise product (PW, Montgomery, which
+        // leaves a factor 2^-32) they carry an extra 2^32 (N^-1 * 2^32, wn * 2^32)
+        LimbConst lcl = lc;
+        if constexpr (PW) { lcl.ninv = lc.ninv_r; lcl.ninv_sh = lc.ninv_r_sh; lcl.wn = lc.wn_r; lcl.wn_sh = lc.wn_r_sh; }
         const uint32_t q = lc.q, q2 = lc.q2;
         const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
         const uint32_t* in = a.in + ((size_t)(EPI == 1 ? row / a.L : row_map(row, a.L, a.in_ls)) << LOGN);
@@ -356,8 +360,9 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     }
                 }
                 if constexpr (PW) {                      // row f1: pointwise product, coalesced
-                    // the warp's own 2 KB slice: in2 read 512 B per instruction, the product
-                    // written back to the same shared-memory slots before stage 3' reads them
+                    // the warp's own 2 KB slice: in2 read 512 B per instruction, the Montgomery
+                    // product a*b*2^-32 in (0, 2q) written back to the same shared-memory slots
+                    // before stage 3' reads them; the last layer's lcl constants restore 2^32
                     const int wbase = (t >> 5) * 512 + 4 * (t & 31);
 #pragma unroll
                     for (int v = 0; v < 4; ++v) {
@@ -365,8 +370,8 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                         uint4* sp = reinterpret_cast<uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
                         const uint4 u = *sp;
                         const uint4 m = __ldcs(reinterpret_cast<const uint4*>(in2 + s * V8_SUBW + e));
-                        *sp = make_uint4(mul_mod(u.x, m.x, lc), mul_mod(u.y, m.y, lc), mul_mod(u.z, m.z, lc),
-                                         mul_mod(u.w, m.w, lc));
+                        *sp = make_uint4(mont_mul(u.x, m.x, lc), mont_mul(u.y, m.y, lc), mont_mul(u.z, m.z, lc),
+                                         mont_mul(u.w, m.w, lc));
                     }
                     __syncwarp();
                 }
@@ -402,7 +407,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     const int b = hi4, c = lo4;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
-                    inv_radix<4, A == 0>(x, tw, A, (uint32_t)s, lc);
+                    inv_radix<4, A == 0>(x, tw, A, (uint32_t)s, lcl);
                     uint32_t* o = out + s * V8_SUBW + b * 16 + c;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) {
@@ -425,7 +430,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     };
                     auto cmp = [&](uint32_t (&v)[R], int pass) {
                         const int c = pass * V8_T + t;
-                        inv_radix<A, true>(v, tw, 0, 0, lc);
+                        inv_radix<A, true>(v, tw, 0, 0, lcl);
 #pragma unroll
                         for (int k = 0; k < R; ++k) __stcs(out + k * V8_SUBW + c, canon2(v[k], q));
                     };
@@ -444,7 +449,7 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
                     uint32_t x[R];
 #pragma unroll
                     for (int k = 0; k < R; ++k) x[k] = __ldcs(out + k * V8_SUBW + c);
-                    inv_radix<A, true>(x, tw, 0, 0, lc);
+                    inv_radix<A, true>(x, tw, 0, 0, lcl);
 #pragma unroll
                     for (int k = 0; k < R; ++k) __stcs(out + k * V8_SUBW + c, canon2(x[k], q));
                 }

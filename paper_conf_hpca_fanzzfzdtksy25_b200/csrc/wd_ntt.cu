@@ -736,6 +736,15 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
         c.ninv = pm_pow(N % q, q - 2, q); c.ninv_sh = pm_shoup(c.ninv, q);
         c.wn = pm_mul(N > 1 ? v[1].x : 1, c.ninv, q); c.wn_sh = pm_shoup(c.wn, q);
         c.mu = ~0ull / q;
+        {
+            uint32_t qi = q;                              // Newton: q * qi = 1 (mod 2^32)
+            for (int it = 0; it < 5; ++it) qi *= 2u - q * qi;
+            c.qinv = qi;
+            const uint32_t r = (uint32_t)((1ull << 32) % q);
+            c.ninv_r = pm_mul(c.ninv, r, q); c.ninv_r_sh = pm_shoup(c.ninv_r, q);
+            c.wn_r = pm_mul(c.wn, r, q); c.wn_r_sh = pm_shoup(c.wn_r, q);
+            c.pad_[0] = c.pad_[1] = c.pad_[2] = 0;
+        }
     }
 
     // ---- device upload (the only H2D copy of the plan's life)
