@@ -115,7 +115,7 @@ __device__ __forceinline__ void v8_store_sub(uint32_t* S, int aa, int b, const u
 // MINB: resident CTAs per SM the register budget is cut for (4 -> 64 registers; 5, 6 -> 48, 40
 // with per-layer just-in-time stage-3 twiddles instead of 15 preloaded pairs).
 // ONLY: 1 = phase 1 only, 2 = phase 2 only, 3..8 other timing experiments (results are wrong); 9 = v8
-// without the column-pass prefetch (correct; A/B runs).
+// with the column-pass prefetch PF (correct; A/B runs).
 // CL > 1: a cluster of CL CTAs shares each row -- CTA rank r takes column passes and sub-rows
 // [r, r+1) * (16|R)/CL, with ONE cluster barrier (release/acquire) between the phases.  Rows
 // in flight, hence the L2 footprint of the intermediate, shrink by CL.
@@ -143,9 +143,10 @@ __global__ void __launch_bounds__(V8_T, MINB) ntt_v8(NttArgs a, uint32_t rows) {
     static_assert(R % CL == 0 && (V8_SUBW / V8_T) % CL == 0, "cluster splits passes and sub-rows evenly");
     constexpr int NP = V8_SUBW / V8_T / CL;  // phase-1 column passes per CTA
     constexpr int NS = R / CL;               // phase-2 sub-rows per CTA
-    // PF: column passes pipelined two deep (needs 2 x 2^A data registers: A <= 4; ONLY = 9 turns
-    // it off for A/B runs)
-    constexpr bool PF = R <= 16 && NP % 2 == 0 && NP >= 2 && ONLY != 9;
+    // PF: column passes pipelined two deep (needs 2 x 2^A data registers: A <= 4).  Opt-in
+    // experiment (ONLY = 9, WD_NTT_KERNEL=v89): same-box A/B at config 3 puts it 1-2% BEHIND the
+    // plain passes (forward 1.050 vs 1.040 ms, inverse 1.073 vs 1.048 ms; the inverse spills)
+    constexpr bool PF = R <= 16 && NP % 2 == 0 && NP >= 2 && ONLY == 9;
     const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
     const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
     extern __shared__ __align__(16) uint32_t smem[];

@@ -300,7 +300,7 @@ void launch_cc(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, 
             if constexpr (LOGN >= 13) cudaLaunchKernelEx(&cfg, ntt_v8<LOGN, true, false, 8, 4, 2>, a, rows);
             return;
         }
-        if (p->kernel_ver == 89) {   // v8 (2-CTA cluster) without the column-pass prefetch
+        if (p->kernel_ver == 89) {   // v8 (2-CTA cluster) with the column-pass prefetch (PF)
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = dim3(p->sm_count * 4); cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM; cfg.stream = s;
             cudaLaunchAttribute at[1];
