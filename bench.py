@@ -510,6 +510,25 @@ def main():
         e2e = {"value": 2 * rows * args.e2e_steps * world / (float(te.item()) / 1e3) / 1e3, "unit": "KOPS",
                "h2d_bytes_per_step": bytes_step, "d2h_bytes_per_step": bytes_step,
                "steps": args.e2e_steps, "api": "wd_ntt_forward_host + wd_ntt_inverse_host (pinned host buffers)"}
+        # the PCIe bound: the same bytes as bare pinned copies, H2D and D2H on two streams at once
+        s_h, s_d = torch.cuda.Stream(), torch.cuda.Stream()
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        c0.record(stream)
+        s_h.wait_stream(stream); s_d.wait_stream(stream)
+        for _ in range(2):
+            with torch.cuda.stream(s_h):
+                work.copy_(hx, non_blocking=True)
+            with torch.cuda.stream(s_d):
+                hy.copy_(x, non_blocking=True)
+        stream.wait_stream(s_h); stream.wait_stream(s_d)
+        c1.record(stream)
+        torch.cuda.synchronize()
+        copy_ms = c0.elapsed_time(c1)            # 2 x batch bytes each way = one e2e step's copies
+        e2e["pcie_bound"] = {"value": 2 * rows / (copy_ms / 1e3) / 1e3, "unit": "KOPS",
+                             "copy_ms_per_step": copy_ms,
+                             "note": "bare pinned H2D || D2H of one step's bytes, no kernels"}
+        e2e["frac_of_pcie_bound"] = e2e["value"] / world / e2e["pcie_bound"]["value"]
         del hx, hy
 
     if rank != 0:

@@ -556,8 +556,12 @@ int run_host(const wd_ntt_plan* pc, bool fwd, const uint32_t* h_in, uint32_t* h_
     int dev = -1;
     if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) return set_err(WD_EINVAL);
     const size_t row_words = (size_t)p->L * p->N;
-    // ~8 chunks, each at least 1 polynomial: H2D(k+1) || kernel(k) || D2H(k-1)
-    const uint32_t nch = std::min<uint32_t>(batch, 8);
+    // chunks of >= 1 polynomial: H2D(k+1) || kernel(k) || D2H(k-1).  The first H2D and the
+    // last D2H are not overlapped, so a call costs ~(nch+1)/nch of one copy direction: 8 chunks
+    // for small jobs, up to 32 chunks of ~32 MB for large ones.
+    const size_t total_bytes = (size_t)batch * row_words * 4;
+    const uint32_t want = (uint32_t)std::min<size_t>(32, std::max<size_t>(8, total_bytes >> 25));
+    const uint32_t nch = std::min<uint32_t>(batch, want);
     cudaEventRecord(p->he[3], s);
     uint32_t total = 0;
     uint32_t b0 = 0;
