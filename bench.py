@@ -2,7 +2,7 @@
 """bench.py -- batched negacyclic RNS NTT/INTT throughput on B200 (BASELINE.json metric).
 
 Contract (task statement / DESIGN.md "Measurement"):
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl wd|reference] [--mode auto|cuda|tensor|fused]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl wd|reference] [--mode auto|cuda|tensor|fused|cuda_gemm|ftc]
 A STEP = one pass of the whole hot path over one batch: forward NTT of every
 (polynomial, limb) row, then the inverse NTT of the result (config 3 of
 BASELINE.json: N=2^16, L=36, 64 ciphertexts = 128 polynomials = 4608 rows per
@@ -349,8 +349,8 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="wd", choices=["wd", "reference"])
-    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused", "cuda_gemm"])
-    ap.add_argument("--share", type=float, default=-1.0, help="tensor share for --mode fused")
+    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused", "cuda_gemm", "ftc"])
+    ap.add_argument("--share", type=float, default=-1.0, help="tensor share for --mode fused / ftc")
     ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--graph", default="auto", choices=["auto", "on", "off"],

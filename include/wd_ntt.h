@@ -59,6 +59,11 @@ typedef struct CUstream_st* wd_stream_t;       /* == cudaStream_t */
 #define WD_MODE_FUSED    3   /* both paths concurrently on the same SMs (WD-FUSE role)  */
 #define WD_MODE_CUDA_GEMM 4  /* inner DFTs as 32-bit GEMMs on the CUDA cores (WD-CUDA,   *
                               * PAPER.md:322/401), N = 2^16 only     */
+#define WD_MODE_FTC      5   /* WD-FTC: the batch *
+                              * split at a polynomial boundary, WD-Tensor on a tensor_share *
+                              * of the polynomials and WD-CUDA on the rest, the two running *
+                              * concurrently on the same GPU (an internal forked stream,    *
+                              * joined back into the caller's stream), N = 2^16 only       */
 
 /*
  * wd_ntt_plan_create -- PAPER.md:358 (initialisation phase: moduli, twiddles
@@ -207,8 +212,9 @@ int      wd_ntt_check_prime(uint32_t q, uint32_t N);
 /* Select the execution path.  tensor_share in [0,1] is, in WD_MODE_FUSED,
  * the fraction of rows whose column phase runs on the tensor-core warps
  * while the CUDA-core warps run the row phase (the rest of the rows run
- * entirely on the CUDA-core warps).  Ignored otherwise; < 0
- * keeps the plan's measured default.  Returns WD_OK,
+ * entirely on the CUDA-core warps).  In WD_MODE_FTC it is the
+ * fraction of polynomials given to WD-Tensor (default 0.7, the best of 0.5 / 0.6 / 0.7
+ * measured at config 3).  Ignored otherwise; < 0 keeps the plan's default.  Returns WD_OK,
  * WD_EINVAL or WD_EUNSUPPORTED.  Not thread-safe against concurrent calls
  * using the same plan. */
 int wd_ntt_plan_set_mode(wd_ntt_plan* plan, int mode, float tensor_share);
@@ -218,8 +224,8 @@ int wd_ntt_plan_get_mode(const wd_ntt_plan* plan);
  * the units' measured throughput): times one forward + inverse over `batch` polynomials of
  * scratch data (allocated and freed inside the call, zero residues) for every execution path
  * available at this N -- WD_MODE_CUDA, and for N = 2^16 also WD_MODE_FUSED (phase-split
- * pipeline and row splits with tensor_share 0.25 / 0.5 / 0.75), WD_MODE_TENSOR and
- * WD_MODE_CUDA_GEMM -- with CUDA events on `stream`, and sets the plan to the fastest.
+ * pipeline and row splits with tensor_share 0.25 / 0.5 / 0.75), WD_MODE_TENSOR,
+ * WD_MODE_CUDA_GEMM and WD_MODE_FTC (at the plan's FTC share) -- with CUDA events on `stream`, and sets the plan to the fastest.
  * Writes that path's milliseconds per forward + inverse to *best_ms if best_ms != NULL.
  * Synchronises `stream`.  Returns WD_OK, WD_EINVAL (NULL plan, batch == 0, wrong device) or
  * WD_ECUDA (allocation or launch failure; the plan's mode is then unchanged).  Not

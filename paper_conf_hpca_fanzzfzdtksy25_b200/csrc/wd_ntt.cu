@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -58,6 +59,10 @@ struct wd_ntt_plan {
     float tensor_share = 0.5f;
     cudaStream_t hs[3] = {nullptr, nullptr, nullptr};   // host-path pipeline streams
     cudaEvent_t he[4] = {nullptr, nullptr, nullptr, nullptr};
+    float ftc_share = 0.7f;        // WD_MODE_FTC: polynomials on WD-Tensor (best of 0.5/0.6/0.7 at config 3)
+    cudaStream_t fs = nullptr;     // WD_MODE_FTC fork stream and its fork / join events
+    cudaEvent_t fe[2] = {nullptr, nullptr};
+    std::mutex ftc_mu;
     std::mutex host_mu;
 };
 
@@ -498,6 +503,23 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     return 1;
 }
 
+// WD-CUDA (row f2): the four radix-16 inner DFTs as 32-bit GEMMs on the CUDA cores, N = 2^16
+int launch_wdcuda(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
+    WdcArgs wa;
+    wa.a = a; wa.mat = p->tc.d_mat;
+    wa.t1 = fwd ? p->tc.d_tw1 : p->tc.d_sg1; wa.t2 = fwd ? p->tc.d_tw2 : p->tc.d_sg2; wa.t3 = fwd ? p->tc.d_tw3 : p->tc.d_sg3;
+    cudaLaunchConfig_t cfg = {};
+    cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM + 2048; cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
+    cfg.attrs = at; cfg.numAttrs = 1;
+    cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)(p->sm_count * 3 / 2)) * 2);
+    if (fwd) cudaLaunchKernelEx(&cfg, ntt_wdcuda16<true>, wa, rows);
+    else cudaLaunchKernelEx(&cfg, ntt_wdcuda16<false>, wa, rows);
+    return 1;
+}
+
 int effective_mode(const wd_ntt_plan* p) {
     if (p->mode != WD_MODE_AUTO) return p->mode;
     return WD_MODE_CUDA;
@@ -521,19 +543,30 @@ int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2,
     const int mode = effective_mode(p);
     int launches = 0;
     if (mode == WD_MODE_CUDA_GEMM && in2 == nullptr && p->logN == 16 && p->tc.ok) {
-        WdcArgs wa;
-        wa.a = a; wa.mat = p->tc.d_mat;
-        wa.t1 = fwd ? p->tc.d_tw1 : p->tc.d_sg1; wa.t2 = fwd ? p->tc.d_tw2 : p->tc.d_sg2; wa.t3 = fwd ? p->tc.d_tw3 : p->tc.d_sg3;
-        cudaLaunchConfig_t cfg = {};
-        cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM + 2048; cfg.stream = s;
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeClusterDimension;
-        at[0].val.clusterDim.x = 2; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
-        cfg.attrs = at; cfg.numAttrs = 1;
-        cfg.gridDim = dim3(std::min<uint32_t>(rows, (uint32_t)(p->sm_count * 3 / 2)) * 2);
-        if (fwd) cudaLaunchKernelEx(&cfg, ntt_wdcuda16<true>, wa, rows);
-        else cudaLaunchKernelEx(&cfg, ntt_wdcuda16<false>, wa, rows);
-        launches = 1;
+        launches = launch_wdcuda(p, fwd, a, rows, s);
+    } else if (mode == WD_MODE_FTC && in2 == nullptr && p->logN == 16 && p->tc.ok) {
+        // WD-FTC: split at a polynomial boundary (rows stay limb-aligned), WD-Tensor on the
+        // first bt polynomials in a forked stream, WD-CUDA on the rest in `s`, then join.
+        const uint32_t bt = std::min<uint32_t>(batch, (uint32_t)std::lround(p->ftc_share * batch));
+        NttArgs ac = a;
+        const size_t off = (size_t)bt * p->L * p->N;
+        ac.in = a.in + off; ac.out = a.out + off;
+        if (bt == 0) {
+            launches = launch_wdcuda(p, fwd, ac, rows, s);
+        } else if (bt == batch) {
+            launches = launch_tensor(p->logN, fwd, a, p->tc, rows, p->sm_count, s);
+        } else {
+            wd_ntt_plan* pm = const_cast<wd_ntt_plan*>(p);
+            std::lock_guard<std::mutex> lk(pm->ftc_mu);
+            cudaEventRecord(p->fe[0], s);
+            cudaStreamWaitEvent(p->fs, p->fe[0], 0);
+            const int n1 = launch_tensor(p->logN, fwd, a, p->tc, bt * p->L, p->sm_count, p->fs);
+            const int n2 = launch_wdcuda(p, fwd, ac, (batch - bt) * p->L, s);
+            cudaEventRecord(p->fe[1], p->fs);
+            cudaStreamWaitEvent(s, p->fe[1], 0);
+            launches = n1 + n2;
+        }
+        if (launches < 0) return set_err(WD_EUNSUPPORTED);
     } else if (mode == WD_MODE_CUDA || mode == WD_MODE_CUDA_GEMM || in2 != nullptr || !tensor_supported(p->logN)) {
         if (mode != WD_MODE_CUDA && in2 == nullptr && mode != WD_MODE_AUTO) return set_err(WD_EUNSUPPORTED);
         launches = launch_cuda_core(p, fwd, a, rows, s);
@@ -597,6 +630,8 @@ void free_plan(wd_ntt_plan* p) {
         free_tensor_tables(p->tc);
         for (auto& s : p->hs) if (s) cudaStreamDestroy(s);
         for (auto& e : p->he) if (e) cudaEventDestroy(e);
+        if (p->fs) cudaStreamDestroy(p->fs);
+        for (auto& e : p->fe) if (e) cudaEventDestroy(e);
         if (cur >= 0 && cur != p->device) cudaSetDevice(cur);
     }
     delete p;
@@ -793,6 +828,8 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     }
     for (auto& s : p->hs) if (cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->he) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
+    if (cudaStreamCreateWithFlags(&p->fs, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
+    for (auto& e : p->fe) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     if (prepare_kernels(p->logN) != WD_OK || prepare_tensor_kernels(p->logN) != WD_OK ||
         prepare_fused_kernels(p->logN) != WD_OK) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
@@ -1059,12 +1096,17 @@ int wd_ntt_check_prime(uint32_t q, uint32_t N) {
 }
 
 int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
-    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_CUDA_GEMM) return set_err(WD_EINVAL);
-    if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED || mode == WD_MODE_CUDA_GEMM) && !tensor_supported(p->logN))
+    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_FTC) return set_err(WD_EINVAL);
+    if ((mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED || mode == WD_MODE_CUDA_GEMM || mode == WD_MODE_FTC) &&
+        !tensor_supported(p->logN))
         return set_err(WD_EUNSUPPORTED);
+    if ((mode == WD_MODE_CUDA_GEMM || mode == WD_MODE_FTC) && p->logN != 16) return set_err(WD_EUNSUPPORTED);
     if (tensor_share > 1.0f) return set_err(WD_EINVAL);
     p->mode = mode;
-    if (tensor_share >= 0.0f) p->tensor_share = tensor_share;
+    if (tensor_share >= 0.0f) {
+        if (mode == WD_MODE_FTC) p->ftc_share = tensor_share;
+        else p->tensor_share = tensor_share;
+    }
     return set_err(WD_OK);
 }
 int wd_ntt_plan_get_mode(const wd_ntt_plan* p) { return p ? effective_mode(p) : -1; }
@@ -1095,7 +1137,10 @@ int wd_ntt_plan_autotune(wd_ntt_plan* p, uint32_t batch, wd_stream_t st, float* 
         cands.push_back({WD_MODE_FUSED, default_tensor_share(p->logN)});
         for (float sh : {0.25f, 0.5f, 0.75f}) cands.push_back({WD_MODE_FUSED, sh});
         cands.push_back({WD_MODE_TENSOR, p->tensor_share});
-        if (p->logN == 16) cands.push_back({WD_MODE_CUDA_GEMM, p->tensor_share});
+        if (p->logN == 16) {
+            cands.push_back({WD_MODE_CUDA_GEMM, p->tensor_share});
+            cands.push_back({WD_MODE_FTC, p->tensor_share});     // split by the plan's ftc_share
+        }
     }
     const int mode0 = p->mode;
     const float share0 = p->tensor_share;

@@ -201,7 +201,8 @@ def _modes(wd):
     return ["cuda", "tensor", "fused"]
 
 
-MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.0), ("fused", 0.6)]
+MODES = [("cuda", -1.0), ("tensor", -1.0), ("fused", -1.0), ("fused", 0.0), ("fused", 0.6),
+         ("ftc", -1.0), ("ftc", 0.0), ("ftc", 0.5), ("ftc", 1.0)]
 
 
 @pytest.mark.parametrize("mode,share", MODES)
@@ -327,6 +328,26 @@ def test_wd_cuda_gemm_mode(wd):
         wd.Plan(1 << 15, P[:2], mode="cuda_gemm")          # N = 2^16 only
 
 
+# -------------------------------------------------------------- WD-FTC (row f2): WD-Tensor || WD-CUDA
+@pytest.mark.parametrize("batch,share", [(1, 0.6), (2, 0.5), (7, 0.6), (5, 0.2)])
+def test_wd_ftc_mode(wd, batch, share):
+    n = 1 << 16
+    primes = [P[0], P[33], 786433, 269221889]
+    x = inputs.uniform_residues(primes, n, batch, 5400 + batch)
+    plan = wd.Plan(n, primes)
+    plan.set_mode("ftc", share)
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (batch, share)
+    assert np.array_equal(gpu_inv(wd, plan, y), x)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes))
+    d = to_dev(x)                                       # in place across the split
+    plan.forward(d, d)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(d), y)
+    with pytest.raises(wd.WdNttError):
+        wd.Plan(1 << 15, P[:2], mode="ftc")                # N = 2^16 only
+
+
 # v11: every tensor / butterfly split of the row phase (bit st-1 of WD_NTT_TMASK = stage st on the
 # tensor cores), over more rows than resident CTAs
 @pytest.mark.parametrize("tmask", ["1", "3", "6", "7"])
@@ -352,7 +373,7 @@ def test_autotune_picks_a_path_and_stays_exact(wd, logn, batch):
     mode, ms = plan.autotune(batch)
     assert ms > 0
     if logn == 16:
-        assert mode in (1, 2, 3, 4)
+        assert mode in (1, 2, 3, 4, 5)
     else:
         assert mode == 1                                   # only the CUDA-core path below 2^16
     x = inputs.uniform_residues(primes, n, batch, 6100 + logn)
