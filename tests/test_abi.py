@@ -83,3 +83,19 @@ def test_check_prime_matches_oracle():
             continue
         expect = oracle.is_prime(q)
         assert (wdntt.wd_ntt_check_prime(q, 4096) == 0) == expect, q
+
+
+def test_binding_constants_match_header():
+    """The Python binding's error and mode codes are the header's #defines (one source of truth)."""
+    import os
+    import re
+    hdr = open(os.path.join(os.path.dirname(__file__), "..", "include", "wd_ntt.h")).read()
+    defs = {m.group(1): int(m.group(2)) for m in re.finditer(r"#define\s+(WD_[A-Z_]+)\s+(\d+)", hdr)}
+    modes = {k: v for k, v in defs.items() if k.startswith("WD_MODE_")}
+    assert len(modes) == 6 and modes["WD_MODE_FTC"] == 5
+    for name, val in defs.items():
+        if hasattr(wdntt, name):
+            assert getattr(wdntt, name) == val, name
+    for name in modes:
+        assert getattr(wdntt, name) == modes[name], name
+    assert sorted(wdntt.MODES.values()) == sorted(modes.values())
