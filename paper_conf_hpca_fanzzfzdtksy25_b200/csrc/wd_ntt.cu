@@ -62,7 +62,7 @@ struct wd_ntt_plan {
     float ftc_share = 0.7f;        // WD_MODE_FTC: polynomials on WD-Tensor (best of 0.5/0.6/0.7 at config 3)
     cudaStream_t fs = nullptr;     // WD_MODE_FTC fork stream and its fork / join events
     cudaEvent_t fe[2] = {nullptr, nullptr};
-    std::mutex ftc_mu;
+    mutable std::mutex ftc_mu;     // orders fork/join event use across host threads
     std::mutex host_mu;
 };
 
@@ -556,8 +556,7 @@ int run(const wd_ntt_plan* p, bool fwd, const uint32_t* in, const uint32_t* in2,
         } else if (bt == batch) {
             launches = launch_tensor(p->logN, fwd, a, p->tc, rows, p->sm_count, s);
         } else {
-            wd_ntt_plan* pm = const_cast<wd_ntt_plan*>(p);
-            std::lock_guard<std::mutex> lk(pm->ftc_mu);
+            std::lock_guard<std::mutex> lk(p->ftc_mu);
             cudaEventRecord(p->fe[0], s);
             cudaStreamWaitEvent(p->fs, p->fe[0], 0);
             const int n1 = launch_tensor(p->logN, fwd, a, p->tc, bt * p->L, p->sm_count, p->fs);

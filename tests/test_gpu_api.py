@@ -2,10 +2,11 @@
 
 * the host-buffer calls wd_ntt_forward_host / wd_ntt_inverse_host (the e2e path bench.py
   times): chunked H2D || kernel || D2H pipeline over 3 streams, batch sizes below, at and
-  above its 8 chunks, ragged chunk splits, in place on the host;
+  above its minimum of 8 chunks, ragged chunk splits, in place on the host;
 * reentrancy across streams (SURVEY.md 8.b "Execution": one plan used from several streams
   at once);
-* the contract for non-canonical inputs (8.b "Errors": result unspecified, no fault).
+* the contract for non-canonical inputs (8.b "Errors": result unspecified, no fault);
+* WD_MODE_FTC (its internal fork stream) under calls from several streams at once.
 """
 import numpy as np
 import pytest
@@ -121,3 +122,25 @@ def test_noncanonical_inputs_do_not_fault(wd, logn):
     plan.forward(d, y)
     torch.cuda.synchronize()
     assert np.array_equal(y.cpu().numpy().view(np.uint32), oracle.ntt_forward(x, primes))
+
+
+def test_ftc_mode_many_streams(wd):
+    """WD_MODE_FTC forks its tensor share onto the plan's own stream and joins it back: calls from
+    several caller streams at once must stay exact (the fork stream is shared by all of them)."""
+    n, primes, batch, ns = 1 << 16, P[:3], 3, 3
+    plan = wd.Plan(n, primes, mode="ftc")
+    xs = [inputs.uniform_residues(primes, n, batch, 500 + k) for k in range(ns)]
+    streams = [torch.cuda.Stream() for _ in range(ns)]
+    ds = [torch.from_numpy(x.view(np.int32)).cuda() for x in xs]
+    fs = [torch.empty_like(d) for d in ds]
+    rs = [torch.empty_like(d) for d in ds]
+    torch.cuda.synchronize()
+    for _ in range(2):
+        for st, d, f, r in zip(streams, ds, fs, rs):
+            with torch.cuda.stream(st):
+                plan.forward(d, f, stream=st.cuda_stream)
+                plan.inverse(f, r, stream=st.cuda_stream)
+    torch.cuda.synchronize()
+    for x, f, r in zip(xs, fs, rs):
+        assert np.array_equal(f.cpu().numpy().view(np.uint32), oracle.ntt_forward(x, primes))
+        assert np.array_equal(r.cpu().numpy().view(np.uint32), x)
