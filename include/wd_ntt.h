@@ -72,10 +72,12 @@ typedef struct CUstream_st* wd_stream_t;       /* == cudaStream_t */
  *   primes  host array of L moduli; each must be prime, < 2^30 and = 1 mod 2N
  *           (read during the call only; the caller keeps ownership)
  *   L       number of RNS limbs, 1 <= L <= 4096
- * Returns a plan owning its device tables (about 16*N*L bytes: forward and
- * inverse psi-power tables in bit-reversed order with Shoup companions, plus
- * the tensor-path inner-DFT byte planes), or NULL with wd_ntt_last_error() set
- * to WD_EINVAL / WD_EPRIME / WD_EUNSUPPORTED / WD_ECUDA / WD_ENOMEM.
+ * Returns a plan owning its device tables (16*N*L bytes: forward and inverse
+ * psi-power tables in bit-reversed order with Shoup companions; the round-1
+ * tensor modes TENSOR / FUSED / CUDA_GEMM / FTC add about 8*N*L more, built on
+ * their first wd_ntt_plan_set_mode / wd_ntt_plan_autotune), or NULL with
+ * wd_ntt_last_error() set to WD_EINVAL / WD_EPRIME / WD_EUNSUPPORTED / WD_ECUDA /
+ * WD_ENOMEM (host or device allocation failure: never an exception).
  * Argument validation happens before any CUDA call, so the WD_EINVAL /
  * WD_EPRIME / WD_EUNSUPPORTED paths work on a machine without a GPU.
  */
@@ -228,17 +230,14 @@ int wd_ntt_plan_get_mode(const wd_ntt_plan* plan);
  * WD_MODE_CUDA_GEMM and WD_MODE_FTC (at the plan's FTC share) -- with CUDA events on `stream`, and sets the plan to the fastest.
  * Writes that path's milliseconds per forward + inverse to *best_ms if best_ms != NULL.
  * Synchronises `stream`.  Returns WD_OK, WD_EINVAL (NULL plan, batch == 0, wrong device) or
- * WD_ECUDA (allocation or launch failure; the plan's mode is then unchanged).  Not
- * thread-safe against concurrent calls using the same plan. */
+ * WD_ECUDA (allocation or launch failure; the plan's mode is then unchanged).  The candidates
+ * are timed with an explicit mode each; the plan's mode is written once, at the end, so other
+ * streams launching with this plan meanwhile run in the old mode or the new one.  Two concurrent
+ * autotune / set_mode calls on one plan are not supported. */
 int wd_ntt_plan_autotune(wd_ntt_plan* plan, uint32_t batch, wd_stream_t stream, float* best_ms);
 
 /* Kernel launches issued by the last forward/inverse call on this thread. */
 uint32_t wd_ntt_last_launches(void);
-
-/* Resident CTAs per SM the driver reports for the plan's main kernel in `mode`
- * (WD_MODE_CUDA: N = 2^16, 2^17; WD_MODE_TENSOR: N = 2^16), fwd != 0 for the forward kernel;
- * a negative value is -(cudaError_t).  Diagnostic only. */
-int wd_ntt_occupancy(const wd_ntt_plan* plan, int mode, int fwd);
 
 int         wd_ntt_last_error(void);
 const char* wd_ntt_strerror(int code);

@@ -1,0 +1,51 @@
+// launch.h -- internal host interface between the C ABI (wd_ntt.cu) and the kernel translation units.
+// Every function here only configures and enqueues kernels on the given stream: no allocation, no
+// synchronisation, no environment reads (those happen once, at plan creation).
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+#include "common.cuh"
+#include "tensor_tables.h"
+
+namespace wd {
+
+// ---- k_cc.cu: v1 (one CTA per row, N = 2^12..2^17), ntt_small (N < 2^12), v5 (row over a cluster,
+//      N = 2^14..2^17)
+int prep_cc(uint32_t logN);
+void launch_v1(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s);
+void launch_v5(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s);
+
+// ---- k_v8.cu: v8 (N = 2^12..2^17) and WD-CUDA (N = 2^16)
+struct V8Occ { int ncl[4] = {0, 0, 0, 0}; };   // resident clusters per GPU for CL = 1, 2, 4, 8
+int prep_v8(uint32_t logN, int sm_count, V8Occ* occ);
+// cl in {1, 2, 4, 8}; epi: 0 plain, 1 RESCALE store map, 2 ModDown store map (forward only)
+void launch_v8(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ,
+               cudaStream_t s);
+int prep_wdcuda();
+void launch_wdcuda(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, cudaStream_t s);
+
+// ---- k_tensor.cu: the round-1 tensor path (TENSOR, FUSED modes; N = 2^16)
+int prep_tensor();
+int launch_tensor(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, cudaStream_t s);
+int launch_fused(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, float share,
+                 cudaStream_t s);
+
+// ---- k_rns.cu: RESCALE gather, fast basis conversion, 64-bit share reduction
+struct BconvTab {
+    const uint4* src;       // [S] {q_i, (Q/q_i)^-1 mod q_i, Shoup, 0}
+    const uint2* w;         // [S][D] {(Q/q_i) mod p_j, its Shoup companion mod p_j}
+    const uint4* dst;       // [D] {p_j, mu_lo, mu_hi, 0}: mu = floor((2^64 - 1) / p_j)
+    uint32_t S, D;
+};
+constexpr int BC_MAX = 64;                // max source / target limbs of a conversion
+int prep_rns();
+void launch_rs_gather(const uint32_t* in, uint32_t* work, uint32_t N, uint32_t L, uint32_t batch, int sm_count,
+                      cudaStream_t s);
+void launch_bconv(const uint32_t* x, uint32_t x_ls, uint32_t* y, uint32_t y_ls, uint32_t y_off, const BconvTab& t,
+                  uint32_t N, uint32_t batch, int sm_count, cudaStream_t s);
+void launch_bconv_partial(const uint32_t* x, uint32_t x_ls, uint64_t* y64, const BconvTab& t, uint32_t N,
+                          uint32_t batch, int sm_count, cudaStream_t s);
+void launch_reduce64(const uint64_t* sum, uint32_t* out, const uint4* dst, uint32_t D, uint32_t N, uint32_t rows,
+                     int sm_count, cudaStream_t s);
+
+}  // namespace wd

@@ -20,9 +20,65 @@
 #include <cstdint>
 #include "modarith.cuh"
 #include "ntt_cuda_core.cuh"
-#include "ntt_smem.cuh"
+#include "common.cuh"
 
 namespace wd {
+
+// 5 forward layers on 32 registers, twiddles of layer ls+t group (hi<<t)+g, fetched
+// just in time as 16-byte pairs (keeps the 1024-thread CTA within 64 registers)
+__device__ __forceinline__ void fwd32(uint32_t* x, const uint2* __restrict__ tw, int ls, uint32_t hi,
+                                      uint32_t q, uint32_t q2) {
+    {
+        const uint2 w = __ldg(tw + (1u << ls) + hi);
+#pragma unroll
+        for (int r = 0; r < 16; ++r) ct_bfly(x[r], x[r + 16], w, q, q2);
+    }
+#pragma unroll
+    for (int t = 1; t < 5; ++t) {
+        const int h = 16 >> t;
+        const uint4* p = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
+#pragma unroll
+        for (int g2 = 0; g2 < (1 << t); g2 += 2) {
+            const uint4 v = __ldg(p + g2 / 2);
+            const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
+#pragma unroll
+            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g2 * h + r], x[2 * g2 * h + r + h], wa, q, q2);
+#pragma unroll
+            for (int r = 0; r < h; ++r) ct_bfly(x[2 * (g2 + 1) * h + r], x[2 * (g2 + 1) * h + r + h], wb, q, q2);
+        }
+    }
+}
+template <bool LAST>
+__device__ __forceinline__ void inv32(uint32_t* x, const uint2* __restrict__ tw, int ls, uint32_t hi,
+                                      const LimbConst& c) {
+#pragma unroll
+    for (int t = 4; t >= 1; --t) {
+        const int h = 16 >> t;
+        const uint4* p = reinterpret_cast<const uint4*>(tw + (1u << (ls + t)) + (hi << t));
+#pragma unroll
+        for (int g2 = 0; g2 < (1 << t); g2 += 2) {
+            const uint4 v = __ldg(p + g2 / 2);
+            const uint2 wa = make_uint2(v.x, v.y), wb = make_uint2(v.z, v.w);
+#pragma unroll
+            for (int r = 0; r < h; ++r) gs_bfly(x[2 * g2 * h + r], x[2 * g2 * h + r + h], wa, c.q, c.q2);
+#pragma unroll
+            for (int r = 0; r < h; ++r) gs_bfly(x[2 * (g2 + 1) * h + r], x[2 * (g2 + 1) * h + r + h], wb, c.q, c.q2);
+        }
+    }
+    if (LAST) {
+#pragma unroll
+        for (int r = 0; r < 16; ++r) gs_bfly_last(x[r], x[r + 16], c);
+    } else {
+        const uint2 w = __ldg(tw + (1u << ls) + hi);
+#pragma unroll
+        for (int r = 0; r < 16; ++r) gs_bfly(x[r], x[r + 16], w, c.q, c.q2);
+    }
+}
+
+__device__ __forceinline__ void cpa16(void* smem_dst, const void* gsrc) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"((uint32_t)__cvta_generic_to_shared(smem_dst)), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void prefetch_wait() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
 constexpr int CL_T = 512;                        // threads per CTA
 constexpr int CL_WORDS = 1 << 14;                // words per CTA

@@ -22,37 +22,9 @@
 #pragma once
 #include <cstdint>
 #include "modarith.cuh"
+#include "common.cuh"
 
 namespace wd {
-
-struct NttArgs {
-    const uint32_t* in;
-    const uint32_t* in2;      // inverse only: if set, transform in o in2 (pointwise product, row f1)
-    uint32_t* out;
-    const uint2* tw;          // [L][N] (psi^+-brv(i), Shoup) for this direction
-    const LimbConst* lc;      // [L]
-    uint32_t L;
-    // RESCALE epilogue of the forward (ntt_v8<..., EPI = 1>): the phase-1
-    // input row of row r is in + (r / L) * N (the last limb's coefficients c of polynomial r / L,
-    // shared by its L output limbs), the output is (aux_i - NTT(c')) * q_last^-1 (ntt_rns.cuh)
-    const uint32_t* aux = nullptr;   // the rescale input [batch][Lfull][N]
-    const uint4* rs = nullptr;       // [L] {-q_last mod q_i, Shoup(1), q_last^-1 mod q_i, Shoup}
-    uint32_t rs_thr = 0;             // q_last - floor(q_last / 2)
-    uint32_t Lfull = 0;
-    // v8 only: rows between consecutive polynomials in `in` / `out` (0 = L, contiguous); lets a
-    // launch cover a limb SECTION of a wider [batch][Lfull][N] tensor (ModUp / ModDown, ntt_rns.cuh)
-    uint32_t in_ls = 0, out_ls = 0;
-    // v8 inverse only: if set, every input row is also copied unchanged to cpy (rows between
-    // polynomials: cpy_ls) as it is staged -- ModUp's pass-through of the Q limbs (ntt_rns.cuh)
-    uint32_t* cpy = nullptr;
-    uint32_t cpy_ls = 0;
-    uint32_t stagger_ns = 0;
-    uint32_t limb_major = 0;         // v8: walk rows limb by limb (rows must be a multiple of L)         // v8 experiment knob (WD_NTT_STAGGER): grid quarters start k * this apart
-};
-
-__device__ __forceinline__ uint32_t row_map(uint32_t row, uint32_t L, uint32_t ls) {
-    return ls ? (row / L) * ls + row % L : row;
-}
 
 constexpr int RS = 272;       // padded row stride (words) of 256-wide rows in SMEM
 

@@ -16,16 +16,15 @@
 // tensor_share is given (0..1), rows are instead assigned statically:
 // row index i of the CTA goes to the tensor group iff frac(i*share) < share.
 #pragma once
-#include <cstdlib>
-#include <cstring>
+#include <algorithm>
 #include "ntt_tensor.cuh"
+#include "ntt_persist.cuh"
 
 namespace wd {
 
-constexpr int FU_CC = 512, FU_TC = 128, FU_T = FU_CC + FU_TC;
+constexpr int FU_CC = 512;
 constexpr int FUP_TC = 256, FUP_T = FU_CC + FUP_TC;      // phase-split pipeline: 8 tensor warps
 constexpr int FU_CC_BAR = 2;
-constexpr int FU_SMEM = PGeo<16>::SMEM_BYTES + TC_SMEM + 64;
 constexpr int FUP_SMEM = PGeo<16>::SMEM_BYTES + TCC_SMEM + 64;
 
 template <int BAR, int NT>
@@ -81,82 +80,6 @@ __device__ __forceinline__ void cc_row(const NttArgs& a, uint32_t* smem, uint32_
     }
 }
 
-template <bool FWD, bool PW>
-__global__ void __launch_bounds__(FU_T, 1) ntt_fused16(TcArgs ta, uint32_t rows, float share) {
-    extern __shared__ __align__(1024) uint8_t fsm[];
-    uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
-    uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
-    int* ctl = reinterpret_cast<int*>(tcb + TC_SMEM);           // [0] counter, [1] cc slot, [2] tc slot
-    TcShared sh;
-    sh.Ain = tcb;
-    sh.Amid = tcb + 4 * TC_TILE;
-    sh.B = tcb + 8 * TC_TILE;
-    sh.bar = reinterpret_cast<uint64_t*>(tcb + 8 * TC_TILE + 8192);
-    sh.tslot = reinterpret_cast<uint32_t*>(sh.bar + 2);
-    const int tid = threadIdx.x;
-    if (tid == 0) {
-        ctl[0] = 0;
-        mbar_init(&sh.bar[0], 1);
-        mbar_init(&sh.bar[1], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    if (tid >= FU_CC && tid < FU_CC + 32) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" :: "r"(smem_addr(sh.tslot)));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
-    tc_fence_before();
-    __syncthreads();
-    tc_fence_after();
-    const uint32_t nmine = rows > blockIdx.x ? (rows - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-    const bool is_tc = tid >= FU_CC;
-    const int gtid = is_tc ? tid - FU_CC : tid;
-    // static split helper: does CTA-local row index i belong to the tensor group?
-    auto tc_owns = [&](uint32_t i) { return floorf((float)(i + 1) * share) > floorf((float)i * share); };
-    uint32_t sidx = 0;                                           // static-mode cursor
-    if (is_tc) {
-        const uint32_t tmem = *sh.tslot;
-        uint32_t ph[2] = {0, 0};
-        for (;;) {
-            uint32_t i;
-            if (share >= 0.0f) {
-                while (sidx < nmine && !tc_owns(sidx)) ++sidx;
-                i = sidx++;
-            } else {
-                if (gtid == 0) ctl[2] = atomicAdd(&ctl[0], 1);
-                named_bar(TC_BAR_ID, FU_TC);
-                i = (uint32_t)ctl[2];
-                named_bar(TC_BAR_ID, FU_TC);
-            }
-            if (i >= nmine) break;
-            tc_transform<FWD>(ta, sh, tmem, ph, blockIdx.x + i * gridDim.x);
-        }
-        tc_fence_before();
-        named_bar(TC_BAR_ID, FU_TC);
-        if (gtid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
-    } else {
-        for (;;) {
-            uint32_t i;
-            if (share >= 0.0f) {
-                while (sidx < nmine && tc_owns(sidx)) ++sidx;
-                i = sidx++;
-            } else {
-                if (gtid == 0) ctl[1] = atomicAdd(&ctl[0], 1);
-                named_bar(FU_CC_BAR, FU_CC);
-                i = (uint32_t)ctl[1];
-                named_bar(FU_CC_BAR, FU_CC);
-            }
-            if (i >= nmine) break;
-            cc_row<FWD, PW, FU_CC_BAR>(ta.a, ccbuf, blockIdx.x + i * gridDim.x);
-        }
-    }
-}
-
-// ---- phase-split pipeline: the tensor warps run the COLUMN phase (phase 1) of each row, the
-// CUDA-core warps run the ROW phase (phase 2); the two groups walk the CTA's row list in
-// step, handing each row over through its L2-resident output slot and a shared-memory
-// counter.  Forward: tensor leads (P1 of row i+1 overlaps P2 of row i).  Inverse: the
-// CUDA-core group leads (P2' first), the tensor group finishes each row with P1'.
-// The leader stays at most FU_LEAD rows ahead, bounding the in-flight intermediates.
 constexpr int FU_LEAD = 2;
 // measured default tensor share of the pipeline (scripts/gpu_sweep.sh)
 constexpr float FUSED_DEFAULT_SHARE = 1.0f;
@@ -193,12 +116,11 @@ __device__ __forceinline__ void cc_row_phase2(const NttArgs& a, uint32_t* smem, 
 }
 
 template <bool FWD>
-// solo: 0 normal; 1 / 2 = DIAGNOSTIC ONLY (WD_NTT_PIPE_SOLO): only the tensor / CUDA-core group
-// computes, the other just passes rows on -- results are wrong, the time is one side's throughput.
 // share: fraction of rows whose column phase runs on the tensor warps (interleaved); the
 // CUDA-core warps run the remaining rows whole (the paper's tensor/CUDA ratio knob).
 __global__ void __launch_bounds__(FUP_T, 1) ntt_fused16_pipe(TcArgs ta, const uint8_t* G, uint32_t rows, uint32_t per_cta,
-                                                             int solo, float share, int lead) {
+                                                             float share) {
+    constexpr int lead = FU_LEAD;
     extern __shared__ __align__(1024) uint8_t fsm[];
     uint32_t* ccbuf = reinterpret_cast<uint32_t*>(fsm);
     uint8_t* tcb = fsm + PGeo<16>::SMEM_BYTES;
@@ -246,10 +168,10 @@ __global__ void __launch_bounds__(FUP_T, 1) ntt_fused16_pipe(TcArgs ta, const ui
         const uint32_t limb = k / Bp, row = (k % Bp) * L + limb;
         const bool tc_row = floorf((float)(i + 1) * share) > floorf((float)i * share);
         if (is_tc) {
-            if (solo != 2 && tc_row)
+            if (tc_row)
                 tcc_columns<FWD, false, FUP_TC>(ta, sh, tmem, ph, row, G + ((size_t)limb * 2 + (FWD ? 0 : 1)) * 17 * 4096,
                                                 loaded, TC_BAR_ID);
-        } else if (solo != 1) {
+        } else {
             if (tc_row) cc_row_phase2<FWD, FU_CC_BAR>(ta.a, ccbuf, row);
             else cc_row<FWD, false, FU_CC_BAR>(ta.a, ccbuf, row);
         }
@@ -270,13 +192,11 @@ inline int prepare_fused_kernels(uint32_t logN) {
         if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, FUP_SMEM) != cudaSuccess ||
             cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
             return 4;
-    for (auto k : {ntt_fused16<true, false>, ntt_fused16<false, false>})
-        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, FU_SMEM) != cudaSuccess ||
-            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
-            return 4;
     return 0;
 }
 
+// FUSED: one persistent CTA per SM; rows split evenly over the CTAs (limb-major), the share of
+// rows whose column phase goes to the tensor warps is `share` (< 0: FUSED_DEFAULT_SHARE)
 inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows,
                         int sm_count, float share, cudaStream_t s) {
     if (logN != 16 || !tc.ok || a.in2) return -1;
@@ -288,18 +208,10 @@ inline int launch_fused(uint32_t logN, bool fwd, const NttArgs& a, const TensorT
     ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
     ta.c16 = tc.d_c16;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
-    static const char* variant = getenv("WD_NTT_FUSED");          // "rows": whole-row split kernel (A/B runs)
-    if (!(variant && strcmp(variant, "rows") == 0)) {              // phase-split pipeline (default)
-        const uint32_t per = (rows + grid - 1) / grid;
-        static const int solo = getenv("WD_NTT_PIPE_SOLO") ? atoi(getenv("WD_NTT_PIPE_SOLO")) : 0;
-        static const int lead = getenv("WD_NTT_PIPE_LEAD") ? std::max(1, atoi(getenv("WD_NTT_PIPE_LEAD"))) : FU_LEAD;
-        const float sh = share < 0.0f ? FUSED_DEFAULT_SHARE : share;
-        if (fwd) ntt_fused16_pipe<true><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per, solo, sh, lead);
-        else ntt_fused16_pipe<false><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per, solo, sh, lead);
-        return 1;
-    }
-    if (fwd) ntt_fused16<true, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);
-    else ntt_fused16<false, false><<<grid, FU_T, FU_SMEM, s>>>(ta, rows, share);
+    const uint32_t per = (rows + grid - 1) / grid;
+    const float sh = share < 0.0f ? FUSED_DEFAULT_SHARE : share;
+    if (fwd) ntt_fused16_pipe<true><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per, sh);
+    else ntt_fused16_pipe<false><<<grid, FUP_T, FUP_SMEM, s>>>(ta, tc.d_G, rows, per, sh);
     return 1;
 }
 

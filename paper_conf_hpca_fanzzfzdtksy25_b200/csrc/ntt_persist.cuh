@@ -1,5 +1,6 @@
-// ntt_persist.cuh -- persistent, cp.async-pipelined CUDA-core NTT/INTT for N = 2^15..2^17
-// (the large-N "dual kernel" case of PAPER.md:366).
+// ntt_persist.cuh -- cp.async-pipelined CUDA-core chunk workers for N = 2^15..2^17, used by the
+// CUDA-core warps of the FUSED pipeline (ntt_fused.cuh).  (Round 1 also
+// built a persistent kernel on them, v2/v6; it was superseded by v8 and removed.)
 //
 // One CTA per SM loops over its share of the batch*L rows (PE-kernel idea,
 // PAPER.md:334-352).  A row is N = N1 x 256: phase 1 = the first log2(N1)
@@ -18,14 +19,6 @@
 #include "ntt_cuda_core.cuh"
 
 namespace wd {
-
-__device__ __forceinline__ void cp_async16(void* smem_dst, const void* gsrc) {
-    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(d), "l"(gsrc) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
 
 // barrier among the 512 CUDA-core threads: __syncthreads when they are the whole CTA,
 // a named barrier when they share the CTA with the tensor group (ntt_fused.cuh)
@@ -121,45 +114,6 @@ __device__ __forceinline__ void fwd_p1_chunk(uint32_t* S, uint32_t* out, int c0,
         fwd_radix<G::A1>(x, tw, G::A0, i1, q, q2);
 #pragma unroll
         for (int r = 0; r < G::R1; ++r) out[((i1 << G::A1) + r) * 256 + c] = x[r];
-    }
-}
-
-// stage-3 twiddles of one 16-point block: Psi[4096+g], Psi[8192+2g..], Psi[16384+4g..], Psi[32768+8g..]
-// (generic: layer ls..ls+3 with group hi) fetched as 16-byte vectors.
-__device__ __forceinline__ void load_tw16(uint2* w, const uint2* __restrict__ tw, int ls, uint32_t hi) {
-    w[0] = __ldg(tw + (1u << ls) + hi);
-    const uint4 a = __ldg(reinterpret_cast<const uint4*>(tw + (2u << ls) + 2 * hi));
-    w[1] = make_uint2(a.x, a.y); w[2] = make_uint2(a.z, a.w);
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-        const uint4 b = __ldg(reinterpret_cast<const uint4*>(tw + (4u << ls) + 4 * hi) + k);
-        w[3 + 2 * k] = make_uint2(b.x, b.y); w[4 + 2 * k] = make_uint2(b.z, b.w);
-    }
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-        const uint4 b = __ldg(reinterpret_cast<const uint4*>(tw + (8u << ls) + 8 * hi) + k);
-        w[7 + 2 * k] = make_uint2(b.x, b.y); w[8 + 2 * k] = make_uint2(b.z, b.w);
-    }
-}
-// radix-16 forward block with explicit twiddles w[0..14] (layer t group g -> w[(1<<t)-1+g])
-__device__ __forceinline__ void fwd16_tw(uint32_t* x, const uint2* w, uint32_t q, uint32_t q2) {
-#pragma unroll
-    for (int t = 0; t < 4; ++t) {
-        const int h = 8 >> t;
-#pragma unroll
-        for (int g = 0; g < (1 << t); ++g)
-#pragma unroll
-            for (int r = 0; r < h; ++r) ct_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w[(1 << t) - 1 + g], q, q2);
-    }
-}
-__device__ __forceinline__ void inv16_tw(uint32_t* x, const uint2* w, uint32_t q, uint32_t q2) {
-#pragma unroll
-    for (int t = 3; t >= 0; --t) {
-        const int h = 8 >> t;
-#pragma unroll
-        for (int g = 0; g < (1 << t); ++g)
-#pragma unroll
-            for (int r = 0; r < h; ++r) gs_bfly(x[2 * g * h + r], x[2 * g * h + r + h], w[(1 << t) - 1 + g], q, q2);
     }
 }
 
@@ -260,70 +214,4 @@ __device__ __forceinline__ void inv_p1_chunk(uint32_t* S, uint32_t* out, int c0,
 // ---- the persistent kernel ---------------------------------------------------------------
 // chunk k of a row: forward  k <  C1 -> phase-1 chunk k (src = in),  else phase-2 chunk k-C1 (src = out)
 //                   inverse  k <  C2 -> phase-2' chunk k (src = in), else phase-1' chunk k-C2 (src = out)
-template <int LOGN, bool FWD, bool PW, int TT = 512>
-__global__ void __launch_bounds__(TT, 1024 / TT) ntt_persist_cc(NttArgs a, uint32_t rows) {
-    using G = PGeo<LOGN, TT>;
-    constexpr int CA = FWD ? G::C1 : G::C2;          // chunks of the first phase
-    constexpr int CH = G::C1 + G::C2;
-    extern __shared__ __align__(16) uint32_t smem[];
-    if (blockIdx.x >= rows) return;
-
-    // row-outer / chunk-inner: per-row constants (limb, LimbConst, pointers) are computed once
-    // per row, and the next row's LimbConst is fetched one row ahead
-    auto issue = [&](uint32_t row_id, int kk, uint32_t* S) {
-        const uint32_t* in = a.in + ((size_t)row_id << LOGN);
-        const uint32_t* mid = a.out + ((size_t)row_id << LOGN);
-        if (FWD) {
-            if (kk < G::C1) load_p1<LOGN, TT>(S, in, kk * G::W1);
-            else load_p2<LOGN, TT>(S, mid, (kk - G::C1) * G::W2);
-        } else {
-            if (kk < G::C2) load_p2<LOGN, TT>(S, in, kk * G::W2);
-            else load_p1<LOGN, TT>(S, mid, (kk - G::C2) * G::W1);
-        }
-        cp_async_commit();
-    };
-    uint32_t row_id = blockIdx.x;
-    LimbConst lc = a.lc[row_id % a.L];
-    uint32_t buf = 0;
-    issue(row_id, 0, smem);
-#pragma unroll 1
-    while (row_id < rows) {
-        const uint32_t next = row_id + gridDim.x;
-        const uint32_t limb = row_id % a.L;
-        const LimbConst lcn = a.lc[(next < rows ? next : row_id) % a.L];    // in flight during this row
-        const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
-        uint32_t* out = a.out + ((size_t)row_id << LOGN);
-        const uint32_t* in2 = a.in2 + ((size_t)row_id << LOGN);
-#pragma unroll 1
-        for (int kk = 0; kk < CH; ++kk, buf ^= 1) {
-            uint32_t* S = smem + buf * G::BUF_WORDS;
-            uint32_t* Sn = smem + (buf ^ 1) * G::BUF_WORDS;
-            // chunk kk+1 may be the first chunk of phase B of this row: it reads what this chunk writes
-            const bool dep = (kk + 1 == CA);
-            const bool more = kk + 1 < CH || next < rows;
-            if (more && !dep) {
-                if (kk + 1 < CH) issue(row_id, kk + 1, Sn);
-                else issue(next, 0, Sn);
-                cp_async_wait<1>();
-            } else {
-                cp_async_wait<0>();
-            }
-            __syncthreads();
-            if (FWD) {
-                if (kk < G::C1) fwd_p1_chunk<LOGN, 0, TT>(S, out, kk * G::W1, tw, lc.q, lc.q2);
-                else fwd_p2_chunk<LOGN, 0, TT>(S, out, (kk - G::C1) * G::W2, tw, lc.q, lc.q2);
-            } else {
-                if (kk < G::C2) inv_p2_chunk<LOGN, PW, 0, TT>(S, out, in2, kk * G::W2, tw, lc);
-                else inv_p1_chunk<LOGN, 0, TT>(S, out, (kk - G::C2) * G::W1, tw, lc);
-            }
-            // bar.sync orders this chunk's global stores of the intermediate before the
-            // next chunk's cp.async reads of it (CTA-scope synchronisation, PTX memory model)
-            __syncthreads();
-            if (dep) issue(row_id, kk + 1, Sn);
-        }
-        lc = lcn;
-        row_id = next;
-    }
-}
-
 }  // namespace wd

@@ -15,7 +15,8 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
-#include "ntt_cuda_core.cuh"
+#include "common.cuh"
+#include "launch.h"
 
 namespace wd {
 
@@ -41,14 +42,6 @@ __global__ void __launch_bounds__(256) rs_gather(const uint4* __restrict__ in, u
 namespace wd {
 
 constexpr int BC_T = 128;                 // coefficients per CTA
-constexpr int BC_MAX = 64;                // max source / target limbs
-
-struct BconvTab {
-    const uint4* src;       // [S] {q_i, (Q/q_i)^-1 mod q_i, Shoup, 0}
-    const uint2* w;         // [S][D] {(Q/q_i) mod p_j, its Shoup companion mod p_j}
-    const uint4* dst;       // [D] {p_j, mu_lo, mu_hi, 0}: mu = floor((2^64 - 1) / p_j)
-    uint32_t S, D;
-};
 
 __device__ __forceinline__ uint32_t reduce64(uint64_t v, uint32_t p, uint64_t mu) {
     const uint64_t quo = __umul64hi(v, mu);

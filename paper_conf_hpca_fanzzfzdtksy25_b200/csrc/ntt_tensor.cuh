@@ -35,21 +35,6 @@
 
 namespace wd {
 
-struct TensorTables {
-    uint8_t* d_G = nullptr;        // [L][2][17][4096]: per direction, [0] = single-group stage (M0 / MI0),
-                                   //   [1+g] = stage-1 block of group g (M1_g / MI1_g), twists folded in
-    uint8_t* d_B = nullptr;        // [L][4][4096]: fwd M0, fwd F, inv MI0 (with N^-1), inv F'
-    uint2* d_tw1 = nullptr;        // [L][16][16]    fwd twist tau, stage 1   (group, j)
-    uint2* d_tw2 = nullptr;        // [L][256][16]   fwd twist tau, stage 2
-    uint2* d_tw3 = nullptr;        // [L][4096][16]  fwd twist tau, stage 3
-    uint2* d_sg1 = nullptr;        // [L][16][16]    inv twist sigma, stage 1' (group, k)
-    uint2* d_sg2 = nullptr;        // [L][256][16]
-    uint2* d_sg3 = nullptr;        // [L][4096][16]
-    uint2* d_c16 = nullptr;        // [L] Shoup companions of 2^16 and of 1
-    uint32_t* d_mat = nullptr;     // [L][4][256] u32 block matrices M0, F, MI0 (N^-1), F' (WD-CUDA, row f2)
-    bool ok = false;
-};
-
 struct TcArgs {
     NttArgs a;
     const uint8_t* B;
@@ -57,8 +42,6 @@ struct TcArgs {
     const uint2* c16;
 };
 
-inline bool tensor_supported(uint32_t logN) { return logN == 16; }
-inline float default_tensor_share(uint32_t) { return -1.0f; }   // < 0: dynamic split in FUSED mode
 
 // ------------------------------------------------------------------ device helpers
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -632,129 +615,6 @@ __global__ void __launch_bounds__(TC_T, TC_CTAS_PER_SM) ntt_tc16(TcArgs ta, uint
     tc_fence_before();
     __syncthreads();
     if (tid < 32) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" :: "r"(tmem));
-}
-
-// ------------------------------------------------------------------ host side
-inline void free_tensor_tables(TensorTables& t) {
-    cudaFree(t.d_G); cudaFree(t.d_B); cudaFree(t.d_tw1); cudaFree(t.d_tw2); cudaFree(t.d_tw3);
-    cudaFree(t.d_sg1); cudaFree(t.d_sg2); cudaFree(t.d_sg3); cudaFree(t.d_c16); cudaFree(t.d_mat);
-    t = TensorTables();
-}
-
-// Builds and verifies the factorised block tables for every limb (logN == 16 only).
-inline int build_tensor_tables(TensorTables& tc, uint32_t logN, const std::vector<uint32_t>& primes,
-                               const std::vector<uint32_t>& psis) {
-    if (logN != 16) return 0;
-    const uint32_t N = 1u << 16, L = (uint32_t)primes.size();
-    std::vector<uint8_t> B((size_t)L * 4 * 4096), Gi((size_t)L * 2 * 17 * 4096);
-    std::vector<uint2> t1((size_t)L * 256), t2((size_t)L * 4096), t3((size_t)L * 65536);
-    std::vector<uint2> s1((size_t)L * 256), s2((size_t)L * 4096), s3((size_t)L * 65536);
-    std::vector<uint2> c16(L);
-    std::vector<uint32_t> mat((size_t)L * 4 * 256);
-    for (uint32_t l = 0; l < L; ++l) {
-        const uint32_t q = primes[l], psi = psis[l], psi_inv = pm_pow(psi, q - 2, q);
-        std::vector<uint32_t> pw(N), pwi(N), fb(N), ib(N);
-        pw[0] = pwi[0] = 1;
-        for (uint32_t i = 1; i < N; ++i) { pw[i] = pm_mul(pw[i - 1], psi, q); pwi[i] = pm_mul(pwi[i - 1], psi_inv, q); }
-        for (uint32_t i = 0; i < N; ++i) { fb[i] = pw[pm_brv(i, 16)]; ib[i] = pwi[pm_brv(i, 16)]; }
-        const uint32_t ninv = pm_pow(N % q, q - 2, q);
-        uint32_t M[16][16], F[16][16], Fi[16][16];
-        block_fwd(M, fb, 0, 0, q);
-        std::memcpy(&mat[((size_t)l * 4 + 0) * 256], M, 1024);
-        byte_planes(&B[((size_t)l * 4 + 0) * 4096], M, q);
-        byte_planes(&Gi[(((size_t)l * 2 + 0) * 17 + 0) * 4096], M, q);
-        block_inv(M, ib, 0, 0, q, ninv);
-        std::memcpy(&mat[((size_t)l * 4 + 2) * 256], M, 1024);
-        byte_planes(&B[((size_t)l * 4 + 2) * 4096], M, q);
-        byte_planes(&Gi[(((size_t)l * 2 + 1) * 17 + 0) * 4096], M, q);
-        for (uint32_t g = 0; g < 16; ++g) {              // stage-1 blocks, one image per group
-            block_fwd(M, fb, 4, g, q);
-            byte_planes(&Gi[(((size_t)l * 2 + 0) * 17 + 1 + g) * 4096], M, q);
-            block_inv(M, ib, 4, g, q, 0);
-            byte_planes(&Gi[(((size_t)l * 2 + 1) * 17 + 1 + g) * 4096], M, q);
-        }
-        // fixed DFTs from one group, then every group of stages 1..3 must factor through them
-        bool have_f = false;
-        struct S { int ls; uint32_t groups; uint2* tw; uint2* sg; };
-        S st[3] = {{4, 16, &t1[(size_t)l * 256], &s1[(size_t)l * 256]},
-                   {8, 256, &t2[(size_t)l * 4096], &s2[(size_t)l * 4096]},
-                   {12, 4096, &t3[(size_t)l * 65536], &s3[(size_t)l * 65536]}};
-        for (auto& s : st) {
-            for (uint32_t g = 0; g < s.groups; ++g) {
-                uint32_t Mf[16][16], Mi[16][16];
-                block_fwd(Mf, fb, s.ls, g, q);
-                block_inv(Mi, ib, s.ls, g, q, 0);
-                for (int j = 0; j < 16; ++j) {
-                    const uint32_t tau = Mf[0][j], taui = pm_pow(tau, q - 2, q);
-                    const uint32_t sig = Mi[j][0], sigi = pm_pow(sig, q - 2, q);
-                    s.tw[g * 16 + j] = make_uint2(tau, pm_shoup(tau, q));
-                    s.sg[g * 16 + j] = make_uint2(sig, pm_shoup(sig, q));
-                    for (int k = 0; k < 16; ++k) {
-                        const uint32_t f = pm_mul(Mf[k][j], taui, q);       // F[k][j]
-                        const uint32_t fi = pm_mul(Mi[j][k], sigi, q);      // F'[j][k]
-                        if (!have_f) { F[k][j] = f; Fi[j][k] = fi; }
-                        else if (F[k][j] != f || Fi[j][k] != fi) return 4;  // factorisation failed
-                    }
-                }
-                have_f = true;
-            }
-        }
-        byte_planes(&B[((size_t)l * 4 + 1) * 4096], F, q);
-        byte_planes(&B[((size_t)l * 4 + 3) * 4096], Fi, q);
-        std::memcpy(&mat[((size_t)l * 4 + 1) * 256], F, 1024);
-        std::memcpy(&mat[((size_t)l * 4 + 3) * 256], Fi, 1024);
-        c16[l] = make_uint2(pm_shoup(65536u % q, q), pm_shoup(1u, q));
-    }
-    auto up = [](void** d, const void* h, size_t n) {
-        if (cudaMalloc(d, n) != cudaSuccess) return false;
-        return cudaMemcpy(*d, h, n, cudaMemcpyHostToDevice) == cudaSuccess;
-    };
-    if (!up((void**)&tc.d_G, Gi.data(), Gi.size()) || !up((void**)&tc.d_B, B.data(), B.size()) || !up((void**)&tc.d_tw1, t1.data(), t1.size() * 8) ||
-        !up((void**)&tc.d_tw2, t2.data(), t2.size() * 8) || !up((void**)&tc.d_tw3, t3.data(), t3.size() * 8) ||
-        !up((void**)&tc.d_sg1, s1.data(), s1.size() * 8) || !up((void**)&tc.d_sg2, s2.data(), s2.size() * 8) ||
-        !up((void**)&tc.d_sg3, s3.data(), s3.size() * 8) || !up((void**)&tc.d_c16, c16.data(), c16.size() * 8) ||
-        !up((void**)&tc.d_mat, mat.data(), mat.size() * 4))
-        return 4;
-    tc.ok = true;
-    return 0;
-}
-
-inline int prepare_tensor_kernels(uint32_t logN) {
-    if (logN != 16) return 0;
-    for (auto k : {ntt_tc16<true>, ntt_tc16<false>, ntt_tc16<true, 2>, ntt_tc16<false, 2>})
-        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM) != cudaSuccess ||
-            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
-            return 4;
-    for (auto k : {ntt_tcc16<true>, ntt_tcc16<false>})
-        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, TCC_SMEM) != cudaSuccess ||
-            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
-            return 4;
-    return 0;
-}
-
-// TENSOR mode launch (FUSED lives in ntt_fused.cuh)
-inline int launch_tensor(uint32_t logN, bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows,
-                         int sm_count, cudaStream_t s) {
-    if (logN != 16 || !tc.ok) return -1;
-    TcArgs ta;
-    ta.a = a;
-    ta.B = tc.d_B;
-    ta.t1 = fwd ? tc.d_tw1 : tc.d_sg1;
-    ta.t2 = fwd ? tc.d_tw2 : tc.d_sg2;
-    ta.t3 = fwd ? tc.d_tw3 : tc.d_sg3;
-    ta.c16 = tc.d_c16;
-    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)(sm_count * TC_CTAS_PER_SM));
-    // column phase: TMEM-staged, both stages folded (one CTA per SM, whole TMEM), limb-major ranges
-    const uint32_t gc = std::min<uint32_t>(rows, (uint32_t)sm_count);
-    const uint32_t per = (rows + gc - 1) / gc;
-    if (fwd) {
-        ntt_tcc16<true><<<gc, TC_T, TCC_SMEM, s>>>(ta, tc.d_G, rows, per);
-        ntt_tc16<true, 2><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
-    } else {
-        ntt_tc16<false, 2><<<grid, TC_T, TC_SMEM, s>>>(ta, rows);
-        ntt_tcc16<false><<<gc, TC_T, TCC_SMEM, s>>>(ta, tc.d_G, rows, per);
-    }
-    return 2;
 }
 
 }  // namespace wd

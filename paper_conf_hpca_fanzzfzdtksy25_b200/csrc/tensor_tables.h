@@ -22,11 +22,27 @@
 // between K-adjacent core matrices, SBO = 512 B between 8-row groups).
 #pragma once
 #include <cstdint>
+#include <vector_types.h>
 #include <cstring>
 #include <vector>
 #include "plan_math.h"
 
 namespace wd {
+
+struct TensorTables {
+    uint8_t* d_G = nullptr;        // [L][2][17][4096]: per direction, [0] = single-group stage (M0 / MI0),
+                                   //   [1+g] = stage-1 block of group g (M1_g / MI1_g), twists folded in
+    uint8_t* d_B = nullptr;        // [L][4][4096]: fwd M0, fwd F, inv MI0 (with N^-1), inv F'
+    uint2* d_tw1 = nullptr;        // [L][16][16]    fwd twist tau, stage 1   (group, j)
+    uint2* d_tw2 = nullptr;        // [L][256][16]   fwd twist tau, stage 2
+    uint2* d_tw3 = nullptr;        // [L][4096][16]  fwd twist tau, stage 3
+    uint2* d_sg1 = nullptr;        // [L][16][16]    inv twist sigma, stage 1' (group, k)
+    uint2* d_sg2 = nullptr;        // [L][256][16]
+    uint2* d_sg3 = nullptr;        // [L][4096][16]
+    uint2* d_c16 = nullptr;        // [L] Shoup companions of 2^16 and of 1
+    uint32_t* d_mat = nullptr;     // [L][4][256] u32 block matrices M0, F, MI0 (N^-1), F' (WD-CUDA, row f2)
+    bool ok = false;
+};
 
 inline uint32_t umma_off(int row, int kbyte) {        // byte offset in a K-major, 64-byte-K tile
     return (uint32_t)((row & 7) * 16 + (row >> 3) * 512 + (kbyte >> 4) * 128 + (kbyte & 15));

@@ -64,7 +64,6 @@ _SIGS = {
     "wd_ntt_plan_autotune": (_i32, [_vp, _u32, _vp, ctypes.POINTER(ctypes.c_float)]),
     "wd_ntt_plan_get_mode": (_i32, [_vp]),
     "wd_ntt_last_launches": (_u32, []),
-    "wd_ntt_occupancy": (_i32, [_vp, _i32, _i32]),
     "wd_ntt_last_error": (_i32, []),
     "wd_ntt_strerror": (ctypes.c_char_p, [_i32]),
     "wd_ntt_version": (ctypes.c_char_p, []),
@@ -216,11 +215,6 @@ def wd_ntt_plan_get_mode(plan: int) -> int:
 
 def wd_ntt_last_launches() -> int:
     return _lib.wd_ntt_last_launches()
-
-
-def wd_ntt_occupancy(plan: int, mode, fwd: bool = True) -> int:
-    mode = MODES[mode] if isinstance(mode, str) else int(mode)
-    return _lib.wd_ntt_occupancy(plan, mode, 1 if fwd else 0)
 
 
 def wd_ntt_last_error() -> int:

@@ -144,7 +144,9 @@ def test_pointwise_inverse_is_negacyclic_product(wd):
 
 
 # -------------------------------------------------------------- BASELINE configs at full size
-def _full_size_check(wd, n, L, batch, seed, nsample=12):
+def _full_size_check(wd, n, L, batch, seed):
+    """Every row of the forward AND the inverse against the (multithreaded) oracle, in the launch
+    configuration bench.py times (AUTO, out of place), plus the exact round trip on the device."""
     primes = P[:L]
     x = inputs.uniform_residues(primes, n, batch, seed)
     plan = wd.Plan(n, primes)
@@ -152,30 +154,22 @@ def _full_size_check(wd, n, L, batch, seed, nsample=12):
     y = torch.empty_like(d)
     plan.forward(d, y)
     torch.cuda.synchronize()
-    # sampled rows vs oracle (same launch configuration as bench.py)
-    rng = np.random.default_rng(seed)
-    rows = rng.choice(batch * L, size=nsample, replace=False)
-    yh = to_host(y.view(batch * L, n)[torch.as_tensor(rows, device="cuda")])
-    for k, r in enumerate(rows):
-        b, l = divmod(int(r), L)
-        assert np.array_equal(yh[k], oracle.ntt_forward_row(x[b, l], primes[l])), (b, l)
-    # every row: sum rule  sum_i out[i] = N * x[0]  (mod q)
-    q = torch.tensor(primes, dtype=torch.int64, device="cuda").view(1, L)
-    s = y.view(batch, L, n).to(torch.int64).sum(-1) % q
-    x0 = d.view(batch, L, n)[:, :, 0].to(torch.int64)
-    assert torch.equal(s, (x0 * n) % q)
-    # every row: canonical range and exact round trip
-    assert bool((y.view(batch, L, n).to(torch.int64) < q.view(1, L, 1)).all())
+    yh = to_host(y)
+    assert np.array_equal(yh, oracle.ntt_forward(x, primes))
     z = torch.empty_like(y)
     plan.inverse(y, z)
     torch.cuda.synchronize()
     assert torch.equal(z, d)
+    # the inverse on its own input distribution (uniform residues read as NTT values)
+    plan.inverse(d, z)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(z), oracle.ntt_inverse(x, primes))
     del d, y, z
     torch.cuda.empty_cache()
 
 
 def test_config2_one_ciphertext(wd):
-    _full_size_check(wd, 1 << 16, 36, 2, inputs.SEED_BASE + 1, nsample=8)
+    _full_size_check(wd, 1 << 16, 36, 2, inputs.SEED_BASE + 1)
 
 
 def test_config3_headline_64_ciphertexts(wd):
@@ -183,7 +177,30 @@ def test_config3_headline_64_ciphertexts(wd):
 
 
 def test_config4_n131072_l48(wd):
-    _full_size_check(wd, 1 << 17, 48, 64, inputs.SEED_BASE + 3, nsample=8)
+    _full_size_check(wd, 1 << 17, 48, 64, inputs.SEED_BASE + 3)
+
+
+# -------------------------------------------------------------- AUTO's decision boundaries
+# AUTO picks the kernel (v1 / v5 / v8) and v8's cluster size (8, 4, 2, 1 CTAs per row) from N and
+# the row count, with thresholds at SM/4, SM/2, SM and 8 x SM rows (wd_ntt.cu launch_cuda_core).
+# Every N, every threshold +-1, every row of both directions against the oracle.
+def _boundary_rows():
+    sm = torch.cuda.get_device_properties(0).multi_processor_count if torch.cuda.is_available() else 148
+    pts = {1, sm // 4 - 1, sm // 4, sm // 2, sm // 2 + 1, sm - 1, sm, sm + 1, 8 * sm - 1, 8 * sm}
+    return sorted(pts)
+
+
+@pytest.mark.parametrize("logn", [12, 13, 14, 15, 16, 17])
+def test_auto_decision_boundaries(wd, logn):
+    n = 1 << logn
+    for rows in _boundary_rows():
+        primes = [P[(rows + logn) % 60]]
+        x = inputs.uniform_residues(primes, n, rows, 7000 + logn * 10007 + rows)
+        plan = wd.Plan(n, primes)
+        y = gpu_fwd(wd, plan, x)
+        assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, rows)
+        assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (logn, rows)
+        plan.close()
 
 
 @pytest.mark.parametrize("logn,L", [(12, 1), (13, 60), (14, 17), (15, 9), (16, 60), (17, 2)])
@@ -250,7 +267,9 @@ def test_modes_headline_config(wd, mode, share):
 
 
 # -------------------------------------------------------------- every CUDA-core kernel generation
-@pytest.mark.parametrize("ver", ["v1", "v2", "v3", "v5", "v6", "v7", "v8", "v9", "v10", "v11", "v12"])
+# WD_NTT_KERNEL (read at plan creation) forces v1 (one CTA per row), v5 (row in a cluster's DSMEM,
+# N >= 2^14) or v8 (the default) regardless of the row count.
+@pytest.mark.parametrize("ver", ["v1", "v5", "v8"])
 @pytest.mark.parametrize("logn", [12, 13, 14, 15, 16, 17])
 def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", ver)
@@ -273,42 +292,53 @@ def test_cuda_core_generations(wd, ver, logn, monkeypatch):
     assert np.array_equal(to_host(o), oracle.ntt_inverse(prod.astype(np.uint32), primes)), (ver, logn)
 
 
-# -------------------------------------------------------------- persistent kernels over many rows
-# More rows than resident CTAs (clusters), so every CTA walks several rows and the cross-row
-# prefetches (v9: next row's first unit staged during the current row) are exercised; the row
-# count is ragged with respect to the grid.
-@pytest.mark.parametrize("ver", ["v8", "v9", "v10", "v11", "v12"])
-@pytest.mark.parametrize("logn,batch", [(14, 161), (15, 97), (16, 83)])
-def test_persistent_many_rows(wd, ver, logn, batch, monkeypatch):
-    monkeypatch.setenv("WD_NTT_KERNEL", ver)
+# v8 at every cluster size (WD_NTT_CL), over more rows than resident clusters and a ragged count
+@pytest.mark.parametrize("cl", ["1", "2", "4", "8"])
+@pytest.mark.parametrize("logn,batch", [(13, 301), (14, 161), (15, 97), (16, 83), (17, 45)])
+def test_v8_cluster_sizes_many_rows(wd, cl, logn, batch, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", "v8")
+    monkeypatch.setenv("WD_NTT_CL", cl)
     n = 1 << logn
     primes = [P[1], P[7], P[30], P[58]]
     x = inputs.uniform_residues(primes, n, batch, 5100 + logn)
     plan = wd.Plan(n, primes, mode="cuda")
     y = gpu_fwd(wd, plan, x)
-    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (ver, logn)
-    assert np.array_equal(gpu_inv(wd, plan, y), x), (ver, logn)
-    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (ver, logn)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (cl, logn)
+    assert np.array_equal(gpu_inv(wd, plan, y), x), (cl, logn)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (cl, logn)
 
 
-# Primes across the range the ABI accepts: the tensor column phase (v10) recombines its byte
-# planes with a cheaper reduction when q > 2^29 and a general one below; both must be exact.
+# Primes across the range the ABI accepts (the lazy bounds [0, 4q) < 2^32 hold for any q < 2^30).
 # 786433 = 3 * 2^18 + 1; the others are the first primes = 1 (mod 2^17) above 2^28, 2^29, 1.5*2^29.
-@pytest.mark.parametrize("ver", ["v8", "v10", "v11", "v12"])
-def test_prime_sizes_n16(wd, ver, monkeypatch):
-    monkeypatch.setenv("WD_NTT_KERNEL", ver)
+@pytest.mark.parametrize("mode", ["cuda", "tensor", "fused", "cuda_gemm"])
+def test_prime_sizes_n16(wd, mode):
     n = 1 << 16
     primes = [786433, 269221889, 537133057, 805961729, P[0]]
     for q in primes:
         assert oracle.is_prime(q) and (q - 1) % (2 * n) == 0
     x = inputs.uniform_residues(primes, n, 3, 5200)
-    plan = wd.Plan(n, primes, mode="cuda")
+    plan = wd.Plan(n, primes, mode=mode)
     y = gpu_fwd(wd, plan, x)
-    assert np.array_equal(y, oracle.ntt_forward(x, primes)), ver
-    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), ver
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), mode
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), mode
     q = np.repeat(inputs.structured("qm1", primes, n), 3, axis=0)
-    assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes)), ver
-    assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes)), ver
+    assert np.array_equal(gpu_fwd(wd, plan, q), oracle.ntt_forward(q, primes)), mode
+    assert np.array_equal(gpu_inv(wd, plan, q), oracle.ntt_inverse(q, primes)), mode
+
+
+# Every tensor-using mode at a ragged batch whose limbs change inside a CTA's row range
+# (335 rows over 148 CTAs: 2-3 rows each, limb-major), every row against the oracle
+@pytest.mark.parametrize("mode,share", [("tensor", -1.0), ("fused", -1.0), ("fused", 0.5), ("cuda_gemm", -1.0),
+                                        ("ftc", 0.6)])
+def test_tensor_modes_ragged_limbs(wd, mode, share):
+    n = 1 << 16
+    primes = [P[4], P[21], P[44], 786433, 805961729]
+    x = inputs.uniform_residues(primes, n, 67, 5600)
+    plan = wd.Plan(n, primes)
+    plan.set_mode(mode, share)
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), mode
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), mode
 
 
 # -------------------------------------------------------------- WD-CUDA (row f2): 32-bit GEMM inner DFTs
@@ -346,22 +376,6 @@ def test_wd_ftc_mode(wd, batch, share):
     assert np.array_equal(to_host(d), y)
     with pytest.raises(wd.WdNttError):
         wd.Plan(1 << 15, P[:2], mode="ftc")                # N = 2^16 only
-
-
-# v11: every tensor / butterfly split of the row phase (bit st-1 of WD_NTT_TMASK = stage st on the
-# tensor cores), over more rows than resident CTAs
-@pytest.mark.parametrize("tmask", ["1", "3", "6", "7"])
-def test_v11_stage_splits(wd, tmask, monkeypatch):
-    monkeypatch.setenv("WD_NTT_KERNEL", "v11")
-    monkeypatch.setenv("WD_NTT_TMASK", tmask)
-    n = 1 << 16
-    primes = [P[2], P[31], 786433, 537133057]
-    x = inputs.uniform_residues(primes, n, 80, 5400 + int(tmask))
-    plan = wd.Plan(n, primes, mode="cuda")
-    y = gpu_fwd(wd, plan, x)
-    assert np.array_equal(y, oracle.ntt_forward(x, primes)), tmask
-    assert np.array_equal(gpu_inv(wd, plan, y), x), tmask
-    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), tmask
 
 
 # -------------------------------------------------------------- row a9: split chosen from measurement
