@@ -64,6 +64,10 @@ typedef struct CUstream_st* wd_stream_t;       /* == cudaStream_t */
                               * of the polynomials and WD-CUDA on the rest, the two running *
                               * concurrently on the same GPU (an internal forked stream,    *
                               * joined back into the caller's stream), N = 2^16 only       */
+#define WD_MODE_TC4      6   /* 4-step tcgen05 kernel, warp-specialised: TMA producer, one   *
+                              * MMA-issuing thread, CUDA-core epilogue warps working on     *
+                              * other tiles at the same time, *
+                              * N = 2^16 only                                              */
 
 /*
  * wd_ntt_plan_create -- PAPER.md:358 (initialisation phase: moduli, twiddles

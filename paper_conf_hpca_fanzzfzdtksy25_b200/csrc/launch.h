@@ -4,6 +4,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <vector>
 #include "common.cuh"
 #include "tensor_tables.h"
 
@@ -29,6 +30,19 @@ int prep_tensor();
 int launch_tensor(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, cudaStream_t s);
 int launch_fused(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, float share,
                  cudaStream_t s);
+
+// ---- k_tc4.cu: the warp-specialised 4-step tcgen05 kernel (N = 2^16, ntt_tc4.cuh)
+struct Tc4Tables {
+    uint8_t* d_mat = nullptr;      // [L][2 sets][17][4096] byte-plane stage matrices (forward)
+    uint2* d_tw = nullptr;         // [L][2][16][16][128] per-element twist in worker-lane order (forward)
+    uint4* d_lq = nullptr;         // [L] {q, Shoup(2^16), Shoup(1), 0}
+    bool ok = false;
+};
+int build_tc4_tables(Tc4Tables& t, const std::vector<uint32_t>& primes, const std::vector<uint32_t>& psis);
+void free_tc4_tables(Tc4Tables& t);
+int prep_tc4();
+// returns launches (> 0), -1 unsupported arguments, -2 tensor-map encoding failure
+int launch_tc4(bool fwd, const NttArgs& a, const Tc4Tables& t, uint32_t rows, int sm_count, cudaStream_t s);
 
 // ---- k_rns.cu: RESCALE gather, fast basis conversion, 64-bit share reduction
 struct BconvTab {

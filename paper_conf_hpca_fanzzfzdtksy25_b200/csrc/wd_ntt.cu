@@ -53,6 +53,7 @@ struct wd_ntt_plan {
     uint32_t rs_thr = 0;           // q_last - floor(q_last / 2)
     bool rs_ok = false;            // L >= 2 and q_last differs from every other prime
     TensorTables tc;               // round-1 tensor-path tables (N = 2^16), built on first use
+    Tc4Tables t4;                  // 4-step tcgen05 kernel tables (N = 2^16), built on first use
     std::mutex tc_mu;
     int mode = WD_MODE_AUTO;
     float tensor_share = -1.0f;    // FUSED: share of rows whose column phase runs on tcgen05 (< 0: default)
@@ -79,6 +80,20 @@ int check_prime(uint32_t q, uint32_t N) {
 
 bool tensor_mode(int mode) {
     return mode == WD_MODE_TENSOR || mode == WD_MODE_FUSED || mode == WD_MODE_CUDA_GEMM || mode == WD_MODE_FTC;
+}
+
+int ensure_tc4_tables(wd_ntt_plan* p) {
+    std::lock_guard<std::mutex> lk(p->tc_mu);
+    if (p->t4.ok) return WD_OK;
+    if (p->logN != 16) return WD_EUNSUPPORTED;
+    int e;
+    try {
+        e = build_tc4_tables(p->t4, p->primes, p->psi);
+    } catch (const std::bad_alloc&) {
+        e = WD_ENOMEM;
+    }
+    if (e != WD_OK) { cudaGetLastError(); free_tc4_tables(p->t4); return e == WD_ENOMEM ? WD_ENOMEM : WD_ECUDA; }
+    return WD_OK;
 }
 
 // the round-1 tensor tables (TENSOR / FUSED / CUDA_GEMM / FTC), built when one of those modes is first
@@ -151,6 +166,12 @@ int run_mode(const wd_ntt_plan* p, int mode, float share, bool fwd, const uint32
     int launches = 0;
     if (in2 != nullptr || mode == WD_MODE_CUDA) {
         launches = launch_cuda_core(p, fwd, a, rows, s);
+    } else if (mode == WD_MODE_TC4) {
+        if (!p->t4.ok) return set_err(WD_EUNSUPPORTED);
+        if (fwd) launches = launch_tc4(fwd, a, p->t4, rows, p->sm_count, s);
+        else launches = launch_cuda_core(p, fwd, a, rows, s);          // inverse kernel: not yet built
+        if (launches == -2) return set_err(WD_ECUDA);
+        if (launches < 0) return set_err(WD_EUNSUPPORTED);
     } else {
         if (!p->tc.ok) return set_err(WD_EUNSUPPORTED);
         if (mode == WD_MODE_CUDA_GEMM) {
@@ -257,6 +278,7 @@ void free_plan(wd_ntt_plan* p) {
         if (cur != p->device) cudaSetDevice(p->device);
         cudaFree(p->d_fwd); cudaFree(p->d_inv); cudaFree(p->d_lc); cudaFree(p->d_rs);
         free_tensor_tables(p->tc);
+        free_tc4_tables(p->t4);
         for (auto& s : p->hs) if (s) cudaStreamDestroy(s);
         for (auto& e : p->he) if (e) cudaEventDestroy(e);
         if (p->fs) cudaStreamDestroy(p->fs);
@@ -415,7 +437,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (cudaStreamCreateWithFlags(&p->fs, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->fe) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     if (prep_cc(p->logN) || prep_v8(p->logN, p->sm_count, &p->occ) || prep_rns() ||
-        (p->logN == 16 && (prep_tensor() || prep_wdcuda()))) {
+        (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4()))) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
     p->mode = WD_MODE_AUTO;
@@ -661,8 +683,13 @@ int wd_ntt_check_prime(uint32_t q, uint32_t N) {
 }
 
 int wd_ntt_plan_set_mode(wd_ntt_plan* p, int mode, float tensor_share) {
-    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_FTC) return set_err(WD_EINVAL);
+    if (!p || mode < WD_MODE_AUTO || mode > WD_MODE_TC4) return set_err(WD_EINVAL);
     if (tensor_share > 1.0f) return set_err(WD_EINVAL);
+    if (mode == WD_MODE_TC4) {
+        if (p->logN != 16) return set_err(WD_EUNSUPPORTED);
+        const int e = ensure_tc4_tables(p);
+        if (e != WD_OK) return set_err(e);
+    }
     if (tensor_mode(mode)) {
         if (p->logN != 16) return set_err(WD_EUNSUPPORTED);
         const int e = ensure_tensor_tables(p);

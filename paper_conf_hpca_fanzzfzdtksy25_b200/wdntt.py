@@ -20,9 +20,9 @@ LIB_PATH = os.path.join(_HERE, "libwdntt.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "wd_ntt.h")
 
 WD_OK, WD_EINVAL, WD_EPRIME, WD_EUNSUPPORTED, WD_ECUDA, WD_ENOMEM = range(6)
-WD_MODE_AUTO, WD_MODE_CUDA, WD_MODE_TENSOR, WD_MODE_FUSED, WD_MODE_CUDA_GEMM, WD_MODE_FTC = range(6)
+WD_MODE_AUTO, WD_MODE_CUDA, WD_MODE_TENSOR, WD_MODE_FUSED, WD_MODE_CUDA_GEMM, WD_MODE_FTC, WD_MODE_TC4 = range(7)
 MODES = {"auto": WD_MODE_AUTO, "cuda": WD_MODE_CUDA, "tensor": WD_MODE_TENSOR, "fused": WD_MODE_FUSED,
-         "cuda_gemm": WD_MODE_CUDA_GEMM, "ftc": WD_MODE_FTC}
+         "cuda_gemm": WD_MODE_CUDA_GEMM, "ftc": WD_MODE_FTC, "tc4": WD_MODE_TC4}
 
 
 class WdNttError(RuntimeError):
