@@ -243,6 +243,11 @@ int wd_ntt_plan_autotune(wd_ntt_plan* plan, uint32_t batch, wd_stream_t stream, 
 /* Kernel launches issued by the last forward/inverse call on this thread. */
 uint32_t wd_ntt_last_launches(void);
 
+/* Diagnostics only: while dev_buf (device memory, 20480 uint64 words) is set, every WD_MODE_TC4 launch
+ * records clock64() timestamps of CTA 0's pipeline events into it (loads, MMAs, accumulator
+ * hand-over, staging hand-over, stores; ntt_tc4.cuh TR_*).  NULL switches it off.  Process-wide. */
+void wd_ntt_debug_tc4_trace(void* dev_buf);
+
 int         wd_ntt_last_error(void);
 const char* wd_ntt_strerror(int code);
 const char* wd_ntt_version(void);

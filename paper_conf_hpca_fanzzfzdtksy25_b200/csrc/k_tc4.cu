@@ -2,6 +2,7 @@
 // the per-element twist in worker-lane order, TMA tensor maps per call, launch.
 #include <cuda.h>
 #include <algorithm>
+#include <cstdio>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -150,7 +151,11 @@ bool encode(CUtensorMap* m, const void* base, uint32_t rank, const cuuint64_t* d
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+unsigned long long* g_trace = nullptr;     // diagnostics (wd_tc4_set_trace)
+
 }  // namespace
+
+void tc4_set_trace(void* p) { g_trace = static_cast<unsigned long long*>(p); }
 
 void free_tc4_tables(Tc4Tables& t) {
     cudaFree(t.d_mat); cudaFree(t.d_tw); cudaFree(t.d_lq);
@@ -244,8 +249,17 @@ int launch_tc4(bool fwd, const NttArgs& a, const Tc4Tables& t, uint32_t rows, in
     ta.tw = t.d_tw;
     ta.lq = t.d_lq;
     ta.rows = rows; ta.L = a.L; ta.nb = rows / a.L;
+    ta.trace = g_trace;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
     tc4::ntt_tc4_fwd<<<grid, tc4::NT, tc4::SMEM, s>>>(mx, mc, mi, mo, ta);
+    const cudaError_t e = cudaPeekAtLastError();
+    if (e != cudaSuccess) {
+        cudaFuncAttributes fa;
+        cudaFuncGetAttributes(&fa, tc4::ntt_tc4_fwd);
+        fprintf(stderr, "wdntt: tc4 launch failed: %s (regs %d, maxThreads %d, smem %u, localBytes %zu)\n",
+                cudaGetErrorString(e), fa.numRegs, fa.maxThreadsPerBlock, tc4::SMEM, fa.localSizeBytes);
+        return -2;
+    }
     return 1;
 }
 

@@ -42,6 +42,7 @@ int build_tc4_tables(Tc4Tables& t, const std::vector<uint32_t>& primes, const st
 void free_tc4_tables(Tc4Tables& t);
 int prep_tc4();
 // returns launches (> 0), -1 unsupported arguments, -2 tensor-map encoding failure
+void tc4_set_trace(void* dev_buf);   // diagnostics: CTA-0 event timestamps (20480 x u64) or nullptr
 int launch_tc4(bool fwd, const NttArgs& a, const Tc4Tables& t, uint32_t rows, int sm_count, cudaStream_t s);
 
 // ---- k_rns.cu: RESCALE gather, fast basis conversion, 64-bit share reduction

@@ -771,6 +771,8 @@ int wd_ntt_plan_autotune(wd_ntt_plan* p, uint32_t batch, wd_stream_t st, float* 
 
 uint32_t wd_ntt_last_launches(void) { return g_last_launches; }
 
+void wd_ntt_debug_tc4_trace(void* dev_buf) { tc4_set_trace(dev_buf); }
+
 int wd_ntt_last_error(void) { return g_last_error; }
 const char* wd_ntt_strerror(int code) {
     switch (code) {

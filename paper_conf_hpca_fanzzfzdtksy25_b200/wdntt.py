@@ -64,6 +64,7 @@ _SIGS = {
     "wd_ntt_plan_autotune": (_i32, [_vp, _u32, _vp, ctypes.POINTER(ctypes.c_float)]),
     "wd_ntt_plan_get_mode": (_i32, [_vp]),
     "wd_ntt_last_launches": (_u32, []),
+    "wd_ntt_debug_tc4_trace": (None, [_vp]),
     "wd_ntt_last_error": (_i32, []),
     "wd_ntt_strerror": (ctypes.c_char_p, [_i32]),
     "wd_ntt_version": (ctypes.c_char_p, []),
