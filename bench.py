@@ -27,6 +27,9 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
+if "WORLD_SIZE" in os.environ:            # under torchrun: NCCL communicator lines for the driver's rank check
+    os.environ.setdefault("NCCL_DEBUG", "INFO")
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
 
 CONFIGS = {
     # name: (logN, L, ciphertexts)
@@ -51,6 +54,26 @@ CONFIG_NAMES.update({"s%d" % _lg: "config5 sweep point N=2^%d, L=16, 128 polynom
 METRIC = "NTT KOPS (N=2^16, L=36) at 1/2/4/8 B200; % of HBM / int8 tensor roofline"
 FALLBACK_HBM_GBS = 6650.0
 BFLY_PER_CLK_SM = 13.57       # measured: scripts/int_probe.cu ct_bfly_hi, 4 CTAs/SM (profiles/r01/int_probe.jsonl)
+
+
+def i8_peak():
+    """Measured tcgen05 kind::i8 peak (scripts/tc4_probe.cu, committed under profiles/r02)."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "r02", "peaks_i8.json")))
+        return float(d["int8_tcgen05_peak_TMAC_per_s"]), float(d.get("n64_TMAC_per_s", 0.0)), "measured"
+    except Exception:
+        return 2250.0, 0.0, "nominal (4.5 POPS dense int8)"
+
+
+# int8 tensor MACs per N-point transform, per mode: every radix-16 byte-plane GEMM stage multiplies
+# 16 coefficients x 4 data bytes by 16 outputs x 4 byte planes, i.e. 256 MACs per output element
+# (SURVEY.md 8 row a5); N = 2^16 has 4 such stages (TENSOR, tc4 forward), FUSED runs the column
+# phase's two stages on tcgen05 (rows with the tensor share), WD-CUDA / CUDA none.
+def tensor_macs_per_transform(mode: str, n: int, fwd: bool) -> float:
+    if n != 1 << 16:
+        return 0.0
+    stages = {"tensor": 4, "tc4": 4 if fwd else 0, "fused": 2, "ftc": 4 * 0.7}.get(mode, 0)
+    return 256.0 * n * stages
 
 
 def peaks():
@@ -343,13 +366,136 @@ def run_polymul(args):
     print(json.dumps(line), flush=True)
 
 
+def run_shard(args):
+    """--shard limbs (SURVEY.md 8 row e; BASELINE configs[3]: N=2^17, L=48, limbs sharded over 2/4/8
+    GPUs).  Rank g owns limbs [g L / G, (g+1) L / G) of ONE batch and builds its own plan over those
+    primes; the NTT has no collective (limbs are independent).  Reported separately:
+      value           the resident-shard rate: every rank transforms its shard, inputs already in
+                      HBM, K steps of forward + inverse, barrier + max over ranks
+      scatter_gather  the same step with NCCL moving the data: rank 0 holds the whole batch, scatters
+                      the limb slices, every rank transforms, rank 0 gathers the results"""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import dist as wdist
+    from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dist.init_process_group("nccl", device_id=torch.device("cuda", local), rank=rank, world_size=world,
+                            init_method="env://" if "MASTER_ADDR" in os.environ else "tcp://127.0.0.1:%d" % (29500 + os.getpid() % 1000))
+    logn, L, nct = CONFIGS[args.config]
+    n = 1 << logn
+    batch = 1 if nct is None else 2 * nct
+    primes = inputs.bench_primes(L)
+    spans = [wdist.limb_range(L, world, g) for g in range(world)]
+    l0, l1 = spans[rank]
+    lg = l1 - l0
+    plan = wdntt.Plan(n, primes[l0:l1])
+    plan.set_mode(args.mode, args.share)
+    full = inputs.uniform_residues_torch(primes, n, batch, inputs.SEED_BASE + 3, device="cuda")
+    x = full[:, l0:l1].contiguous()
+    y, z = torch.empty_like(x), torch.empty_like(x)
+    sp = torch.cuda.current_stream().cuda_stream
+    stream = torch.cuda.current_stream()
+
+    def step():
+        wdntt.wd_ntt_forward(plan.handle, x, y, batch, sp)
+        a = wdntt.wd_ntt_last_launches()
+        wdntt.wd_ntt_inverse(plan.handle, y, z, batch, sp)
+        return a + wdntt.wd_ntt_last_launches()
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    assert torch.equal(z, x), "round trip failed"
+    dist.barrier()
+    torch.cuda.synchronize()
+    launches = 0
+    with ClockSampler(local) as clk:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            launches += step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+    t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device="cuda")
+    dist.barrier()
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    kops = 2 * batch * L * args.steps / (ms / 1e3) / 1e3
+
+    # ---- scatter + transform + gather through NCCL (rank 0 owns the whole batch; dist.py helpers,
+    # the same code the gloo CPU tests run)
+    sg_steps = max(1, min(args.steps, 5))
+    src_full = full if rank == 0 else None
+    result = {}
+
+    def sg_step():
+        xl = wdist.scatter_limbs(src_full, L, n, batch, src=0)
+        wdntt.wd_ntt_forward(plan.handle, xl, y, batch, sp)
+        wdntt.wd_ntt_inverse(plan.handle, y, z, batch, sp)
+        result["full"] = wdist.gather_limbs(z, L, n, batch, dst=0)
+
+    sg_step()
+    torch.cuda.synchronize()
+    if rank == 0:
+        assert torch.equal(result["full"], full), "scatter/gather round trip failed"
+    dist.barrier()
+    torch.cuda.synchronize()
+    g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    g0.record(stream)
+    for _ in range(sg_steps):
+        sg_step()
+    g1.record(stream)
+    torch.cuda.synchronize()
+    tg = torch.tensor([g0.elapsed_time(g1)], dtype=torch.float64, device="cuda")
+    dist.all_reduce(tg, op=dist.ReduceOp.MAX)
+    sg_ms = float(tg.item())
+    if rank == 0:
+        pk, pk_kind = peaks()
+        hbm = float(pk.get("hbm_gbs", FALLBACK_HBM_GBS))
+        per_rank_ms = ms / args.steps / 2
+        alg = 8.0 * n * batch * lg
+        line = {
+            "metric": METRIC, "value": kops, "unit": "KOPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic (splitmix64 uniform residues, SURVEY.md 8.d)",
+            "config": {"workload": "%s: N=2^%d, L=%d limbs of %d polynomials sharded over %d GPU(s) (%s limbs per "
+                                   "rank), forward+inverse per step" % (CONFIG_NAMES.get(args.config, args.config), logn,
+                                                                         L, batch, world, "/".join(
+                                                                             str(b_ - a_) for a_, b_ in spans)),
+                       "N": n, "L": L, "polys": batch, "mode": args.mode, "parallelism": "limb shards, no collective in the NTT",
+                       "l2": "shard %.2f GB per rank" % (batch * lg * n * 4 / 1e9)},
+            "roofline": {"bound": "hbm", "kernel": "forward+inverse average (rank 0)",
+                         "achieved": alg / (per_rank_ms / 1e3) / 1e9, "peak": hbm, "unit": "GB/s",
+                         "frac": alg / (per_rank_ms / 1e3) / 1e9 / hbm, "traffic": None, "peak_kind": pk_kind},
+            "scatter_gather": {"value": 2 * batch * L * sg_steps / (sg_ms / 1e3) / 1e3, "unit": "KOPS",
+                               "ms_per_step": sg_ms / sg_steps, "bytes_scattered_per_step": batch * L * n * 4,
+                               "bytes_gathered_per_step": batch * L * n * 4,
+                               "api": "torch.distributed scatter/gather (NCCL) around wd_ntt_forward/inverse"},
+            "gpu_launches": launches, "clocks": clk.summary(),
+            "e2e": {"value": 2 * batch * L * sg_steps / (sg_ms / 1e3) / 1e3, "unit": "KOPS",
+                    "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+                    "note": "device-resident full batch on rank 0; the data movement is the NCCL scatter + gather"},
+        }
+        print(json.dumps(line), flush=True)
+    dist.destroy_process_group()
+
+
 def main():
+    if os.environ.get("WD_BENCH_WATCHDOG"):                    # debugging hangs: dump all stacks, exit
+        import faulthandler
+        faulthandler.dump_traceback_later(float(os.environ["WD_BENCH_WATCHDOG"]), exit=True)
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="wd", choices=["wd", "reference"])
-    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused", "cuda_gemm", "ftc"])
+    ap.add_argument("--mode", default="auto", choices=["auto", "cuda", "tensor", "fused", "cuda_gemm", "ftc", "tc4"])
+    ap.add_argument("--shard", default="none", choices=["none", "limbs"],
+                    help="limbs: under torchrun every rank owns L/G limbs of ONE batch (config 4's split); "
+                         "reports the resident-shard rate and the scatter + gather end to end separately")
     ap.add_argument("--share", type=float, default=-1.0, help="tensor share for --mode fused / ftc")
     ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -374,6 +520,9 @@ def main():
 
     if args.impl == "reference":
         run_reference(args)
+        return
+    if args.shard == "limbs":
+        run_shard(args)
         return
 
     import torch
@@ -536,15 +685,24 @@ def main():
 
     pk, pk_kind = peaks()
     hbm = float(pk.get("hbm_gbs", FALLBACK_HBM_GBS))
+    sms = torch.cuda.get_device_properties(local).multi_processor_count
     dom_ms, dom_name = (fwd_ms, "forward") if fwd_ms >= inv_ms else (inv_ms, "inverse")
     alg_bytes = 8.0 * n * rows                       # read 4N + write 4N bytes per transform
     achieved = alg_bytes / (dom_ms / 1e3) / 1e9
-    traffic = None
+    # DRAM traffic of the dominant launch: NOT measured in this run (that needs ncu); taken from the
+    # committed ncu --set full capture of the same launch and labelled with its source
+    traffic, traffic_src = None, None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        traffic = tr.get("%s_%s_%s" % (args.config, args.mode, dom_name))
+        key = "%s_%s_%s" % (args.config, args.mode, dom_name)
+        traffic = tr.get(key)
+        traffic_src = tr.get("_source", {}).get(key) if traffic is not None else None
     except Exception:
         pass
+    i8_pk, i8_pk64, i8_kind = i8_peak()
+    macs_f = tensor_macs_per_transform(args.mode, n, True) * rows
+    macs_i = tensor_macs_per_transform(args.mode, n, False) * rows
+    tmacs = max(macs_f / (fwd_ms / 1e3), macs_i / (inv_ms / 1e3)) / 1e12
     line = {
         "metric": METRIC, "value": kops, "unit": "KOPS", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
@@ -561,19 +719,25 @@ def main():
         "fwd_kops": rows * world / (fwd_ms / 1e3) / 1e3, "inv_kops": rows * world / (inv_ms / 1e3) / 1e3,
         "fwd_ms": fwd_ms, "inv_ms": inv_ms,
         "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved / hbm, "traffic": traffic,
+                     "frac": achieved / hbm, "traffic": traffic, "traffic_source": traffic_src,
                      "peak_kind": "%s (MEASURED_PEAKS.json hbm_gbs copy bandwidth)" % pk_kind,
                      "algorithmic_bytes_per_launch": alg_bytes},
+        # int8 tensor pipe: algorithmic byte-plane MACs of the launch / time / the measured kind::i8 peak
+        # (M=128 N=256 back-to-back MMAs; the N=64 tile shape of the NTT stages peaks at n64_peak)
+        "roofline_tensor": {"bound": "tensor", "achieved": tmacs, "peak": i8_pk, "unit": "TMAC/s (int8)",
+                            "frac": tmacs / i8_pk, "n64_peak": i8_pk64, "peak_kind": i8_kind,
+                            "macs_per_launch": {"forward": macs_f, "inverse": macs_i},
+                            "note": "0 for modes without tcgen05 work (cuda = v8 butterflies)"},
         # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
         # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
         # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
         # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
         "roofline_alu": {"bound": "alu", "kernel": dom_name,
                          "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
-                         "peak": BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3,
+                         "peak": BFLY_PER_CLK_SM * sms * (clk.summary()["sm_mhz"] or 1965) / 1e3,
                          "unit": "G butterflies/s",
                          "frac": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9
-                                 / (BFLY_PER_CLK_SM * 148 * (clk.summary()["sm_mhz"] or 1965) / 1e3),
+                                 / (BFLY_PER_CLK_SM * sms * (clk.summary()["sm_mhz"] or 1965) / 1e3),
                          "note": "algorithmic butterflies (N/2 log2 N per transform); the WD-CUDA and tensor "
                                  "modes do other work per element, for them this is a normalised rate"},
         "gpu_launches": launches,

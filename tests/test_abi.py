@@ -90,9 +90,9 @@ def test_binding_constants_match_header():
     import os
     import re
     hdr = open(os.path.join(os.path.dirname(__file__), "..", "include", "wd_ntt.h")).read()
-    defs = {m.group(1): int(m.group(2)) for m in re.finditer(r"#define\s+(WD_[A-Z_]+)\s+(\d+)", hdr)}
+    defs = {m.group(1): int(m.group(2)) for m in re.finditer(r"#define\s+(WD_[A-Z0-9_]+)\s+(\d+)", hdr)}
     modes = {k: v for k, v in defs.items() if k.startswith("WD_MODE_")}
-    assert len(modes) == 6 and modes["WD_MODE_FTC"] == 5
+    assert len(modes) == 7 and modes["WD_MODE_FTC"] == 5 and modes["WD_MODE_TC4"] == 6
     for name, val in defs.items():
         if hasattr(wdntt, name):
             assert getattr(wdntt, name) == val, name
