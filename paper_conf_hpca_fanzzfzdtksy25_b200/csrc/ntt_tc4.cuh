@@ -384,7 +384,10 @@ __global__ void __launch_bounds__(NT, 1) ntt_tc4_fwd(const __grid_constant__ CUt
     } else if (warp == W_STORE) {
         // ===================================================================== TMA store issuer
         if (lane == 0) {
-            uint32_t ns = 0;
+            // staging slots are released in order, SLAG stores behind the newest (their smem reads done)
+            constexpr uint32_t SLAG = 3;
+            static_assert(SLAG < NSTG, "staging ring");
+            uint32_t ns = 0, rel = 0;
             for (uint32_t p = 0; p < npass; ++p) {
                 uint32_t i, h; bool col;
                 pass_info(p, n, i, col, h);
@@ -397,13 +400,14 @@ __global__ void __launch_bounds__(NT, 1) ntt_tc4_fwd(const __grid_constant__ CUt
                     if (col) tma_store2(&tm_i, (int)(128 * h), (int)(row * 256 + 16 * brv4(k)), src);
                     else tma_store2(&tm_o, (int)(16 * brv4(k)), (int)(row * 256 + 128 * h), src);
                     bulk_commit();
-                    if (ns > 0) {                                 // store ns-1 has read its staging slot
-                        bulk_wait_read1();
-                        bar_arrive(&B.stg_empty[(ns - 1) % NSTG]);
+                    if (ns + 1 > rel + SLAG) {
+                        asm volatile("cp.async.bulk.wait_group.read %0;" :: "n"(SLAG) : "memory");
+                        for (; rel + SLAG < ns + 1; ++rel) bar_arrive(&B.stg_empty[rel % NSTG]);
                     }
                 }
                 if (col && h == 1) {                              // row i's intermediate complete in global
                     bulk_wait0();
+                    for (; rel < ns; ++rel) bar_arrive(&B.stg_empty[rel % NSTG]);
                     bar_arrive(&B.inter_done);
                 }
             }
