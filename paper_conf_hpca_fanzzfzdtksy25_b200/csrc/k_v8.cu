@@ -1,6 +1,7 @@
 // k_v8.cu -- launchers of the CUDA-core v8 kernel and of
 // WD-CUDA (row f2).  Kernels in ntt_v8.cuh.
 #include <algorithm>
+#include <cstdlib>
 #include "launch.h"
 #include "ntt_v8.cuh"
 
@@ -29,7 +30,9 @@ int prep_cl(int sm_count, V8Occ* occ) {
         if (CL == (LOGN > 12 ? 2 : 1))
             e |= set_smem(ntt_v8<LOGN, true, false, CL, 1>, V8_SMEM) | set_smem(ntt_v8<LOGN, true, false, CL, 2>, V8_SMEM);
         if (e) return e;
-        int ncl = sm_count * 4 / CL;
+        // WD_NTT_V8_CTAS (A/B runs, read once per plan): CTAs per SM the persistent grid is sized for
+        static const int ctas_env = getenv("WD_NTT_V8_CTAS") ? std::max(1, std::min(4, atoi(getenv("WD_NTT_V8_CTAS")))) : 4;
+        int ncl = sm_count * ctas_env / CL;
         if (CL > 1) {                    // resident clusters, queried once per plan (not per launch)
             cudaLaunchConfig_t cfg = {};
             cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM;
@@ -43,7 +46,7 @@ int prep_cl(int sm_count, V8Occ* occ) {
                 cudaGetLastError();
                 n = sm_count * 4 / CL;
             }
-            ncl = n;
+            ncl = std::min(n, sm_count * ctas_env / CL);
         }
         occ->ncl[v8_cl_index(CL)] = ncl;
         return 0;

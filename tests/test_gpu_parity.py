@@ -394,3 +394,42 @@ def test_autotune_picks_a_path_and_stays_exact(wd, logn, batch):
     y = gpu_fwd(wd, plan, x)
     assert np.array_equal(y, oracle.ntt_forward(x, primes)), (mode, logn)
     assert np.array_equal(gpu_inv(wd, plan, y), x), (mode, logn)
+
+
+# -------------------------------------------------------------- tc4: the warp-specialised 4-step tcgen05 kernel
+# (rows a3, a5, a9; forward; the inverse of a tc4 plan runs on the CUDA-core kernels).  Every row against the
+# oracle: few rows (fewer CTAs than SMs), several rows per CTA with limbs changing inside a CTA's range (the
+# stage matrices are reloaded), primes across the accepted range, edge inputs, in place.
+@pytest.mark.parametrize("L,batch", [(1, 1), (3, 2), (5, 67), (36, 8), (7, 41)])
+def test_tc4_forward_vs_oracle(wd, L, batch):
+    n = 1 << 16
+    primes = P[:L]
+    x = inputs.uniform_residues(primes, n, batch, 8000 + 7 * L + batch)
+    plan = wd.Plan(n, primes, mode="tc4")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (L, batch)
+    assert np.array_equal(gpu_inv(wd, plan, y), x)
+
+
+def test_tc4_prime_sizes_and_edges(wd):
+    n = 1 << 16
+    primes = [786433, 269221889, 537133057, 805961729, P[0]]
+    plan = wd.Plan(n, primes, mode="tc4")
+    for kind in ("zeros", "qm1", "alt", "delta", "mono1", "gauss"):
+        x = np.repeat(inputs.structured(kind, primes, n, seed=3), 3, axis=0)
+        assert np.array_equal(gpu_fwd(wd, plan, x), oracle.ntt_forward(x, primes)), kind
+    x = inputs.uniform_residues(primes, n, 9, 8100)
+    assert np.array_equal(gpu_fwd(wd, plan, x), oracle.ntt_forward(x, primes))
+
+
+def test_tc4_in_place_and_full_config3(wd):
+    n, L, batch = 1 << 16, 36, 128
+    primes = P[:L]
+    x = inputs.uniform_residues(primes, n, batch, inputs.SEED_BASE + 2)
+    plan = wd.Plan(n, primes, mode="tc4")
+    d = to_dev(x)
+    plan.forward(d, d)                                  # in place over the whole config-3 batch
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(d), oracle.ntt_forward(x, primes))
+    with pytest.raises(wd.WdNttError):
+        wd.Plan(1 << 15, P[:2], mode="tc4")             # N = 2^16 only
