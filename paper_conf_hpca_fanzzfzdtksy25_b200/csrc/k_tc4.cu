@@ -155,6 +155,11 @@ unsigned long long* g_trace = nullptr;     // diagnostics (wd_tc4_set_trace)
 
 }  // namespace
 
+bool tma_encode_u32(CUtensorMap* m, const void* base, uint32_t rank, const cuuint64_t* dims, const cuuint64_t* strides,
+                    const cuuint32_t* box, CUtensorMapSwizzle sw) {
+    return encode(m, base, rank, dims, strides, box, sw);
+}
+
 void tc4_set_trace(void* p) { g_trace = static_cast<unsigned long long*>(p); }
 
 void free_tc4_tables(Tc4Tables& t) {

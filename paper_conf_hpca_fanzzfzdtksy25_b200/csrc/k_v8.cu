@@ -2,6 +2,7 @@
 // WD-CUDA (row f2).  Kernels in ntt_v8.cuh.
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
 #include "launch.h"
 #include "ntt_v8.cuh"
 
@@ -19,6 +20,8 @@ int set_smem(K kern, int bytes) {
 
 template <int LOGN, int CL>
 constexpr bool cl_ok() { return (1 << (LOGN - 12)) % CL == 0; }
+template <int LOGN>
+constexpr bool tm_ok() { return LOGN >= 13 && LOGN <= 16; }   // the TMA column phase: 2 <= 2^A <= 16
 
 template <int LOGN, int CL>
 int prep_cl(int sm_count, V8Occ* occ) {
@@ -27,6 +30,10 @@ int prep_cl(int sm_count, V8Occ* occ) {
     } else {
         int e = set_smem(ntt_v8<LOGN, true, false, CL>, V8_SMEM) | set_smem(ntt_v8<LOGN, false, false, CL>, V8_SMEM) |
                 set_smem(ntt_v8<LOGN, false, true, CL>, V8_SMEM);
+        if constexpr (tm_ok<LOGN>())
+            e |= set_smem(ntt_v8<LOGN, true, false, CL, 0, 1>, V8_SMEM_TM) |
+                 set_smem(ntt_v8<LOGN, false, false, CL, 0, 1>, V8_SMEM_TM) |
+                 set_smem(ntt_v8<LOGN, false, false, CL, 0, 2>, V8_SMEM_TM);
         if (CL == (LOGN > 12 ? 2 : 1))
             e |= set_smem(ntt_v8<LOGN, true, false, CL, 1>, V8_SMEM) | set_smem(ntt_v8<LOGN, true, false, CL, 2>, V8_SMEM);
         if (e) return e;
@@ -59,42 +66,66 @@ int prep_logn(int sm_count, V8Occ* occ) {
            prep_cl<LOGN, 8>(sm_count, occ);
 }
 
+// the column-phase input as a 2-D tensor: inner dimension the 4096 columns, outer one line per
+// (physical row, k); box = one column pass (256 columns x 2^A lines)
+// (forward: the input rows; inverse: the output rows, which hold the intermediate)
+bool encode_v8_cols(CUtensorMap* m, uint32_t logN, const uint32_t* base, uint32_t ls, uint32_t L, uint32_t rows) {
+    const uint32_t R = 1u << (logN - 12);
+    const uint64_t phys = ls ? (uint64_t)(rows / L - 1) * ls + L : rows;
+    const cuuint64_t dims[2] = {V8_SUBW, phys * R}, strides[1] = {V8_SUBW * 4};
+    const cuuint32_t box[2] = {V8_T, R};
+    return tma_encode_u32(m, base, 2, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_NONE);
+}
+
 template <int LOGN, int CL, int EPI>
-void launch_k(bool fwd, const NttArgs& a, uint32_t rows, int ncl, cudaStream_t s) {
+void launch_k(bool fwd, const NttArgs& a, uint32_t rows, int ncl, int tma, cudaStream_t s) {
     if constexpr (!cl_ok<LOGN, CL>()) {
         return;
     } else {
         auto k = fwd ? ntt_v8<LOGN, true, false, CL, EPI> : (a.in2 ? ntt_v8<LOGN, false, true, CL> : ntt_v8<LOGN, false, false, CL>);
+        alignas(64) CUtensorMap tm;
+        std::memset(&tm, 0, sizeof(tm));
+        int smem = V8_SMEM;
+        if constexpr (tm_ok<LOGN>() && EPI == 0) {
+            if ((tma & 1) && fwd && encode_v8_cols(&tm, LOGN, a.in, a.in_ls, a.L, rows)) {
+                k = ntt_v8<LOGN, true, false, CL, 0, 1>; smem = V8_SMEM_TM;
+            } else if ((tma & 2) && !fwd && !a.in2 && encode_v8_cols(&tm, LOGN, a.out, a.out_ls, a.L, rows)) {
+                k = ntt_v8<LOGN, false, false, CL, 0, 1>; smem = V8_SMEM_TM;
+            } else if ((tma & 4) && !fwd && !a.in2) {
+                k = ntt_v8<LOGN, false, false, CL, 0, 2>;
+            }
+        }
         const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)ncl) * CL;
         if constexpr (CL == 1) {
-            k<<<grid, V8_T, V8_SMEM, s>>>(a, rows);
+            k<<<grid, V8_T, smem, s>>>(a, rows, tm);
         } else {
             cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3(grid); cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM; cfg.stream = s;
+            cfg.gridDim = dim3(grid); cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = smem; cfg.stream = s;
             cudaLaunchAttribute at[1];
             at[0].id = cudaLaunchAttributeClusterDimension;
             at[0].val.clusterDim.x = CL; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = 1;
             cfg.attrs = at; cfg.numAttrs = 1;
-            cudaLaunchKernelEx(&cfg, k, a, rows);
+            cudaLaunchKernelEx(&cfg, k, a, rows, tm);
         }
     }
 }
 
 template <int LOGN>
-void launch_logn(bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ, cudaStream_t s) {
+void launch_logn(bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ, int tma,
+                 cudaStream_t s) {
     const int n = occ.ncl[v8_cl_index(cl)];
     if (epi) {                           // the RNS store maps exist at the default cluster size only
         constexpr int CD = LOGN > 12 ? 2 : 1;
         const int nd = occ.ncl[v8_cl_index(CD)];
-        if (epi == 1) launch_k<LOGN, CD, 1>(true, a, rows, nd, s);
-        else launch_k<LOGN, CD, 2>(true, a, rows, nd, s);
+        if (epi == 1) launch_k<LOGN, CD, 1>(true, a, rows, nd, 0, s);
+        else launch_k<LOGN, CD, 2>(true, a, rows, nd, 0, s);
         return;
     }
     switch (cl) {
-        case 8: launch_k<LOGN, 8, 0>(fwd, a, rows, n, s); break;
-        case 4: launch_k<LOGN, 4, 0>(fwd, a, rows, n, s); break;
-        case 2: launch_k<LOGN, 2, 0>(fwd, a, rows, n, s); break;
-        default: launch_k<LOGN, 1, 0>(fwd, a, rows, n, s); break;
+        case 8: launch_k<LOGN, 8, 0>(fwd, a, rows, n, tma, s); break;
+        case 4: launch_k<LOGN, 4, 0>(fwd, a, rows, n, tma, s); break;
+        case 2: launch_k<LOGN, 2, 0>(fwd, a, rows, n, tma, s); break;
+        default: launch_k<LOGN, 1, 0>(fwd, a, rows, n, tma, s); break;
     }
 }
 
@@ -112,17 +143,17 @@ int prep_v8(uint32_t logN, int sm_count, V8Occ* occ) {
     }
 }
 
-void launch_v8(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ,
+void launch_v8(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ, int tma,
                cudaStream_t s) {
     const int maxcl = 1 << std::min<int>(3, (int)logN - 12);
     cl = std::max(1, std::min(cl, maxcl));
     switch (logN) {
-        case 12: launch_logn<12>(fwd, a, rows, cl, epi, occ, s); break;
-        case 13: launch_logn<13>(fwd, a, rows, cl, epi, occ, s); break;
-        case 14: launch_logn<14>(fwd, a, rows, cl, epi, occ, s); break;
-        case 15: launch_logn<15>(fwd, a, rows, cl, epi, occ, s); break;
-        case 16: launch_logn<16>(fwd, a, rows, cl, epi, occ, s); break;
-        default: launch_logn<17>(fwd, a, rows, cl, epi, occ, s); break;
+        case 12: launch_logn<12>(fwd, a, rows, cl, epi, occ, tma, s); break;
+        case 13: launch_logn<13>(fwd, a, rows, cl, epi, occ, tma, s); break;
+        case 14: launch_logn<14>(fwd, a, rows, cl, epi, occ, tma, s); break;
+        case 15: launch_logn<15>(fwd, a, rows, cl, epi, occ, tma, s); break;
+        case 16: launch_logn<16>(fwd, a, rows, cl, epi, occ, tma, s); break;
+        default: launch_logn<17>(fwd, a, rows, cl, epi, occ, tma, s); break;
     }
 }
 

@@ -2,6 +2,7 @@
 // Every function here only configures and enqueues kernels on the given stream: no allocation, no
 // synchronisation, no environment reads (those happen once, at plan creation).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <vector>
@@ -20,7 +21,10 @@ void launch_v5(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int sm_
 struct V8Occ { int ncl[4] = {0, 0, 0, 0}; };   // resident clusters per GPU for CL = 1, 2, 4, 8
 int prep_v8(uint32_t logN, int sm_count, V8Occ* occ);
 // cl in {1, 2, 4, 8}; epi: 0 plain, 1 RESCALE store map, 2 ModDown store map (forward only)
-void launch_v8(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ,
+// tma (N = 2^13..2^16, epi = 0; ignored otherwise), bits: 1 = forward column phase fed by TMA,
+// 2 = inverse column phase fed by TMA, 4 = inverse: next row's first sub-row requested during the
+// column phase (register-fed)
+void launch_v8(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int cl, int epi, const V8Occ& occ, int tma,
                cudaStream_t s);
 int prep_wdcuda();
 void launch_wdcuda(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, cudaStream_t s);
@@ -30,6 +34,11 @@ int prep_tensor();
 int launch_tensor(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, cudaStream_t s);
 int launch_fused(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, float share,
                  cudaStream_t s);
+
+// ---- k_tc4.cu: tensor-map encoding (cuTensorMapEncodeTiled through the runtime's driver entry
+//      point), u32 elements, no interleave, 256-B L2 promotion; false if unavailable or rejected
+bool tma_encode_u32(CUtensorMap* m, const void* base, uint32_t rank, const cuuint64_t* dims,
+                    const cuuint64_t* strides, const cuuint32_t* box, CUtensorMapSwizzle sw);
 
 // ---- k_tc4.cu: the warp-specialised 4-step tcgen05 kernel (N = 2^16, ntt_tc4.cuh)
 struct Tc4Tables {

@@ -25,12 +25,14 @@
 #pragma once
 #include "common.cuh"
 #include "ntt_cuda_core.cuh"
+#include "tma.cuh"
 
 namespace wd {
 
 constexpr int V8_T = 256;                    // threads per CTA (4 CTAs per SM at 64 registers)
 constexpr int V8_SUBW = 4096;                // words per phase-2 sub-row
 constexpr int V8_SMEM = 2 * V8_SUBW * 4;     // two sub-row buffers = 32 KB
+constexpr int V8_SMEM_TM = V8_SMEM + 64;     // + the TMA column phase's mbarriers
 
 __device__ __forceinline__ int v8_phys(int a, int b, int c) {
     return a * 256 + ((b ^ (a & 1)) << 4) + (c ^ (((b >> 1) & 3) << 2));
@@ -101,8 +103,16 @@ __device__ __forceinline__ uint32_t rs_out(uint32_t aval, uint32_t y, const uint
 
 // EPI (forward only): 0 = plain NTT; 1 = RESCALE (shared last-limb input row through rs_in, output
 // through rs_out against aux); 2 = ModDown (plain input rows, output through rs_out against aux)
-template <int LOGN, bool FWD, bool PW, int CL = 1, int EPI = 0>
-__global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows) {
+// TM (EPI = 0, no pointwise product, 2 <= 2^A <= 16): the column phase is fed by TMA instead of
+// register loads.  Each column pass (256 columns x 2^A lines = 2^A KB, one 2-D box of tm_in) lands in
+// one of the two sub-row buffers and the next pass is in flight while a pass computes; threads read
+// their column with conflict-free LDS.  Forward: tm_in maps the input, and the first pass of the CTA's
+// next row is issued during the last sub-row of the current one, so the HBM latency of the column
+// loads is no longer exposed.  Inverse: tm_in maps the output slot (the L2-resident intermediate,
+// made visible to the async proxy by fence.proxy.async.global before the cluster barrier), and the
+// last pass starts the cp.async of the next row's first sub-row.
+template <int LOGN, bool FWD, bool PW, int CL = 1, int EPI = 0, int TM = 0>
+__global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, const __grid_constant__ CUtensorMap tm_in) {
     constexpr int A = LOGN - 12;             // phase-1 layers (radix 2^A columns)
     constexpr int R = 1 << A;                // column length = number of sub-rows
     static_assert(A >= 0 && A <= 5, "N = 2^12 .. 2^17");
@@ -111,18 +121,42 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows) {
     constexpr int NS = R / CL;               // phase-2 sub-rows per CTA
     const int rank = CL > 1 ? (int)(blockIdx.x % CL) : 0;
     const int p0 = rank * NP, s0 = rank * NS, s1 = s0 + NS;
-    extern __shared__ __align__(16) uint32_t smem[];
+    extern __shared__ __align__(1024) uint32_t smem[];
     const int t = threadIdx.x;
     const int hi4 = t >> 4, lo4 = t & 15;
 
     const uint32_t nb = rows / a.L;              // polynomials in the launch
+    static_assert(TM != 1 || (EPI == 0 && !PW && A >= 1 && R <= 16), "TMA column phase: EPI 0, no PW, 2 <= R <= 16");
+    static_assert(TM != 2 || (!FWD && EPI == 0 && A >= 1), "early sub-row prefetch: inverse with a column phase");
+    constexpr int PF = ((NS - 1) & 1) ^ 1;       // TM: the buffer free during a row's last sub-row
+    // TM: one mbarrier per buffer, after the two buffers (dynamic shared memory V8_SMEM_TM; a static
+    // __shared__ would shift the dynamic buffers off the alignment TMA needs)
+    uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + 2 * V8_SUBW);
+    uint32_t tph = 0;                            // TM: parity of each buffer's next completion
+    auto map_row = [&](uint32_t sr) {            // limb-major schedule (below)
+        const uint32_t lb = a.limb_major ? sr / nb : sr % a.L;
+        return a.limb_major ? (sr - lb * nb) * a.L + lb : sr;
+    };
+    if constexpr (TM == 1) {
+        if (t == 0) {
+            mb_init(&tbar[0], 1); mb_init(&tbar[1], 1);
+            mb_init_fence();
+            const uint32_t sr = blockIdx.x / CL;
+            if (FWD && sr < rows) {              // the CTA's first column pass
+                mb_expect(&tbar[PF], R * V8_T * 4);
+                tma2_load(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R), &tbar[PF]);
+            }
+        }
+        __syncthreads();
+    }
+    bool sub0_ready = false;                     // TM inverse: this row's first sub-row already requested
 #pragma unroll 1
     for (uint32_t srow = blockIdx.x / CL; srow < rows; srow += gridDim.x / CL) {
         // limb-major schedule (a.limb_major): the rows in flight at any time share a few limbs,
         // so their twiddle tables (N x 8 bytes per limb and direction) stay a small part of L2
         // next to the L2-resident intermediates; the data layout is unchanged
         const uint32_t limb = a.limb_major ? srow / nb : srow % a.L;
-        const uint32_t row = a.limb_major ? (srow - limb * nb) * a.L + limb : srow;
+        const uint32_t row = map_row(srow);
         const LimbConst lc = a.lc[limb];
         // the last inverse layer's constants: with the pointwise product (PW, Montgomery, which
         // leaves a factor 2^-32) they carry an extra 2^32 (N^-1 * 2^32, wn * 2^32)
@@ -146,10 +180,26 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows) {
                 for (int pass = p0; pass < p0 + NP; ++pass) {
                     const int c = pass * V8_T + t;
                     uint32_t x[R];
+                    if constexpr (TM == 1) {
+                        const int b = (pass - p0 + PF) & 1;
+                        if (t == 0 && pass + 1 < p0 + NP) {   // the next pass into the other buffer
+                            fence_proxy_async();
+                            mb_expect(&tbar[b ^ 1], R * V8_T * 4);
+                            tma2_load(smem + (b ^ 1) * V8_SUBW, &tm_in, (pass + 1) * V8_T,
+                                      (int)(row_map(row, a.L, a.in_ls) * R), &tbar[b ^ 1]);
+                        }
+                        mb_wait(&tbar[b], (tph >> b) & 1);
+                        tph ^= 1u << b;
+                        const uint32_t* B = smem + b * V8_SUBW;
 #pragma unroll
-                    for (int k = 0; k < R; ++k) {
-                        if constexpr (EPI == 1) x[k] = rs_in(__ldg(in + k * V8_SUBW + c), a.rs_thr, rsc, q);
-                        else x[k] = __ldcs(in + k * V8_SUBW + c);
+                        for (int k = 0; k < R; ++k) x[k] = B[k * V8_T + t];
+                        __syncthreads();                      // buffer b read by every thread
+                    } else {
+#pragma unroll
+                        for (int k = 0; k < R; ++k) {
+                            if constexpr (EPI == 1) x[k] = rs_in(__ldg(in + k * V8_SUBW + c), a.rs_thr, rsc, q);
+                            else x[k] = __ldcs(in + k * V8_SUBW + c);
+                        }
                     }
                     fwd_radix<A>(x, tw, 0, 0, q, q2);
 #pragma unroll
@@ -180,7 +230,17 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows) {
                     for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
                 }
                 __syncthreads();                         // stage 1 done everywhere; sub-row s-1 fully consumed
-                if (s + 1 < s1) v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
+                if (s + 1 < s1) {
+                    v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
+                } else if constexpr (TM == 1) {               // the next row's first column pass
+                    const uint32_t sr = srow + gridDim.x / CL;
+                    if (t == 0 && sr < rows) {
+                        fence_proxy_async();
+                        mb_expect(&tbar[PF], R * V8_T * 4);
+                        tma2_load(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R),
+                                  &tbar[PF]);
+                    }
+                }
                 uint2 w3[15];
                 load_tw16(w3, tw, A + 8, st * 256 + t);  // stage-3 twiddles, in flight
                 {   // stage 2: layers A+4..A+7, thread (a, c), elements b (stride 16)
@@ -235,7 +295,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows) {
         } else {
             // ---- phase 2': layers A+11..A on sub-rows s (input in bit-reversed order) ----
             const uint32_t* in2 = a.in2 + ((size_t)row << LOGN);
-            v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+            if (!sub0_ready) v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+            sub0_ready = false;
 #pragma unroll 1
             for (int s = s0; s < s1; ++s) {
                 uint32_t* S = smem + ((s - s0) & 1) * V8_SUBW;
@@ -311,14 +372,53 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows) {
             }
             // ---- phase 1': layers A-1..0 on columns, N^-1 folded into layer 0 ----
             if constexpr (A > 0) {
+                if constexpr (TM == 1) fence_proxy_async_global();   // the intermediate is read back by TMA
                 if constexpr (CL > 1) cluster_sync();    // the whole intermediate is written
                 else __syncthreads();
+                const int orow = (int)(row_map(row, a.L, a.out_ls) * R);
+                if constexpr (TM == 2) {                 // the register-fed column phase leaves both buffers
+                    const uint32_t sr = srow + gridDim.x / CL;     // idle: next row's first sub-row now
+                    if (sr < rows) {
+                        v8_load_inv_slice(smem, a.in + ((size_t)row_map(map_row(sr), a.L, a.in_ls) << LOGN) + s0 * V8_SUBW);
+                        sub0_ready = true;
+                    }
+                }
+                if constexpr (TM == 1) {
+                    if (t == 0) {
+                        mb_expect(&tbar[0], R * V8_T * 4);
+                        tma2_load(smem, &tm_in, p0 * V8_T, orow, &tbar[0]);
+                    }
+                }
 #pragma unroll 1
                 for (int pass = p0; pass < p0 + NP; ++pass) {
                     const int c = pass * V8_T + t;
                     uint32_t x[R];
+                    if constexpr (TM == 1) {
+                        const int b = (pass - p0) & 1;
+                        if (t == 0 && pass + 1 < p0 + NP) {   // the next pass into the other buffer
+                            fence_proxy_async();
+                            mb_expect(&tbar[b ^ 1], R * V8_T * 4);
+                            tma2_load(smem + (b ^ 1) * V8_SUBW, &tm_in, (pass + 1) * V8_T, orow, &tbar[b ^ 1]);
+                        }
+                        mb_wait(&tbar[b], (tph >> b) & 1);
+                        tph ^= 1u << b;
+                        const uint32_t* B = smem + b * V8_SUBW;
 #pragma unroll
-                    for (int k = 0; k < R; ++k) x[k] = __ldcs(out + k * V8_SUBW + c);
+                        for (int k = 0; k < R; ++k) x[k] = B[k * V8_T + t];
+                        __syncthreads();                      // buffer b read by every thread
+                        static_assert((NP & 1) == 0, "the last pass reads buffer 1: buffer 0 is free");
+                        if (pass + 1 == p0 + NP) {            // the next row's first sub-row into buffer 0
+                            const uint32_t sr = srow + gridDim.x / CL;
+                            if (sr < rows) {
+                                v8_load_inv_slice(smem, a.in + ((size_t)row_map(map_row(sr), a.L, a.in_ls) << LOGN) +
+                                                            s0 * V8_SUBW);
+                                sub0_ready = true;
+                            }
+                        }
+                    } else {
+#pragma unroll
+                        for (int k = 0; k < R; ++k) x[k] = __ldcs(out + k * V8_SUBW + c);
+                    }
                     inv_radix<A, true>(x, tw, 0, 0, lcl);
 #pragma unroll
                     for (int k = 0; k < R; ++k) __stcs(out + k * V8_SUBW + c, canon2(x[k], q));

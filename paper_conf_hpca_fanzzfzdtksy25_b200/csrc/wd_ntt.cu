@@ -44,6 +44,7 @@ struct wd_ntt_plan {
     int kernel_ver = 0;
     int v8_cl = 0;
     uint32_t limb_major = 1;
+    int v8_tma = 5;               // v8 column-phase feed (launch.h launch_v8; WD_NTT_V8_TMA)
     V8Occ occ;                     // v8 resident clusters per CL (grid sizing without per-launch queries)
     std::vector<uint32_t> primes, psi;
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
@@ -135,13 +136,13 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
         // between half and one SM count of rows: 4-CTA clusters (config 5 sweep)
         else if (logN >= 15 && rows <= sm) cl = 4;
     }
-    launch_v8(logN, fwd, a, rows, cl, 0, p->occ, s);
+    launch_v8(logN, fwd, a, rows, cl, 0, p->occ, p->v8_tma, s);
     return 1;
 }
 
 // v8 with a RESCALE / ModDown store map (EPI 1 / 2) or a plain v8 launch at the default cluster size
 void launch_v8_default(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, int epi, cudaStream_t s) {
-    launch_v8(p->logN, fwd, a, rows, p->logN > 12 ? 2 : 1, epi, p->occ, s);
+    launch_v8(p->logN, fwd, a, rows, p->logN > 12 ? 2 : 1, epi, p->occ, p->v8_tma, s);
 }
 
 int effective_mode(const wd_ntt_plan* p) { return p->mode == WD_MODE_AUTO ? WD_MODE_CUDA : p->mode; }
@@ -405,6 +406,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     }
     if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 8 ? 8 : atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
     if (const char* ev = getenv("WD_NTT_LM")) p->limb_major = atoi(ev) != 0;
+    if (const char* ev = getenv("WD_NTT_V8_TMA")) p->v8_tma = atoi(ev) & 7;
     const size_t tb = sizeof(uint2) * (size_t)L * N;
     if (cudaMalloc(&p->d_fwd, tb) != cudaSuccess || cudaMalloc(&p->d_inv, tb) != cudaSuccess ||
         cudaMalloc(&p->d_lc, sizeof(LimbConst) * L) != cudaSuccess) {

@@ -308,6 +308,30 @@ def test_v8_cluster_sizes_many_rows(wd, cl, logn, batch, monkeypatch):
     assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (cl, logn)
 
 
+# v8's column-phase feeds (WD_NTT_V8_TMA, read at plan creation; default 5): 0 register loads, 1 TMA
+# forward, 2 TMA inverse, 4 inverse next-row sub-row prefetch; every cluster size, more rows than
+# resident clusters (so the cross-row prefetches run), in place, and a ModUp-style strided section
+@pytest.mark.parametrize("feed", ["0", "1", "2", "4", "7"])
+@pytest.mark.parametrize("logn,cl", [(13, "2"), (14, "1"), (14, "4"), (15, "8"), (16, "2"), (16, "1")])
+def test_v8_column_feeds(wd, feed, logn, cl, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", "v8")
+    monkeypatch.setenv("WD_NTT_CL", cl)
+    monkeypatch.setenv("WD_NTT_V8_TMA", feed)
+    n = 1 << logn
+    primes = [P[2], P[9], P[44]]
+    batch = 600 if logn <= 14 else 211
+    x = inputs.uniform_residues(primes, n, batch, 5300 + logn)
+    plan = wd.Plan(n, primes, mode="cuda")
+    y = gpu_fwd(wd, plan, x)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (feed, logn, cl)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (feed, logn, cl)
+    t = to_dev(x)
+    plan.forward(t, t)                                   # in place
+    plan.inverse(t, t)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(t), x), (feed, logn, cl)
+
+
 # Primes across the range the ABI accepts (the lazy bounds [0, 4q) < 2^32 hold for any q < 2^30).
 # 786433 = 3 * 2^18 + 1; the others are the first primes = 1 (mod 2^17) above 2^28, 2^29, 1.5*2^29.
 @pytest.mark.parametrize("mode", ["cuda", "tensor", "fused", "cuda_gemm"])
