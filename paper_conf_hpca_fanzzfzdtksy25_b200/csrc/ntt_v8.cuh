@@ -144,7 +144,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
             const uint32_t sr = blockIdx.x / CL;
             if (FWD && sr < rows) {              // the CTA's first column pass
                 mb_expect(&tbar[PF], R * V8_T * 4);
-                tma2_load(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R), &tbar[PF]);
+                tma2_load_hint(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R), &tbar[PF],
+                               l2_evict_first_policy());
             }
         }
         __syncthreads();
@@ -185,8 +186,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                         if (t == 0 && pass + 1 < p0 + NP) {   // the next pass into the other buffer
                             fence_proxy_async();
                             mb_expect(&tbar[b ^ 1], R * V8_T * 4);
-                            tma2_load(smem + (b ^ 1) * V8_SUBW, &tm_in, (pass + 1) * V8_T,
-                                      (int)(row_map(row, a.L, a.in_ls) * R), &tbar[b ^ 1]);
+                            tma2_load_hint(smem + (b ^ 1) * V8_SUBW, &tm_in, (pass + 1) * V8_T,
+                                           (int)(row_map(row, a.L, a.in_ls) * R), &tbar[b ^ 1], l2_evict_first_policy());
                         }
                         mb_wait(&tbar[b], (tph >> b) & 1);
                         tph ^= 1u << b;
@@ -237,8 +238,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                     if (t == 0 && sr < rows) {
                         fence_proxy_async();
                         mb_expect(&tbar[PF], R * V8_T * 4);
-                        tma2_load(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R),
-                                  &tbar[PF]);
+                        tma2_load_hint(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R),
+                                       &tbar[PF], l2_evict_first_policy());
                     }
                 }
                 uint2 w3[15];
@@ -386,7 +387,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                 if constexpr (TM == 1) {
                     if (t == 0) {
                         mb_expect(&tbar[0], R * V8_T * 4);
-                        tma2_load(smem, &tm_in, p0 * V8_T, orow, &tbar[0]);
+                        tma2_load_hint(smem, &tm_in, p0 * V8_T, orow, &tbar[0], l2_evict_first_policy());
                     }
                 }
 #pragma unroll 1
@@ -398,7 +399,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                         if (t == 0 && pass + 1 < p0 + NP) {   // the next pass into the other buffer
                             fence_proxy_async();
                             mb_expect(&tbar[b ^ 1], R * V8_T * 4);
-                            tma2_load(smem + (b ^ 1) * V8_SUBW, &tm_in, (pass + 1) * V8_T, orow, &tbar[b ^ 1]);
+                            tma2_load_hint(smem + (b ^ 1) * V8_SUBW, &tm_in, (pass + 1) * V8_T, orow, &tbar[b ^ 1], l2_evict_first_policy());
                         }
                         mb_wait(&tbar[b], (tph >> b) & 1);
                         tph ^= 1u << b;

@@ -29,5 +29,17 @@ __device__ __forceinline__ void tma2_load(void* dst, const CUtensorMap* m, int c
                  " [%0], [%1, {%2, %3}], [%4];"
                  :: "r"(smem_u32(dst)), "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(b)) : "memory");
 }
-
+// an L2 policy that marks the lines a load brings in as first to evict (streamed, read-once input):
+// keeps them from displacing the L2-resident intermediates (the register loads they replace were
+// ld.global.cs)
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ void tma2_load_hint(void* dst, const CUtensorMap* m, int c0, int c1, uint64_t* b, uint64_t pol) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                 " [%0], [%1, {%2, %3}], [%4], %5;"
+                 :: "r"(smem_u32(dst)), "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(b)), "l"(pol) : "memory");
+}
 }  // namespace wd
