@@ -28,21 +28,21 @@ int prep_cl(int sm_count, V8Occ* occ) {
     if constexpr (!cl_ok<LOGN, CL>()) {
         return 0;
     } else {
-        int e = set_smem(ntt_v8<LOGN, true, false, CL>, V8_SMEM) | set_smem(ntt_v8<LOGN, false, false, CL>, V8_SMEM) |
-                set_smem(ntt_v8<LOGN, false, true, CL>, V8_SMEM);
+        int e = set_smem(ntt_v8<LOGN, true, false, CL>, V8_SMEM_K) | set_smem(ntt_v8<LOGN, false, false, CL>, V8_SMEM_K) |
+                set_smem(ntt_v8<LOGN, false, true, CL>, V8_SMEM_K);
         if constexpr (tm_ok<LOGN>())
-            e |= set_smem(ntt_v8<LOGN, true, false, CL, 0, 1>, V8_SMEM_TM) |
-                 set_smem(ntt_v8<LOGN, false, false, CL, 0, 1>, V8_SMEM_TM) |
-                 set_smem(ntt_v8<LOGN, false, false, CL, 0, 2>, V8_SMEM_TM);
+            e |= set_smem(ntt_v8<LOGN, true, false, CL, 0, 1>, V8_SMEM_K) |
+                 set_smem(ntt_v8<LOGN, false, false, CL, 0, 1>, V8_SMEM_K) |
+                 set_smem(ntt_v8<LOGN, false, false, CL, 0, 2>, V8_SMEM_K);
         if (CL == (LOGN > 12 ? 2 : 1))
-            e |= set_smem(ntt_v8<LOGN, true, false, CL, 1>, V8_SMEM) | set_smem(ntt_v8<LOGN, true, false, CL, 2>, V8_SMEM);
+            e |= set_smem(ntt_v8<LOGN, true, false, CL, 1>, V8_SMEM_K) | set_smem(ntt_v8<LOGN, true, false, CL, 2>, V8_SMEM_K);
         if (e) return e;
         // WD_NTT_V8_CTAS (A/B runs, read once per plan): CTAs per SM the persistent grid is sized for
         static const int ctas_env = getenv("WD_NTT_V8_CTAS") ? std::max(1, std::min(4, atoi(getenv("WD_NTT_V8_CTAS")))) : 4;
         int ncl = sm_count * ctas_env / CL;
         if (CL > 1) {                    // resident clusters, queried once per plan (not per launch)
             cudaLaunchConfig_t cfg = {};
-            cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM;
+            cfg.blockDim = dim3(V8_T); cfg.dynamicSmemBytes = V8_SMEM_K;
             cfg.gridDim = dim3(sm_count * 4 / CL * CL);
             cudaLaunchAttribute at[1];
             at[0].id = cudaLaunchAttributeClusterDimension;
@@ -85,12 +85,12 @@ void launch_k(bool fwd, const NttArgs& a, uint32_t rows, int ncl, int tma, cudaS
         auto k = fwd ? ntt_v8<LOGN, true, false, CL, EPI> : (a.in2 ? ntt_v8<LOGN, false, true, CL> : ntt_v8<LOGN, false, false, CL>);
         alignas(64) CUtensorMap tm;
         std::memset(&tm, 0, sizeof(tm));
-        int smem = V8_SMEM;
+        const int smem = V8_SMEM_K;
         if constexpr (tm_ok<LOGN>() && EPI == 0) {
             if ((tma & 1) && fwd && encode_v8_cols(&tm, LOGN, a.in, a.in_ls, a.L, rows)) {
-                k = ntt_v8<LOGN, true, false, CL, 0, 1>; smem = V8_SMEM_TM;
+                k = ntt_v8<LOGN, true, false, CL, 0, 1>;
             } else if ((tma & 2) && !fwd && !a.in2 && encode_v8_cols(&tm, LOGN, a.out, a.out_ls, a.L, rows)) {
-                k = ntt_v8<LOGN, false, false, CL, 0, 1>; smem = V8_SMEM_TM;
+                k = ntt_v8<LOGN, false, false, CL, 0, 1>;
             } else if ((tma & 4) && !fwd && !a.in2) {
                 k = ntt_v8<LOGN, false, false, CL, 0, 2>;
             }

@@ -32,7 +32,117 @@ namespace wd {
 constexpr int V8_T = 256;                    // threads per CTA (4 CTAs per SM at 64 registers)
 constexpr int V8_SUBW = 4096;                // words per phase-2 sub-row
 constexpr int V8_SMEM = 2 * V8_SUBW * 4;     // two sub-row buffers = 32 KB
-constexpr int V8_SMEM_TM = V8_SMEM + 64;     // + the TMA column phase's mbarriers
+// The radix-16 twiddles of row stages 1 and 2 (1 + 16 groups x 15 per sub-row) are staged in shared
+// memory by cp.async together with the sub-row they belong to (one sub-row ahead), instead of being
+// __ldg'd right before use: with the 228 KB carveout L1 is small and those loads were L2 round trips
+// on the critical path (config 3: forward 1.097 -> 1.062 ms, inverse 1.086 -> 1.037 ms)
+constexpr int V8_TWW = 768;                  // words per buffer's twiddle area (<= 384 pairs)
+constexpr int V8_TWOFF = 2 * V8_SUBW + 16;   // its word offset: after the buffers and the mbarriers
+// the v8 kernel's dynamic shared memory: two sub-row buffers, the TMA column phase's mbarriers (64 B)
+// and two twiddle areas
+constexpr int V8_SMEM_K = V8_SMEM + 64 + 2 * V8_TWW * 4;
+
+__device__ __forceinline__ void cp_async8(void* smem_dst, const void* gsrc) {
+    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" :: "r"(d), "l"(gsrc) : "memory");
+}
+// forward, sub-row s: every warp copies the stage-1 runs (group s, layers A..A+3: 1, 2, 4, 8 pairs at
+// 0, 2, 4, 8) into its own 16 pairs at TW + 16w (read before the CTA barrier, after the warp's own
+// cp.async wait), and threads 0..239 copy the stage-2 runs (groups 16s..16s+15, layers A+4..A+7:
+// 16, 32, 64, 128 pairs at 128 + 0, 16, 48, 112; read after the barrier).  No commit (the caller's
+// slice load commits the group).
+template <int A>
+__device__ __forceinline__ void v8_tw_fwd(uint2* TW, const uint2* __restrict__ tw, uint32_t s) {
+    const int t = threadIdx.x, w = t >> 5, l = t & 31;
+    if (l < 15) {
+        const int k = 31 - __clz(l + 1), g = l - ((1 << k) - 1);
+        cp_async8(TW + 16 * w + (k ? (1 << k) : 0) + g, tw + (1u << (A + k)) + (s << k) + g);
+    }
+    if (t < 240) {
+        const int k = 31 - __clz((t >> 4) + 1), g = t - 16 * ((1 << k) - 1);
+        cp_async8(TW + 128 + 16 * ((1 << k) - 1) + g, tw + (16u << (A + k)) + ((s * 16) << k) + g);
+    }
+}
+// inverse, sub-row s: every warp copies the stage-2' runs of its two groups 16s + 2w, 16s + 2w + 1
+// (2, 4, 8, 16 pairs at TW + 32w + 0, 2, 6, 14; read before the barrier), threads 0..14 the stage-1'
+// runs of group s (at 256 + 0, 2, 4, 8; read after it)
+template <int A>
+__device__ __forceinline__ void v8_tw_inv(uint2* TW, const uint2* __restrict__ tw, uint32_t s) {
+    const int t = threadIdx.x, w = t >> 5, l = t & 31;
+    if (l < 30) {
+        const int k = 31 - __clz((l >> 1) + 1), g = l - 2 * ((1 << k) - 1);
+        cp_async8(TW + 32 * w + 2 * ((1 << k) - 1) + g, tw + (16u << (A + k)) + ((s * 16 + 2 * w) << k) + g);
+    }
+    if (t < 15) {
+        const int k = 31 - __clz(t + 1), g = t - ((1 << k) - 1);
+        cp_async8(TW + 256 + (k ? (1 << k) : 0) + g, tw + (1u << (A + k)) + (s << k) + g);
+    }
+}
+__device__ __forceinline__ uint2 lo2(uint4 v) { return make_uint2(v.x, v.y); }
+__device__ __forceinline__ uint2 hi2(uint4 v) { return make_uint2(v.z, v.w); }
+// radix-16 blocks whose layer-t twiddle of group g is p_t[g] (shared memory; p1..p3 16-byte aligned),
+// the same butterfly network as fwd16_tw / inv16_tw
+__device__ __forceinline__ void fwd16_sp(uint32_t* x, const uint2* p0, const uint2* p1, const uint2* p2,
+                                         const uint2* p3, uint32_t q, uint32_t q2) {
+    {
+        const uint2 w = *p0;
+#pragma unroll
+        for (int r = 0; r < 8; ++r) ct_bfly(x[r], x[r + 8], w, q, q2);
+    }
+    {
+        const uint4 v = *reinterpret_cast<const uint4*>(p1);
+#pragma unroll
+        for (int r = 0; r < 4; ++r) { ct_bfly(x[r], x[r + 4], lo2(v), q, q2); ct_bfly(x[8 + r], x[12 + r], hi2(v), q, q2); }
+    }
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const uint4 v = reinterpret_cast<const uint4*>(p2)[k];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            ct_bfly(x[8 * k + r], x[8 * k + r + 2], lo2(v), q, q2);
+            ct_bfly(x[8 * k + 4 + r], x[8 * k + 6 + r], hi2(v), q, q2);
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const uint4 v = reinterpret_cast<const uint4*>(p3)[k];
+        ct_bfly(x[4 * k], x[4 * k + 1], lo2(v), q, q2);
+        ct_bfly(x[4 * k + 2], x[4 * k + 3], hi2(v), q, q2);
+    }
+}
+template <bool LAST>
+__device__ __forceinline__ void inv16_sp(uint32_t* x, const uint2* p0, const uint2* p1, const uint2* p2,
+                                         const uint2* p3, const LimbConst& c) {
+    const uint32_t q = c.q, q2 = c.q2;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const uint4 v = reinterpret_cast<const uint4*>(p3)[k];
+        gs_bfly(x[4 * k], x[4 * k + 1], lo2(v), q, q2);
+        gs_bfly(x[4 * k + 2], x[4 * k + 3], hi2(v), q, q2);
+    }
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const uint4 v = reinterpret_cast<const uint4*>(p2)[k];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            gs_bfly(x[8 * k + r], x[8 * k + r + 2], lo2(v), q, q2);
+            gs_bfly(x[8 * k + 4 + r], x[8 * k + 6 + r], hi2(v), q, q2);
+        }
+    }
+    {
+        const uint4 v = *reinterpret_cast<const uint4*>(p1);
+#pragma unroll
+        for (int r = 0; r < 4; ++r) { gs_bfly(x[r], x[r + 4], lo2(v), q, q2); gs_bfly(x[8 + r], x[12 + r], hi2(v), q, q2); }
+    }
+    if constexpr (LAST) {
+#pragma unroll
+        for (int r = 0; r < 8; ++r) gs_bfly_last(x[r], x[r + 8], c);
+    } else {
+        const uint2 w = *p0;
+#pragma unroll
+        for (int r = 0; r < 8; ++r) gs_bfly(x[r], x[r + 8], w, q, q2);
+    }
+}
 
 __device__ __forceinline__ int v8_phys(int a, int b, int c) {
     return a * 256 + ((b ^ (a & 1)) << 4) + (c ^ (((b >> 1) & 3) << 2));
@@ -129,9 +239,10 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
     static_assert(TM != 1 || (EPI == 0 && !PW && A >= 1 && R <= 16), "TMA column phase: EPI 0, no PW, 2 <= R <= 16");
     static_assert(TM != 2 || (!FWD && EPI == 0 && A >= 1), "early sub-row prefetch: inverse with a column phase");
     constexpr int PF = ((NS - 1) & 1) ^ 1;       // TM: the buffer free during a row's last sub-row
-    // TM: one mbarrier per buffer, after the two buffers (dynamic shared memory V8_SMEM_TM; a static
+    // TM: one mbarrier per buffer, after the two buffers (dynamic shared memory V8_SMEM_K; a static
     // __shared__ would shift the dynamic buffers off the alignment TMA needs)
     uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + 2 * V8_SUBW);
+    auto TWB = [&](int b) { return reinterpret_cast<uint2*>(smem + V8_TWOFF + b * V8_TWW); };
     uint32_t tph = 0;                            // TM: parity of each buffer's next completion
     auto map_row = [&](uint32_t sr) {            // limb-major schedule (below)
         const uint32_t lb = a.limb_major ? sr / nb : sr % a.L;
@@ -211,6 +322,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
             }
             // ---- phase 2: layers A..A+11 on sub-rows s ----
             const uint32_t* src = A > 0 ? out : in;
+            v8_tw_fwd<A>(TWB(0), tw, s0);
             v8_load_fwd_slice(smem, src + s0 * V8_SUBW);
 #pragma unroll 1
             for (int s = s0; s < s1; ++s) {
@@ -226,12 +338,14 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                         x[i] = S[v8_phys(i, b, c)];
                         if constexpr (EPI == 1 && A == 0) x[i] = rs_in(x[i], a.rs_thr, rsc, q);
                     }
-                    fwd_radix<4>(x, tw, A, st, q, q2);
+                    const uint2* W = TWB((s - s0) & 1) + 16 * (t >> 5);
+                    fwd16_sp(x, W, W + 2, W + 4, W + 8, q, q2);
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(i, b, c)] = x[i];
                 }
                 __syncthreads();                         // stage 1 done everywhere; sub-row s-1 fully consumed
                 if (s + 1 < s1) {
+                    v8_tw_fwd<A>(TWB((s + 1 - s0) & 1), tw, s + 1);
                     v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
                 } else if constexpr (TM == 1) {               // the next row's first column pass
                     const uint32_t sr = srow + gridDim.x / CL;
@@ -248,7 +362,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                     const int aa = hi4, c = lo4;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
-                    fwd_radix<4>(x, tw, A + 4, st * 16 + aa, q, q2);
+                    const uint2* T2 = TWB((s - s0) & 1) + 128;
+                    fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, q, q2);
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
                 }
@@ -296,7 +411,10 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
         } else {
             // ---- phase 2': layers A+11..A on sub-rows s (input in bit-reversed order) ----
             const uint32_t* in2 = a.in2 + ((size_t)row << LOGN);
-            if (!sub0_ready) v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+            if (!sub0_ready) {
+                v8_tw_inv<A>(TWB(0), tw, s0);
+                v8_load_inv_slice(smem, in + s0 * V8_SUBW);
+            }
             sub0_ready = false;
 #pragma unroll 1
             for (int s = s0; s < s1; ++s) {
@@ -352,17 +470,22 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                     const int aa = hi4, c = lo4;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
-                    inv_radix<4, false>(x, tw, A + 4, (uint32_t)s * 16 + aa, lc);
+                    const uint2* W = TWB((s - s0) & 1) + 32 * (t >> 5) + (aa & 1);
+                    inv16_sp<false>(x, W, W + 2 + (aa & 1), W + 6 + 3 * (aa & 1), W + 14 + 7 * (aa & 1), lc);
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
                 }
                 __syncthreads();                         // stage 2' done everywhere; sub-row s-1 fully consumed
-                if (s + 1 < s1) v8_load_inv_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, in + (s + 1) * V8_SUBW);
+                if (s + 1 < s1) {
+                    v8_tw_inv<A>(TWB((s + 1 - s0) & 1), tw, s + 1);
+                    v8_load_inv_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, in + (s + 1) * V8_SUBW);
+                }
                 {   // stage 1': layers A+3..A, thread (b, c), elements a -> global (coalesced)
                     const int b = hi4, c = lo4;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, b, c)];
-                    inv_radix<4, A == 0>(x, tw, A, (uint32_t)s, lcl);
+                    const uint2* T1 = TWB((s - s0) & 1) + 256;
+                    inv16_sp<A == 0>(x, T1, T1 + 2, T1 + 4, T1 + 8, lcl);
                     uint32_t* o = out + s * V8_SUBW + b * 16 + c;
 #pragma unroll
                     for (int i = 0; i < 16; ++i) {
@@ -380,6 +503,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                 if constexpr (TM == 2) {                 // the register-fed column phase leaves both buffers
                     const uint32_t sr = srow + gridDim.x / CL;     // idle: next row's first sub-row now
                     if (sr < rows) {
+                        const uint32_t nl = a.limb_major ? sr / nb : sr % a.L;
+                        v8_tw_inv<A>(TWB(0), a.tw + ((size_t)nl << LOGN), s0);
                         v8_load_inv_slice(smem, a.in + ((size_t)row_map(map_row(sr), a.L, a.in_ls) << LOGN) + s0 * V8_SUBW);
                         sub0_ready = true;
                     }
@@ -411,6 +536,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                         if (pass + 1 == p0 + NP) {            // the next row's first sub-row into buffer 0
                             const uint32_t sr = srow + gridDim.x / CL;
                             if (sr < rows) {
+                                const uint32_t nl = a.limb_major ? sr / nb : sr % a.L;
+                                v8_tw_inv<A>(TWB(0), a.tw + ((size_t)nl << LOGN), s0);
                                 v8_load_inv_slice(smem, a.in + ((size_t)row_map(map_row(sr), a.L, a.in_ls) << LOGN) +
                                                             s0 * V8_SUBW);
                                 sub0_ready = true;
