@@ -231,7 +231,8 @@ int wd_ntt_plan_get_mode(const wd_ntt_plan* plan);
  * scratch data (allocated and freed inside the call, zero residues) for every execution path
  * available at this N -- WD_MODE_CUDA, and for N = 2^16 also WD_MODE_FUSED (phase-split
  * pipeline and row splits with tensor_share 0.25 / 0.5 / 0.75), WD_MODE_TENSOR,
- * WD_MODE_CUDA_GEMM and WD_MODE_FTC (at the plan's FTC share) -- with CUDA events on `stream`, and sets the plan to the fastest.
+ * WD_MODE_CUDA_GEMM, WD_MODE_FTC (at the plan's FTC share) and WD_MODE_TC4 -- with CUDA events on
+ * `stream`, and sets the plan to the fastest (building the tensor tables of N = 2^16 first).
  * Writes that path's milliseconds per forward + inverse to *best_ms if best_ms != NULL.
  * Synchronises `stream`.  Returns WD_OK, WD_EINVAL (NULL plan, batch == 0, wrong device) or
  * WD_ECUDA (allocation or launch failure; the plan's mode is then unchanged).  The candidates

@@ -2,16 +2,20 @@
 //
 // The paper's WD-FUSE idea (Fig. 3: tensor-core and CUDA-core work of different
 // tiles at the same time on one SM; Alg. 2: inner DFTs as u8 GEMMs with the
-// twiddles in the matrices) re-derived for sm_100a.  One persistent CTA per SM, 11 warps:
-//   warp 0  TMA producer: input tiles HBM/L2 -> shared memory (cp.async.bulk.tensor), the limb's
-//           stage matrices (cp.async.bulk)
-//   warp 1  MMA issuer (one thread): tcgen05.mma.cta_group::1.kind::i8, accumulators in TMEM,
-//           completion by tcgen05.commit -> mbarrier; owns the TMEM allocation (512 columns)
+// twiddles in the matrices) re-derived for sm_100a.  One persistent CTA per SM, 20 warps (<= 96
+// registers each):
+//   warp 0  producers: lane 0 streams the input / intermediate tiles HBM/L2 -> shared memory
+//           (cp.async.bulk.tensor, mbarrier complete_tx), lane 1 the per-group stage matrices
+//           (cp.async.bulk) one tile ahead of their MMA
+//   warps 1, 3  MMA issuers (one thread each, even / odd tiles): tcgen05.mma.cta_group::1.kind::i8,
+//           accumulators in TMEM, completion by tcgen05.commit -> mbarrier; warp 1 owns the TMEM
+//           allocation (512 columns)
 //   warp 2  TMA store issuer: shared-memory staging tiles -> global (cp.async.bulk.tensor store)
-//   warps 3..10  CUDA-core workers (two per TMEM lane quarter): operand transposition, the
-//           accumulator epilogues (byte-plane recombination, Shoup fold), the 4-step twist
-// The units overlap through rings (4 input slots, 4 A-operand slots, 4 TMEM accumulators, 2
-// staging slots): the tensor pipe runs tile t+1..t+3 while the workers finish tile t.
+//   warps 4..19  CUDA-core workers, two groups of 8 (in a group, two warps per TMEM lane quarter,
+//           one per output half): operand transposition, the accumulator epilogues (byte-plane
+//           recombination, Shoup fold), the 4-step twist
+// The units overlap through rings (8 input slots, 4 A-operand slots, 4 TMEM accumulators, 6 staging
+// slots, 8 matrix slots): the tensor pipe runs the next tiles while the workers finish tile t.
 //
 // Decomposition (reading C-1 negacyclic, C-3 bit-reversed output).  Row x[j],
 // j = 256 j1 + j2.  With psi of order 2N, zeta = psi^256, omega = psi^512:

@@ -714,7 +714,8 @@ int wd_ntt_plan_autotune(wd_ntt_plan* p, uint32_t batch, wd_stream_t st, float* 
     if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) return set_err(WD_EINVAL);
     if ((uint64_t)batch * p->L > 0x7fffffffull) return set_err(WD_EINVAL);
     if (p->logN == 16) {
-        const int e = ensure_tensor_tables(p);
+        int e = ensure_tensor_tables(p);
+        if (e == WD_OK) e = ensure_tc4_tables(p);
         if (e != WD_OK) return set_err(e);
     }
     cudaStream_t s = (cudaStream_t)st;
@@ -740,6 +741,7 @@ int wd_ntt_plan_autotune(wd_ntt_plan* p, uint32_t batch, wd_stream_t st, float* 
         cands.push_back({WD_MODE_CUDA_GEMM, p->tensor_share});
         cands.push_back({WD_MODE_FTC, p->tensor_share});
     }
+    if (p->logN == 16 && p->t4.ok) cands.push_back({WD_MODE_TC4, p->tensor_share});
     int best = -1;
     float best_t = 0.0f;
     for (size_t i = 0; i < cands.size(); ++i) {

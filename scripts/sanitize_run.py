@@ -1,6 +1,6 @@
 """Drive every launch path of libwdntt.so once on small shapes, for compute-sanitizer
 (memcheck / racecheck / synccheck).  Usage: python scripts/sanitize_run.py [group ...]
-Groups: v8 cc cl small tensor fused ftc gemm tc4 rns host.  Each group prints one line; the round trip
+Groups: v8 v8feeds cc cl small tensor fused ftc gemm tc4 rns host.  Each group prints one line; the round trip
 is checked (INTT(NTT(x)) == x) so a wrong result under the sanitizer is visible too."""
 import os
 import sys
@@ -30,6 +30,18 @@ def group_v8():
         p = wdntt.Plan(1 << logn, pr)
         rt(p, 1 << logn, pr, batch)
         p.close()
+
+
+def group_v8feeds():
+    # every v8 column feed (WD_NTT_V8_TMA is read at plan creation) and cluster size at N = 2^14, 2^16
+    for feed in ("0", "1", "2", "4", "7"):
+        for logn, cl, batch in ((16, "2", 30), (16, "1", 30), (14, "4", 300)):
+            os.environ["WD_NTT_V8_TMA"], os.environ["WD_NTT_CL"] = feed, cl
+            pr = inputs.bench_primes(2)
+            p = wdntt.Plan(1 << logn, pr)
+            rt(p, 1 << logn, pr, batch)
+            p.close()
+    os.environ.pop("WD_NTT_V8_TMA"); os.environ.pop("WD_NTT_CL")
 
 
 def group_cc():
