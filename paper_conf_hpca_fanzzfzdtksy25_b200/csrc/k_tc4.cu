@@ -30,29 +30,6 @@ struct Pow {
     uint32_t operator()(uint64_t e) const { return pw[e % pw.size()]; }
 };
 
-// inverse of a 16x16 matrix mod q (Gauss-Jordan); false if singular
-bool mat_inv(const uint32_t M[16][16], uint32_t R[16][16], uint32_t q) {
-    uint64_t A[16][32];
-    for (int i = 0; i < 16; ++i)
-        for (int j = 0; j < 32; ++j) A[i][j] = j < 16 ? M[i][j] : (j - 16 == i ? 1 : 0);
-    for (int c = 0; c < 16; ++c) {
-        int piv = -1;
-        for (int r = c; r < 16; ++r) if (A[r][c]) { piv = r; break; }
-        if (piv < 0) return false;
-        if (piv != c) for (int j = 0; j < 32; ++j) std::swap(A[piv][j], A[c][j]);
-        const uint64_t inv = pm_pow((uint32_t)A[c][c], q - 2, q);
-        for (int j = 0; j < 32; ++j) A[c][j] = A[c][j] * inv % q;
-        for (int r = 0; r < 16; ++r) {
-            if (r == c || !A[r][c]) continue;
-            const uint64_t f = A[r][c];
-            for (int j = 0; j < 32; ++j) A[r][j] = (A[r][j] + (q - f) * A[c][j]) % q;
-        }
-    }
-    for (int i = 0; i < 16; ++i)
-        for (int j = 0; j < 16; ++j) R[i][j] = (uint32_t)A[i][16 + j];
-    return true;
-}
-
 // the forward stage matrices of one limb (tc4 header):
 //   MA[c][a] = psi^(4096 a (2c+1)); MB_c[d][b] = psi^(256 b (2c+1+32d)); MC[g][f] = psi^(8192 g f);
 //   MD_g[h'][e] = psi^(512 e (g + 16 brv4(h')))

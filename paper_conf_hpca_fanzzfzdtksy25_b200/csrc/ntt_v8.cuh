@@ -27,6 +27,10 @@
 #include "ntt_cuda_core.cuh"
 #include "tma.cuh"
 
+// the v8 kernels declare their dynamic shared memory 1024-byte aligned (TMA destinations); the
+// kernels of ntt_cuda_core.cuh declare the same extern array with 16 (same storage, harmless)
+#pragma nv_diag_suppress 1886
+
 namespace wd {
 
 constexpr int V8_T = 256;                    // threads per CTA (4 CTAs per SM at 64 registers)
