@@ -234,15 +234,7 @@ int launch_tc4(bool fwd, const NttArgs& a, const Tc4Tables& t, uint32_t rows, in
     ta.trace = g_trace;
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
     tc4::ntt_tc4_fwd<<<grid, tc4::NT, tc4::SMEM, s>>>(mx, mc, mi, mo, ta);
-    const cudaError_t e = cudaPeekAtLastError();
-    if (e != cudaSuccess) {
-        cudaFuncAttributes fa;
-        cudaFuncGetAttributes(&fa, tc4::ntt_tc4_fwd);
-        fprintf(stderr, "wdntt: tc4 launch failed: %s (regs %d, maxThreads %d, smem %u, localBytes %zu)\n",
-                cudaGetErrorString(e), fa.numRegs, fa.maxThreadsPerBlock, tc4::SMEM, fa.localSizeBytes);
-        return -2;
-    }
-    return 1;
+    return cudaPeekAtLastError() == cudaSuccess ? 1 : -2;   // the caller reports WD_ECUDA
 }
 
 }  // namespace wd

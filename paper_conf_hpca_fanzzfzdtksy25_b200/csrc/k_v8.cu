@@ -37,7 +37,8 @@ int prep_cl(int sm_count, V8Occ* occ) {
         if (CL == (LOGN > 12 ? 2 : 1))
             e |= set_smem(ntt_v8<LOGN, true, false, CL, 1>, V8_SMEM_K) | set_smem(ntt_v8<LOGN, true, false, CL, 2>, V8_SMEM_K);
         if (e) return e;
-        // WD_NTT_V8_CTAS (A/B runs, read once per plan): CTAs per SM the persistent grid is sized for
+        // WD_NTT_V8_CTAS (A/B runs; read once per process, at the first plan): CTAs per SM the
+        // persistent grid is sized for
         static const int ctas_env = getenv("WD_NTT_V8_CTAS") ? std::max(1, std::min(4, atoi(getenv("WD_NTT_V8_CTAS")))) : 4;
         int ncl = sm_count * ctas_env / CL;
         if (CL > 1) {                    // resident clusters, queried once per plan (not per launch)

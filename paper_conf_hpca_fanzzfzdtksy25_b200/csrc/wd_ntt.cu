@@ -44,7 +44,7 @@ struct wd_ntt_plan {
     int kernel_ver = 0;
     int v8_cl = 0;
     uint32_t limb_major = 1;
-    int v8_tma = 5;               // v8 column-phase feed (launch.h launch_v8; WD_NTT_V8_TMA)
+    int v8_tma = 1;               // v8 column-phase feed (launch.h launch_v8; WD_NTT_V8_TMA)
     V8Occ occ;                     // v8 resident clusters per CL (grid sizing without per-launch queries)
     std::vector<uint32_t> primes, psi;
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)

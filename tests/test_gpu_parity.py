@@ -308,7 +308,7 @@ def test_v8_cluster_sizes_many_rows(wd, cl, logn, batch, monkeypatch):
     assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (cl, logn)
 
 
-# v8's column-phase feeds (WD_NTT_V8_TMA, read at plan creation; default 5): 0 register loads, 1 TMA
+# v8's column-phase feeds (WD_NTT_V8_TMA, read at plan creation; default 1): 0 register loads, 1 TMA
 # forward, 2 TMA inverse, 4 inverse next-row sub-row prefetch; every cluster size, more rows than
 # resident clusters (so the cross-row prefetches run), in place, and a ModUp-style strided section
 @pytest.mark.parametrize("feed", ["0", "1", "2", "4", "7"])
