@@ -1,0 +1,36 @@
+// k_tmr.cu -- launcher of the TMEM-resident CUDA-core NTT "tm" (N = 2^16; kernels in ntt_tmr.cuh,
+// DESIGN.md 5.1a).
+#include <algorithm>
+#include <cstring>
+#include "launch.h"
+#include "ntt_tmr.cuh"
+
+namespace wd {
+
+int prep_tmr() {
+    for (auto k : {tmr::ntt_tmr16<true>, tmr::ntt_tmr16<false>}) {
+        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, tmr::SMEM) != cudaSuccess ||
+            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+            return 4;
+    }
+    return 0;
+}
+
+// plain transforms only (contiguous [batch][L][N] rows, no pointwise product / store maps / copies);
+// returns launches (1), -1 if the arguments need v8, -2 if the tensor map cannot be encoded
+int launch_tmr(bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
+    if (a.in2 || a.aux || a.cpy || a.in_ls || a.out_ls || rows % a.L) return -1;
+    alignas(64) CUtensorMap tm;
+    std::memset(&tm, 0, sizeof(tm));
+    if (fwd) {   // the column passes: inner dimension the 4096 columns, one line per (row, k); box 256 x 16
+        const cuuint64_t dims[2] = {tmr::SUBW, (cuuint64_t)rows * 16}, strides[1] = {tmr::SUBW * 4};
+        const cuuint32_t box[2] = {tmr::TT, 16};
+        if (!tma_encode_u32(&tm, a.in, 2, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_NONE)) return -2;
+    }
+    const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
+    if (fwd) tmr::ntt_tmr16<true><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows, tm);
+    else tmr::ntt_tmr16<false><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows, tm);
+    return 1;
+}
+
+}  // namespace wd

@@ -1,0 +1,406 @@
+// ntt_tmr.cuh -- "tm": the TMEM-resident CUDA-core NTT, N = 2^16.
+//
+// Same butterfly network and decomposition as v8 (ntt_v8.cuh: N = 16 x 4096, layers 0..3 on the 4096
+// columns of 16 elements, layers 4..15 as three radix-16 register stages on the 16 contiguous 4096-word
+// sub-rows; merged-psi CT, PAPER.md:85-91 with reading C-1), but the phase-1 <-> phase-2 intermediate
+// never leaves the SM: a whole row (2^16 words = 256 KB) sits in the SM's tensor memory (TMEM, 128
+// lanes x 512 columns x 32 bit), which the CUDA-core NTT otherwise leaves idle.  v8 keeps it in the
+// row's output slot in L2 instead, with a 2-CTA cluster per row and a cluster barrier between the
+// phases; here there is no L2 round trip, no cluster and no excess DRAM traffic.
+//
+// One persistent CTA per SM (1024 threads = 4 teams of 256).  Team tau owns sub-rows / column passes
+// s = tau, tau+4, tau+8, tau+12 of every row.  Team thread t (warp w = t/32, h = t/128) uses TMEM lane
+// t % 128 -- its own warp's lane quadrant (w % 4) -- and half h of the lane's columns:
+//   column pass p, thread t: column c = 256 p + t, elements k = 0..15 (x[k*4096 + c])
+//   sub-row s, stage 1, thread t: elements a*256 + t of sub-row s, a = 0..15, i.e. (k = s, c = 256 a + t)
+// so stage 1 of sub-row s reads exactly what column pass a = 0..15 of the same thread index t wrote:
+// TMEM cell (lane t % 128, column col(p, k, h)).  Two layouts alternate from row to row,
+//   A: col(p, k, h) = 32 k + 16 h + p          B: col(p, k, h) = 32 p + 16 h + k,
+// so that the 32 cells sub-row s of row j has consumed are exactly the cells column pass s of row j+1
+// writes, by the same thread (forward; the inverse mirrors it).  A team therefore interleaves
+//   forward:  R(j, s) C(j+1, s)  for its four s, then one CTA barrier per row,
+//   inverse:  C'(j, s) R'(j+1, s) for its four s, then one CTA barrier per row,
+// with the column pass of the next row overwriting the sub-row just consumed -- the classic in-place
+// ping-pong.  In each row one of the two accesses is 16 contiguous columns (one tcgen05.ld/st .x16),
+// the other 16 strided ones (.x1).
+// Forward column passes are fed by TMA (one 256 x 16 box per pass, issued one pass ahead); inverse
+// sub-rows by 16-byte cp.async, double-buffered as in v8; forward outputs leave by coalesced 512-byte
+// STG from the sub-row buffer, inverse outputs straight from registers (128-byte lines per warp).
+#pragma once
+#include "ntt_v8.cuh"
+
+namespace wd {
+namespace tmr {
+
+constexpr int TEAMS = 4, TT = 256, NT = TEAMS * TT;
+constexpr int SUBW = 4096;
+constexpr int TWW = 768;                        // words per twiddle area (<= 384 (w, w') pairs)
+constexpr int TEAM_W = 2 * SUBW + 2 * TWW;      // per team: two sub-row buffers, two twiddle areas
+constexpr int SMEM = TEAMS * TEAM_W * 4 + 64;   // + one TMA mbarrier per team + the TMEM base slot
+
+// ---------------------------------------------------------------- tensor memory
+__device__ __forceinline__ void tfence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tfence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tm_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+// 16 consecutive columns of the warp's lanes -> x[0..15]; complete on return (wait::ld in the same asm,
+// so no use of x can be scheduled before it)
+__device__ __forceinline__ void tm_ld16(uint32_t ta, uint32_t* x) {
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+                 "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n\t"
+                 "tcgen05.wait::ld.sync.aligned;"
+                 : "=r"(x[0]), "=r"(x[1]), "=r"(x[2]), "=r"(x[3]), "=r"(x[4]), "=r"(x[5]), "=r"(x[6]), "=r"(x[7]),
+                   "=r"(x[8]), "=r"(x[9]), "=r"(x[10]), "=r"(x[11]), "=r"(x[12]), "=r"(x[13]), "=r"(x[14]), "=r"(x[15])
+                 : "r"(ta) : "memory");
+}
+// columns ta, ta + 32, ..., ta + 480 -> x[0..15]
+__device__ __forceinline__ void tm_ld16s(uint32_t ta, uint32_t* x) {
+    asm volatile("{\n\t.reg .b32 a;\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%16];\n\t"
+                 "add.u32 a, %16, 32;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%1}, [a];\n\t"
+                 "add.u32 a, %16, 64;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%2}, [a];\n\t"
+                 "add.u32 a, %16, 96;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%3}, [a];\n\t"
+                 "add.u32 a, %16, 128;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%4}, [a];\n\t"
+                 "add.u32 a, %16, 160;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%5}, [a];\n\t"
+                 "add.u32 a, %16, 192;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%6}, [a];\n\t"
+                 "add.u32 a, %16, 224;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%7}, [a];\n\t"
+                 "add.u32 a, %16, 256;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%8}, [a];\n\t"
+                 "add.u32 a, %16, 288;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%9}, [a];\n\t"
+                 "add.u32 a, %16, 320;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%10}, [a];\n\t"
+                 "add.u32 a, %16, 352;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%11}, [a];\n\t"
+                 "add.u32 a, %16, 384;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%12}, [a];\n\t"
+                 "add.u32 a, %16, 416;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%13}, [a];\n\t"
+                 "add.u32 a, %16, 448;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%14}, [a];\n\t"
+                 "add.u32 a, %16, 480;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%15}, [a];\n\t"
+                 "tcgen05.wait::ld.sync.aligned;\n\t}"
+                 : "=r"(x[0]), "=r"(x[1]), "=r"(x[2]), "=r"(x[3]), "=r"(x[4]), "=r"(x[5]), "=r"(x[6]), "=r"(x[7]),
+                   "=r"(x[8]), "=r"(x[9]), "=r"(x[10]), "=r"(x[11]), "=r"(x[12]), "=r"(x[13]), "=r"(x[14]), "=r"(x[15])
+                 : "r"(ta) : "memory");
+}
+__device__ __forceinline__ void tm_st16(uint32_t ta, const uint32_t* x) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+                 "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};"
+                 :: "r"(ta), "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7]),
+                    "r"(x[8]), "r"(x[9]), "r"(x[10]), "r"(x[11]), "r"(x[12]), "r"(x[13]), "r"(x[14]), "r"(x[15])
+                 : "memory");
+}
+__device__ __forceinline__ void tm_st16s(uint32_t ta, const uint32_t* x) {
+    asm volatile("{\n\t.reg .b32 a;\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};\n\t"
+                 "add.u32 a, %0, 32;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%2};\n\t"
+                 "add.u32 a, %0, 64;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%3};\n\t"
+                 "add.u32 a, %0, 96;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%4};\n\t"
+                 "add.u32 a, %0, 128;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%5};\n\t"
+                 "add.u32 a, %0, 160;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%6};\n\t"
+                 "add.u32 a, %0, 192;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%7};\n\t"
+                 "add.u32 a, %0, 224;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%8};\n\t"
+                 "add.u32 a, %0, 256;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%9};\n\t"
+                 "add.u32 a, %0, 288;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%10};\n\t"
+                 "add.u32 a, %0, 320;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%11};\n\t"
+                 "add.u32 a, %0, 352;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%12};\n\t"
+                 "add.u32 a, %0, 384;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%13};\n\t"
+                 "add.u32 a, %0, 416;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%14};\n\t"
+                 "add.u32 a, %0, 448;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%15};\n\t"
+                 "add.u32 a, %0, 480;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%16};\n\t}"
+                 :: "r"(ta), "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7]),
+                    "r"(x[8]), "r"(x[9]), "r"(x[10]), "r"(x[11]), "r"(x[12]), "r"(x[13]), "r"(x[14]), "r"(x[15])
+                 : "memory");
+}
+
+__device__ __forceinline__ void team_bar(int team) {
+    asm volatile("bar.sync %0, %1;" :: "r"(team + 1), "n"(TT) : "memory");
+}
+// every TMEM store of this thread done and ordered before the CTA barrier; TMEM reads after it ordered
+// after it (PTX tcgen05 memory-consistency rules)
+__device__ __forceinline__ void cta_sync_tmem() {
+    tm_wait_st();
+    tfence_before();
+    __syncthreads();
+    tfence_after();
+}
+
+// twiddles of one sub-row, staged by cp.async (team thread t; no commit): v8_tw_fwd / v8_tw_inv with
+// the team-local thread index
+template <int A>
+__device__ __forceinline__ void tw_fwd(uint2* TW, const uint2* __restrict__ tw, uint32_t s, int t) {
+    const int w = t >> 5, l = t & 31;
+    if (l < 15) {
+        const int k = 31 - __clz(l + 1), g = l - ((1 << k) - 1);
+        cp_async8(TW + 16 * w + (k ? (1 << k) : 0) + g, tw + (1u << (A + k)) + (s << k) + g);
+    }
+    if (t < 240) {
+        const int k = 31 - __clz((t >> 4) + 1), g = t - 16 * ((1 << k) - 1);
+        cp_async8(TW + 128 + 16 * ((1 << k) - 1) + g, tw + (16u << (A + k)) + ((s * 16) << k) + g);
+    }
+}
+template <int A>
+__device__ __forceinline__ void tw_inv(uint2* TW, const uint2* __restrict__ tw, uint32_t s, int t) {
+    const int w = t >> 5, l = t & 31;
+    if (l < 30) {
+        const int k = 31 - __clz((l >> 1) + 1), g = l - 2 * ((1 << k) - 1);
+        cp_async8(TW + 32 * w + 2 * ((1 << k) - 1) + g, tw + (16u << (A + k)) + ((s * 16 + 2 * w) << k) + g);
+    }
+    if (t < 15) {
+        const int k = 31 - __clz(t + 1), g = t - ((1 << k) - 1);
+        cp_async8(TW + 256 + (k ? (1 << k) : 0) + g, tw + (1u << (A + k)) + (s << k) + g);
+    }
+}
+// inverse sub-row slice (stage 3' reads of warp w: words 512w .. 512w+511), no commit
+__device__ __forceinline__ void load_inv_slice(uint32_t* S, const uint32_t* src, int t) {
+    const int w = t >> 5, l = t & 31;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const int e = 512 * w + 4 * (32 * k + l);
+        cp_async16(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15), src + e);
+    }
+}
+
+template <bool FWD>
+__global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, const __grid_constant__ CUtensorMap tm_in) {
+    constexpr int LOGN = 16, A = 4;
+    extern __shared__ __align__(1024) uint32_t smem[];
+    const int team = (int)(threadIdx.x >> 8), t = (int)(threadIdx.x & (TT - 1));
+    const int w = t >> 5, h = w >> 2, hi4 = t >> 4, lo4 = t & 15;
+    uint32_t* TS = smem + team * TEAM_W;
+    uint32_t* const B0 = TS;                     // forward: sub-row exchange; inverse: input buffer 0
+    uint32_t* const B1 = TS + SUBW;              // forward: TMA column staging; inverse: input buffer 1
+    auto TWB = [&](int b) { return reinterpret_cast<uint2*>(TS + 2 * SUBW + b * TWW); };
+    uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + team;
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(smem + TEAMS * TEAM_W + 2 * TEAMS);
+
+    if (threadIdx.x < 32) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" :: "r"(smem_u32(tslot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    if (t == 0) { mb_init(tbar, 1); mb_init_fence(); }
+    tfence_before();
+    __syncthreads();
+    tfence_after();
+    // this thread's TMEM lane (its warp's quadrant) and column half
+    const uint32_t tl = *tslot + ((uint32_t)(32 * (w & 3)) << 16) + 16u * h;
+
+    const uint32_t G = gridDim.x;
+    const uint32_t nrow = rows > blockIdx.x ? (rows - blockIdx.x + G - 1) / G : 0;
+    const uint32_t nb = rows / a.L;
+    // limb-major schedule as in v8: the CTA's j-th row is schedule slot blockIdx.x + j G
+    auto limb_of = [&](uint32_t j) {
+        const uint32_t sr = blockIdx.x + j * G;
+        return a.limb_major ? sr / nb : sr % a.L;
+    };
+    auto row_of = [&](uint32_t j) {
+        const uint32_t sr = blockIdx.x + j * G;
+        if (!a.limb_major) return sr;
+        const uint32_t lb = sr / nb;
+        return (sr - lb * nb) * a.L + lb;
+    };
+
+    if (nrow > 0) {
+        if constexpr (FWD) {
+            uint32_t tph = 0;
+            auto issue_col = [&](uint32_t j, int s) {   // team thread 0: column pass s of row j -> B1
+                fence_proxy_async();
+                mb_expect(tbar, 16 * TT * 4);
+                tma2_load_hint(B1, &tm_in, s * TT, (int)(row_of(j) * 16), tbar, l2_evict_first_policy());
+            };
+            // column pass s of row j: layers 0..3, into TMEM (layout j & 1)
+            auto colpass = [&](uint32_t j, int s) {
+                const uint32_t limb = limb_of(j);
+                const LimbConst lc = a.lc[limb];
+                const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+                mb_wait(tbar, tph);
+                tph ^= 1;
+                uint32_t x[16];
+#pragma unroll
+                for (int k = 0; k < 16; ++k) x[k] = B1[k * TT + t];
+                team_bar(team);                          // staging read by the whole team
+                if (t == 0) {                            // the team's next column pass
+                    if (s + TEAMS < 16) issue_col(j, s + TEAMS);
+                    else if (j + 1 < nrow) issue_col(j + 1, team);
+                }
+                fwd_radix<A>(x, tw, 0, 0, lc.q, lc.q2);
+                if (j & 1) tm_st16(tl + 32 * s, x);      // B: 32 s + 16 h + k
+                else tm_st16s(tl + s, x);                // A: 32 k + 16 h + s
+            };
+            // sub-row s of row j: layers 4..15 (stage 1 from TMEM), canonical output
+            auto rowpass = [&](uint32_t j, int s, uint32_t u) {
+                const uint32_t limb = limb_of(j), row = row_of(j);
+                const LimbConst lc = a.lc[limb];
+                const uint32_t q = lc.q, q2 = lc.q2;
+                const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+                uint32_t* out = a.out + ((size_t)row << LOGN) + s * SUBW;
+                uint32_t* S = B0;
+                cp_async_wait<0>();
+                __syncwarp();                            // this warp's stage-1 twiddles landed
+                uint32_t x[16];
+                if (j & 1) tm_ld16s(tl + s, x);          // B: element 256 a + t at 32 a + 16 h + s
+                else tm_ld16(tl + 32 * s, x);            // A: 32 s + 16 h + a
+                {   // stage 1: layers 4..7, thread (b, c), elements a
+                    const uint2* W = TWB(u & 1) + 16 * w;
+                    fwd16_sp(x, W, W + 2, W + 4, W + 8, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(i, hi4, lo4)] = x[i];
+                }
+                team_bar(team);                          // stage 1 done team-wide
+                {   // the team's next sub-row's twiddles
+                    uint32_t nj = j, ns = (uint32_t)s + TEAMS;
+                    if (ns >= 16) { nj = j + 1; ns = team; }
+                    if (nj < nrow) tw_fwd<A>(TWB((u + 1) & 1), a.tw + ((size_t)limb_of(nj) << LOGN), ns, t);
+                    cp_async_commit();
+                }
+                uint2 w3[15];
+                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                {   // stage 2: layers 8..11, thread (a, c), elements b
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    const uint2* T2 = TWB(u & 1) + 128;
+                    fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, q, q2);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                __syncwarp();
+                {   // stage 3: layers 12..15, thread (a, b), 16 contiguous elements; coalesced store
+                    const int aa = hi4, b = lo4;
+                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
+                    }
+                    fwd16_tw(x, w3, q, q2);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                    __syncwarp();
+                    const int wbase = w * 512 + 4 * (t & 31);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const int e = wbase + 128 * v;
+                        const uint4 r = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
+                        __stcs(reinterpret_cast<uint4*>(out + e),
+                               make_uint4(canon4(r.x, q, q2), canon4(r.y, q, q2), canon4(r.z, q, q2), canon4(r.w, q, q2)));
+                    }
+                }
+            };
+
+            if (t == 0) issue_col(0, team);
+            tw_fwd<A>(TWB(0), a.tw + ((size_t)limb_of(0) << LOGN), team, t);
+            cp_async_commit();
+#pragma unroll 1
+            for (int s = team; s < 16; s += TEAMS) colpass(0, s);
+            cta_sync_tmem();
+            uint32_t u = 0;
+#pragma unroll 1
+            for (uint32_t j = 0; j < nrow; ++j) {
+                const bool more = j + 1 < nrow;
+#pragma unroll 1
+                for (int s = team; s < 16; s += TEAMS, ++u) {
+                    rowpass(j, s, u);
+                    if (more) colpass(j + 1, s);         // overwrites exactly the cells rowpass just read
+                    else team_bar(team);                 // B0 read by the whole team before the next stage 1
+                }
+                cta_sync_tmem();
+            }
+        } else {
+            // sub-row s of row j: layers 15..4 (input bit-reversed), stage 1' into TMEM (layout j & 1)
+            auto rowpass = [&](uint32_t j, int s, uint32_t u) {
+                const uint32_t limb = limb_of(j);
+                const LimbConst lc = a.lc[limb];
+                const uint32_t q = lc.q, q2 = lc.q2;
+                const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+                uint32_t* S = (u & 1) ? B1 : B0;
+                uint2 w3[15];
+                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                cp_async_wait<0>();
+                __syncwarp();                            // this warp's slice of sub-row s landed
+                uint32_t x[16];
+                {   // stage 3': layers 15..12, thread (a, b), 16 contiguous elements
+                    const int aa = hi4, b = lo4;
+                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                    const int sw = (b >> 1) & 3;
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) {
+                        const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                        x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
+                    }
+                    inv16_tw(x, w3, q, q2);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                }
+                __syncwarp();
+                {   // stage 2': layers 11..8, thread (a, c), elements b
+                    const int aa = hi4, c = lo4;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
+                    const uint2* W = TWB(u & 1) + 32 * w + (aa & 1);
+                    inv16_sp<false>(x, W, W + 2 + (aa & 1), W + 6 + 3 * (aa & 1), W + 14 + 7 * (aa & 1), lc);
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
+                }
+                team_bar(team);                          // stage 2' done team-wide; the other buffer is free
+                {   // the team's next sub-row: data and twiddles into the other buffer
+                    uint32_t nj = j, ns = (uint32_t)s + TEAMS;
+                    if (ns >= 16) { nj = j + 1; ns = team; }
+                    if (nj < nrow) {
+                        const uint32_t nl = limb_of(nj);
+                        tw_inv<A>(TWB((u + 1) & 1), a.tw + ((size_t)nl << LOGN), ns, t);
+                        load_inv_slice((u & 1) ? B0 : B1, a.in + ((size_t)row_of(nj) << LOGN) + ns * SUBW, t);
+                    }
+                    cp_async_commit();
+                }
+                {   // stage 1': layers 7..4, thread (b, c), elements a -> TMEM (lazy, in [0, 2q))
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, hi4, lo4)];
+                    const uint2* T1 = TWB(u & 1) + 256;
+                    inv16_sp<false>(x, T1, T1 + 2, T1 + 4, T1 + 8, lc);
+                    if (j & 1) tm_st16s(tl + s, x);      // B: element 256 a + t at 32 a + 16 h + s
+                    else tm_st16(tl + 32 * s, x);        // A: 32 s + 16 h + a
+                }
+            };
+            // column pass s of row j: layers 3..0 with N^-1, canonical output
+            auto colpass = [&](uint32_t j, int s) {
+                const uint32_t limb = limb_of(j), row = row_of(j);
+                const LimbConst lc = a.lc[limb];
+                const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
+                uint32_t x[16];
+                if (j & 1) tm_ld16(tl + 32 * s, x);      // B: 32 s + 16 h + k
+                else tm_ld16s(tl + s, x);                // A: 32 k + 16 h + s
+                inv_radix<A, true>(x, tw, 0, 0, lc);
+                uint32_t* o = a.out + ((size_t)row << LOGN) + s * TT + t;
+#pragma unroll
+                for (int k = 0; k < 16; ++k) __stcs(o + k * SUBW, canon2(x[k], lc.q));
+            };
+
+            tw_inv<A>(TWB(0), a.tw + ((size_t)limb_of(0) << LOGN), team, t);
+            load_inv_slice(B0, a.in + ((size_t)row_of(0) << LOGN) + team * SUBW, t);
+            cp_async_commit();
+            uint32_t u = 0;
+#pragma unroll 1
+            for (int s = team; s < 16; s += TEAMS, ++u) rowpass(0, s, u);
+            cta_sync_tmem();
+#pragma unroll 1
+            for (uint32_t j = 0; j < nrow; ++j) {
+                const bool more = j + 1 < nrow;
+#pragma unroll 1
+                for (int s = team; s < 16; s += TEAMS) {
+                    colpass(j, s);
+                    if (more) { rowpass(j + 1, s, u); ++u; }   // refills exactly the cells colpass just read
+                }
+                cta_sync_tmem();
+            }
+        }
+    }
+    cp_async_wait<0>();
+    tfence_before();
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        tfence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(*tslot));
+    }
+}
+
+}  // namespace tmr
+}  // namespace wd

@@ -123,6 +123,11 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
         else if (rows >= sm || logN >= 15) ver = 8;
         else ver = 1;                                                   // N <= 2^14, few rows
     }
+    if (ver == 20 && logN == 16) {                                     // tm: TMEM-resident rows
+        const int n = launch_tmr(fwd, a, rows, p->sm_count, s);
+        if (n > 0) return n;
+        ver = 8;
+    }
     if (ver == 5 && logN >= 14) { launch_v5(logN, fwd, a, rows, p->sm_count, s); return 1; }
     if (ver == 1 || ver == 5) { launch_v1(logN, fwd, a, rows, s); return 1; }
     int cl = p->v8_cl;
@@ -401,8 +406,8 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     cudaDeviceGetAttribute(&p->sm_count, cudaDevAttrMultiProcessorCount, p->device);
     // A/B knobs: read here once, never on the launch path.  Unknown generations keep AUTO.
     if (const char* ev = getenv("WD_NTT_KERNEL")) {
-        const int v = ev[0] == 'v' ? atoi(ev + 1) : 0;
-        if (v == 1 || v == 5 || v == 8) p->kernel_ver = v;
+        const int v = ev[0] == 'v' ? atoi(ev + 1) : (ev[0] == 't' && ev[1] == 'm') ? 20 : 0;
+        if (v == 1 || v == 5 || v == 8 || v == 20) p->kernel_ver = v;
     }
     if (const char* ev = getenv("WD_NTT_CL")) p->v8_cl = atoi(ev) >= 8 ? 8 : atoi(ev) >= 4 ? 4 : atoi(ev) >= 2 ? 2 : 1;
     if (const char* ev = getenv("WD_NTT_LM")) p->limb_major = atoi(ev) != 0;
@@ -439,7 +444,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (cudaStreamCreateWithFlags(&p->fs, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->fe) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     if (prep_cc(p->logN) || prep_v8(p->logN, p->sm_count, &p->occ) || prep_rns() ||
-        (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4()))) {
+        (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4() || prep_tmr()))) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
     p->mode = WD_MODE_AUTO;
