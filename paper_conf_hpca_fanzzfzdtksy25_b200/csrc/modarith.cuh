@@ -55,13 +55,21 @@ __device__ __forceinline__ uint32_t shoup_mul(uint32_t a, uint32_t w, uint32_t w
 __device__ __forceinline__ void ct_bfly(uint32_t& X, uint32_t& Y, uint2 w, uint32_t q, uint32_t q2) {
     const uint32_t x = umin32(X, X - q2);          // [0, 2q)
     const uint32_t t = shoup_mul(Y, w.x, w.y, q);  // [0, 2q)
+#ifdef WD_BFLY_ALU
+    X = umin32(x + t, q2 << 1);                    // = x + t (< 4q): VIADDMNMX, kept off the fma pipe
+#else
     X = x + t;
+#endif
     Y = x - t + q2;
 }
 
 // inverse Gentleman-Sande butterfly: (X, Y) -> (X + Y, (X - Y) w), lazy in [0,2q)
 __device__ __forceinline__ void gs_bfly(uint32_t& X, uint32_t& Y, uint2 w, uint32_t q, uint32_t q2) {
+#ifdef WD_BFLY_ALU
+    uint32_t u = umin32(X + Y, q2 << 1);           // = X + Y (< 4q): VIADDMNMX, kept off the fma pipe
+#else
     uint32_t u = X + Y;
+#endif
     u = umin32(u, u - q2);
     const uint32_t t = X - Y + q2;
     Y = shoup_mul(t, w.x, w.y, q);

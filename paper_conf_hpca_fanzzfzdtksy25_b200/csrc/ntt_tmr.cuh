@@ -35,8 +35,10 @@ namespace tmr {
 constexpr int TEAMS = 4, TT = 256, NT = TEAMS * TT;
 constexpr int SUBW = 4096;
 constexpr int TWW = 768;                        // words per twiddle area (<= 384 (w, w') pairs)
-constexpr int TEAM_W = 2 * SUBW + 2 * TWW;      // per team: two sub-row buffers, two twiddle areas
-constexpr int SMEM = TEAMS * TEAM_W * 4 + 64;   // + one TMA mbarrier per team + the TMEM base slot
+// per team: three sub-row buffers (forward: the sub-row exchange and two TMA column stagings; inverse:
+// two input buffers), two twiddle areas
+constexpr int TEAM_W = 3 * SUBW + 2 * TWW;
+constexpr int SMEM = TEAMS * TEAM_W * 4 + 128;  // + three mbarriers per team + the TMEM base slot
 
 // ---------------------------------------------------------------- tensor memory
 __device__ __forceinline__ void tfence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -162,16 +164,18 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
     const int w = t >> 5, h = w >> 2, hi4 = t >> 4, lo4 = t & 15;
     uint32_t* TS = smem + team * TEAM_W;
     uint32_t* const B0 = TS;                     // forward: sub-row exchange; inverse: input buffer 0
-    uint32_t* const B1 = TS + SUBW;              // forward: TMA column staging; inverse: input buffer 1
-    auto TWB = [&](int b) { return reinterpret_cast<uint2*>(TS + 2 * SUBW + b * TWW); };
-    uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + team;
-    uint32_t* tslot = reinterpret_cast<uint32_t*>(smem + TEAMS * TEAM_W + 2 * TEAMS);
+    uint32_t* const B1 = TS + SUBW;              // forward: TMA column staging 0; inverse: input buffer 1
+    auto TWB = [&](int b) { return reinterpret_cast<uint2*>(TS + 3 * SUBW + b * TWW); };
+    // per team: tbar[0..1] the forward TMA stagings, tbar[2] "B0 free" (the team's 8 warps are done with
+    // the previous sub-row's exchange buffer)
+    uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + 3 * team;
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(smem + TEAMS * TEAM_W + 6 * TEAMS);
 
     if (threadIdx.x < 32) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" :: "r"(smem_u32(tslot)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
-    if (t == 0) { mb_init(tbar, 1); mb_init_fence(); }
+    if (t == 0) { mb_init(tbar, 1); mb_init(tbar + 1, 1); mb_init(tbar + 2, TT / 32); mb_init_fence(); }
     tfence_before();
     __syncthreads();
     tfence_after();
@@ -195,34 +199,41 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
 
     if (nrow > 0) {
         if constexpr (FWD) {
-            uint32_t tph = 0;
-            auto issue_col = [&](uint32_t j, int s) {   // team thread 0: column pass s of row j -> B1
+            // column pass m of the CTA (m = 4 j + i: row j, s = team + 4 i) lands in staging buffer m & 1
+            // (B1 / B2) and completes on mbarrier m & 1.  Its TMA is issued 1.5 passes ahead: the buffer was
+            // last read by column pass m - 2, and every warp of the team has passed a team barrier since
+            // (the stage-1 barrier of the sub-row in between), so column passes need no barrier of their own.
+            uint32_t* const B2 = TS + 2 * SUBW;
+            uint32_t tph = 0;                            // bit b: parity of mbarrier b's next completion
+            // (limb, physical row) of the CTA's current row j and of row j + 1 (one division per row)
+            uint32_t lbc = limb_of(0), rwc = row_of(0);
+            uint32_t lbn = nrow > 1 ? limb_of(1) : 0, rwn = nrow > 1 ? row_of(1) : 0;
+            auto issue_col = [&](uint32_t m, uint32_t prow) {   // team thread 0: column pass m of row `prow`
                 fence_proxy_async();
-                mb_expect(tbar, 16 * TT * 4);
-                tma2_load_hint(B1, &tm_in, s * TT, (int)(row_of(j) * 16), tbar, l2_evict_first_policy());
+                mb_expect(tbar + (m & 1), 16 * TT * 4);
+                tma2_load_hint((m & 1) ? B2 : B1, &tm_in, (team + 4 * (int)(m & 3)) * TT, (int)(prow * 16),
+                               tbar + (m & 1), l2_evict_first_policy());
             };
-            // column pass s of row j: layers 0..3, into TMEM (layout j & 1)
-            auto colpass = [&](uint32_t j, int s) {
-                const uint32_t limb = limb_of(j);
+            // column pass m (row j = m / 4, s = team + 4 (m & 3)): layers 0..3, into TMEM (layout j & 1)
+            auto colpass = [&](uint32_t m, uint32_t limb) {
+                const int s = team + 4 * (int)(m & 3);
                 const LimbConst lc = a.lc[limb];
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
-                mb_wait(tbar, tph);
-                tph ^= 1;
+                const uint32_t b = m & 1;
+                mb_wait(tbar + b, (tph >> b) & 1);
+                tph ^= 1u << b;
+                const uint32_t* SB = b ? B2 : B1;
                 uint32_t x[16];
 #pragma unroll
-                for (int k = 0; k < 16; ++k) x[k] = B1[k * TT + t];
-                team_bar(team);                          // staging read by the whole team
-                if (t == 0) {                            // the team's next column pass
-                    if (s + TEAMS < 16) issue_col(j, s + TEAMS);
-                    else if (j + 1 < nrow) issue_col(j + 1, team);
-                }
+                for (int k = 0; k < 16; ++k) x[k] = SB[k * TT + t];
                 fwd_radix<A>(x, tw, 0, 0, lc.q, lc.q2);
-                if (j & 1) tm_st16(tl + 32 * s, x);      // B: 32 s + 16 h + k
-                else tm_st16s(tl + s, x);                // A: 32 k + 16 h + s
+                if ((m >> 2) & 1) tm_st16(tl + 32 * s, x);   // B: 32 s + 16 h + k
+                else tm_st16s(tl + s, x);                    // A: 32 k + 16 h + s
             };
-            // sub-row s of row j: layers 4..15 (stage 1 from TMEM), canonical output
-            auto rowpass = [&](uint32_t j, int s, uint32_t u) {
-                const uint32_t limb = limb_of(j), row = row_of(j);
+            // sub-row s of row j: layers 4..15 (stage 1 from TMEM), canonical output; after its stage-1
+            // barrier, the TMA of column pass mnext (row prow_next) is issued
+            auto rowpass = [&](uint32_t j, int s, uint32_t u, uint32_t mnext, uint32_t prow_next) {
+                const uint32_t limb = lbc, row = rwc;
                 const LimbConst lc = a.lc[limb];
                 const uint32_t q = lc.q, q2 = lc.q2;
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
@@ -236,14 +247,16 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 {   // stage 1: layers 4..7, thread (b, c), elements a
                     const uint2* W = TWB(u & 1) + 16 * w;
                     fwd16_sp(x, W, W + 2, W + 4, W + 8, q, q2);
+                    if (u > 0) mb_wait(tbar + 2, (u - 1) & 1);   // every warp done with sub-row u - 1 in B0
 #pragma unroll
                     for (int i = 0; i < 16; ++i) S[v8_phys(i, hi4, lo4)] = x[i];
                 }
                 team_bar(team);                          // stage 1 done team-wide
+                if (t == 0 && mnext != ~0u) issue_col(mnext, prow_next);
                 {   // the team's next sub-row's twiddles
                     uint32_t nj = j, ns = (uint32_t)s + TEAMS;
                     if (ns >= 16) { nj = j + 1; ns = team; }
-                    if (nj < nrow) tw_fwd<A>(TWB((u + 1) & 1), a.tw + ((size_t)limb_of(nj) << LOGN), ns, t);
+                    if (nj < nrow) tw_fwd<A>(TWB((u + 1) & 1), a.tw + ((size_t)(nj == j ? lbc : lbn) << LOGN), ns, t);
                     cp_async_commit();
                 }
                 uint2 w3[15];
@@ -281,31 +294,52 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                         __stcs(reinterpret_cast<uint4*>(out + e),
                                make_uint4(canon4(r.x, q, q2), canon4(r.y, q, q2), canon4(r.z, q, q2), canon4(r.w, q, q2)));
                     }
+                    __syncwarp();
+                    if ((t & 31) == 0) mb_arrive(tbar + 2);   // this warp's last read of B0
                 }
             };
 
-            if (t == 0) issue_col(0, team);
-            tw_fwd<A>(TWB(0), a.tw + ((size_t)limb_of(0) << LOGN), team, t);
+            // prologue: the column passes 0..3 of row 0 (TMA 0, 1 up front; pass m issues m + 2 <= 4 after a
+            // team barrier, there being no sub-row in between yet)
+            const uint32_t mtot = 4 * nrow;              // column passes of the CTA
+            if (t == 0) {
+                issue_col(0, rwc);
+                issue_col(1, rwc);
+            }
+            tw_fwd<A>(TWB(0), a.tw + ((size_t)lbc << LOGN), team, t);
             cp_async_commit();
 #pragma unroll 1
-            for (int s = team; s < 16; s += TEAMS) colpass(0, s);
+            for (uint32_t m = 0; m < 4; ++m) {
+                colpass(m, lbc);
+                if (m + 2 <= 4 && m + 2 < mtot) {
+                    team_bar(team);
+                    if (t == 0) issue_col(m + 2, m + 2 < 4 ? rwc : rwn);
+                }
+            }
             cta_sync_tmem();
             uint32_t u = 0;
 #pragma unroll 1
             for (uint32_t j = 0; j < nrow; ++j) {
+                // rows j (lbc, rwc) and j + 1 (lbn, rwn) known; row j + 2 is the TMA target of the last
+                // column passes of row j + 1
                 const bool more = j + 1 < nrow;
+                const uint32_t r2 = j + 2 < nrow ? row_of(j + 2) : 0;
 #pragma unroll 1
-                for (int s = team; s < 16; s += TEAMS, ++u) {
-                    rowpass(j, s, u);
-                    if (more) colpass(j + 1, s);         // overwrites exactly the cells rowpass just read
-                    else team_bar(team);                 // B0 read by the whole team before the next stage 1
+                for (int i = 0; i < 4; ++i, ++u) {
+                    const int s = team + 4 * i;
+                    const uint32_t m = 4 * (j + 1) + i;  // the column pass after this sub-row
+                    const uint32_t mn = m + 1;           // its successor, whose TMA this sub-row issues
+                    rowpass(j, s, u, mn < mtot ? mn : ~0u, (mn >> 2) == j + 1 ? rwn : r2);
+                    if (more) colpass(m, lbn);           // overwrites exactly the cells rowpass read
                 }
+                lbc = lbn; rwc = rwn;
+                if (j + 2 < nrow) { lbn = limb_of(j + 2); rwn = r2; }
                 cta_sync_tmem();
             }
         } else {
             // sub-row s of row j: layers 15..4 (input bit-reversed), stage 1' into TMEM (layout j & 1)
-            auto rowpass = [&](uint32_t j, int s, uint32_t u) {
-                const uint32_t limb = limb_of(j);
+            auto rowpass = [&](uint32_t j, int s, uint32_t u, uint32_t limb, uint32_t row_self, uint32_t limb_next,
+                               uint32_t row_next) {
                 const LimbConst lc = a.lc[limb];
                 const uint32_t q = lc.q, q2 = lc.q2;
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
@@ -342,12 +376,11 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 }
                 team_bar(team);                          // stage 2' done team-wide; the other buffer is free
                 {   // the team's next sub-row: data and twiddles into the other buffer
-                    uint32_t nj = j, ns = (uint32_t)s + TEAMS;
-                    if (ns >= 16) { nj = j + 1; ns = team; }
+                    uint32_t nj = j, ns = (uint32_t)s + TEAMS, nl = limb, nr = row_self;
+                    if (ns >= 16) { nj = j + 1; ns = team; nl = limb_next; nr = row_next; }
                     if (nj < nrow) {
-                        const uint32_t nl = limb_of(nj);
                         tw_inv<A>(TWB((u + 1) & 1), a.tw + ((size_t)nl << LOGN), ns, t);
-                        load_inv_slice((u & 1) ? B0 : B1, a.in + ((size_t)row_of(nj) << LOGN) + ns * SUBW, t);
+                        load_inv_slice((u & 1) ? B0 : B1, a.in + ((size_t)nr << LOGN) + ns * SUBW, t);
                     }
                     cp_async_commit();
                 }
@@ -361,12 +394,11 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 }
             };
             // column pass s of row j: layers 3..0 with N^-1, canonical output
-            auto colpass = [&](uint32_t j, int s) {
-                const uint32_t limb = limb_of(j), row = row_of(j);
+            auto colpass = [&](int s, uint32_t limb, uint32_t row, bool jpar) {
                 const LimbConst lc = a.lc[limb];
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
                 uint32_t x[16];
-                if (j & 1) tm_ld16(tl + 32 * s, x);      // B: 32 s + 16 h + k
+                if (jpar) tm_ld16(tl + 32 * s, x);       // B: 32 s + 16 h + k
                 else tm_ld16s(tl + s, x);                // A: 32 k + 16 h + s
                 inv_radix<A, true>(x, tw, 0, 0, lc);
                 uint32_t* o = a.out + ((size_t)row << LOGN) + s * TT + t;
@@ -374,21 +406,28 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 for (int k = 0; k < 16; ++k) __stcs(o + k * SUBW, canon2(x[k], lc.q));
             };
 
-            tw_inv<A>(TWB(0), a.tw + ((size_t)limb_of(0) << LOGN), team, t);
-            load_inv_slice(B0, a.in + ((size_t)row_of(0) << LOGN) + team * SUBW, t);
+            // (limb, physical row) of rows j, j + 1, j + 2 (one division per row)
+            uint32_t lbc = limb_of(0), rwc = row_of(0);
+            uint32_t lbn = nrow > 1 ? limb_of(1) : 0, rwn = nrow > 1 ? row_of(1) : 0;
+            tw_inv<A>(TWB(0), a.tw + ((size_t)lbc << LOGN), team, t);
+            load_inv_slice(B0, a.in + ((size_t)rwc << LOGN) + team * SUBW, t);
             cp_async_commit();
             uint32_t u = 0;
+            bool jpar = false;                           // layout of row j (j & 1)
 #pragma unroll 1
-            for (int s = team; s < 16; s += TEAMS, ++u) rowpass(0, s, u);
+            for (int s = team; s < 16; s += TEAMS, ++u) rowpass(0, s, u, lbc, rwc, lbn, rwn);
             cta_sync_tmem();
 #pragma unroll 1
             for (uint32_t j = 0; j < nrow; ++j) {
                 const bool more = j + 1 < nrow;
+                const uint32_t lb2 = j + 2 < nrow ? limb_of(j + 2) : 0, rw2 = j + 2 < nrow ? row_of(j + 2) : 0;
 #pragma unroll 1
                 for (int s = team; s < 16; s += TEAMS) {
-                    colpass(j, s);
-                    if (more) { rowpass(j + 1, s, u); ++u; }   // refills exactly the cells colpass just read
+                    colpass(s, lbc, rwc, jpar);
+                    if (more) { rowpass(j + 1, s, u, lbn, rwn, lb2, rw2); ++u; }   // refills the cells colpass read
                 }
+                lbc = lbn; rwc = rwn; lbn = lb2; rwn = rw2;
+                jpar = !jpar;
                 cta_sync_tmem();
             }
         }

@@ -16,6 +16,9 @@ __device__ __forceinline__ void mb_wait(uint64_t* b, uint32_t parity) {
                  "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
                  "@!P1 bra MBW_%=;\n\t}\n" :: "r"(smem_u32(b)), "r"(parity) : "memory");
 }
+__device__ __forceinline__ void mb_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(b)) : "memory");
+}
 __device__ __forceinline__ void mb_expect(uint64_t* b, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(b)), "r"(bytes) : "memory");
 }
