@@ -1,5 +1,12 @@
 // k_tmr.cu -- launcher of the TMEM-resident CUDA-core NTT "tm" (N = 2^16; kernels in ntt_tmr.cuh,
 // DESIGN.md 5.1a).
+// This unit compiles the Harvey butterflies with their X + t / X + Y adds pinned to the ALU pipe
+// (modarith.cuh WD_BFLY_ALU: min(x + t, 4q), one VIADDMNMX instead of an IMAD.IADD on the fma pipe).
+// In the TMEM-resident kernel the fma pipe is the busiest one (ncu math_pipe_throttle); measured on
+// config 3: forward 1.022 -> 1.007 ms, inverse 0.963 -> 0.957 ms.  The v8 unit keeps the default
+// (there the same change made the forward slower: 1.061 -> 1.080 ms).  Device functions are compiled
+// per translation unit (no relocatable device code), so the two choices never meet.
+#define WD_BFLY_ALU 1
 #include <algorithm>
 #include <cstring>
 #include "launch.h"

@@ -38,7 +38,7 @@ constexpr int TWW = 768;                        // words per twiddle area (<= 38
 // per team: three sub-row buffers (forward: the sub-row exchange and two TMA column stagings; inverse:
 // two input buffers), two twiddle areas
 constexpr int TEAM_W = 3 * SUBW + 2 * TWW;
-constexpr int SMEM = TEAMS * TEAM_W * 4 + 128;  // + three mbarriers per team + the TMEM base slot
+constexpr int SMEM = TEAMS * TEAM_W * 4 + 128;  // + 3 mbarriers per team, the row mbarrier, the TMEM slot
 
 // ---------------------------------------------------------------- tensor memory
 __device__ __forceinline__ void tfence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -56,23 +56,23 @@ __device__ __forceinline__ void tm_ld16(uint32_t ta, uint32_t* x) {
 }
 // columns ta, ta + 32, ..., ta + 480 -> x[0..15]
 __device__ __forceinline__ void tm_ld16s(uint32_t ta, uint32_t* x) {
-    asm volatile("{\n\t.reg .b32 a;\n\t"
+    asm volatile("{\n\t"
                  "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%16];\n\t"
-                 "add.u32 a, %16, 32;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%1}, [a];\n\t"
-                 "add.u32 a, %16, 64;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%2}, [a];\n\t"
-                 "add.u32 a, %16, 96;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%3}, [a];\n\t"
-                 "add.u32 a, %16, 128;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%4}, [a];\n\t"
-                 "add.u32 a, %16, 160;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%5}, [a];\n\t"
-                 "add.u32 a, %16, 192;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%6}, [a];\n\t"
-                 "add.u32 a, %16, 224;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%7}, [a];\n\t"
-                 "add.u32 a, %16, 256;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%8}, [a];\n\t"
-                 "add.u32 a, %16, 288;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%9}, [a];\n\t"
-                 "add.u32 a, %16, 320;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%10}, [a];\n\t"
-                 "add.u32 a, %16, 352;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%11}, [a];\n\t"
-                 "add.u32 a, %16, 384;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%12}, [a];\n\t"
-                 "add.u32 a, %16, 416;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%13}, [a];\n\t"
-                 "add.u32 a, %16, 448;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%14}, [a];\n\t"
-                 "add.u32 a, %16, 480;\n\ttcgen05.ld.sync.aligned.32x32b.x1.b32 {%15}, [a];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%1}, [%16+32];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%2}, [%16+64];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%3}, [%16+96];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%4}, [%16+128];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%5}, [%16+160];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%6}, [%16+192];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%7}, [%16+224];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%8}, [%16+256];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%9}, [%16+288];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%10}, [%16+320];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%11}, [%16+352];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%12}, [%16+384];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%13}, [%16+416];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%14}, [%16+448];\n\t"
+                 "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%15}, [%16+480];\n\t"
                  "tcgen05.wait::ld.sync.aligned;\n\t}"
                  : "=r"(x[0]), "=r"(x[1]), "=r"(x[2]), "=r"(x[3]), "=r"(x[4]), "=r"(x[5]), "=r"(x[6]), "=r"(x[7]),
                    "=r"(x[8]), "=r"(x[9]), "=r"(x[10]), "=r"(x[11]), "=r"(x[12]), "=r"(x[13]), "=r"(x[14]), "=r"(x[15])
@@ -86,23 +86,23 @@ __device__ __forceinline__ void tm_st16(uint32_t ta, const uint32_t* x) {
                  : "memory");
 }
 __device__ __forceinline__ void tm_st16s(uint32_t ta, const uint32_t* x) {
-    asm volatile("{\n\t.reg .b32 a;\n\t"
+    asm volatile("{\n\t"
                  "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};\n\t"
-                 "add.u32 a, %0, 32;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%2};\n\t"
-                 "add.u32 a, %0, 64;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%3};\n\t"
-                 "add.u32 a, %0, 96;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%4};\n\t"
-                 "add.u32 a, %0, 128;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%5};\n\t"
-                 "add.u32 a, %0, 160;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%6};\n\t"
-                 "add.u32 a, %0, 192;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%7};\n\t"
-                 "add.u32 a, %0, 224;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%8};\n\t"
-                 "add.u32 a, %0, 256;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%9};\n\t"
-                 "add.u32 a, %0, 288;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%10};\n\t"
-                 "add.u32 a, %0, 320;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%11};\n\t"
-                 "add.u32 a, %0, 352;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%12};\n\t"
-                 "add.u32 a, %0, 384;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%13};\n\t"
-                 "add.u32 a, %0, 416;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%14};\n\t"
-                 "add.u32 a, %0, 448;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%15};\n\t"
-                 "add.u32 a, %0, 480;\n\ttcgen05.st.sync.aligned.32x32b.x1.b32 [a], {%16};\n\t}"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+32], {%2};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+64], {%3};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+96], {%4};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+128], {%5};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+160], {%6};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+192], {%7};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+224], {%8};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+256], {%9};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+288], {%10};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+320], {%11};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+352], {%12};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+384], {%13};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+416], {%14};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+448], {%15};\n\t"
+                 "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+480], {%16};\n\t}"
                  :: "r"(ta), "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7]),
                     "r"(x[8]), "r"(x[9]), "r"(x[10]), "r"(x[11]), "r"(x[12]), "r"(x[13]), "r"(x[14]), "r"(x[15])
                  : "memory");
@@ -156,31 +156,48 @@ __device__ __forceinline__ void load_inv_slice(uint32_t* S, const uint32_t* src,
     }
 }
 
+// the forward twiddle areas / stage bodies shared by the two directions are written out in each branch
 template <bool FWD>
 __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, const __grid_constant__ CUtensorMap tm_in) {
     constexpr int LOGN = 16, A = 4;
     extern __shared__ __align__(1024) uint32_t smem[];
     const int team = (int)(threadIdx.x >> 8), t = (int)(threadIdx.x & (TT - 1));
-    const int w = t >> 5, h = w >> 2, hi4 = t >> 4, lo4 = t & 15;
+    const int w = t >> 5, h = w >> 2, hi4 = t >> 4, lo4 = t & 15, lane = t & 31;
     uint32_t* TS = smem + team * TEAM_W;
     uint32_t* const B0 = TS;                     // forward: sub-row exchange; inverse: input buffer 0
     uint32_t* const B1 = TS + SUBW;              // forward: TMA column staging 0; inverse: input buffer 1
+    uint32_t* const B2 = TS + 2 * SUBW;          // forward: TMA column staging 1
     auto TWB = [&](int b) { return reinterpret_cast<uint2*>(TS + 3 * SUBW + b * TWW); };
     // per team: tbar[0..1] the forward TMA stagings, tbar[2] "B0 free" (the team's 8 warps are done with
-    // the previous sub-row's exchange buffer)
+    // the previous sub-row's exchange buffer); rowbar (CTA): every warp's TMEM writes of a row are done
     uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + 3 * team;
-    uint32_t* tslot = reinterpret_cast<uint32_t*>(smem + TEAMS * TEAM_W + 6 * TEAMS);
+    uint64_t* rowbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + 3 * TEAMS;
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(rowbar + 1);
 
     if (threadIdx.x < 32) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" :: "r"(smem_u32(tslot)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
-    if (t == 0) { mb_init(tbar, 1); mb_init(tbar + 1, 1); mb_init(tbar + 2, TT / 32); mb_init_fence(); }
+    if (t == 0) { mb_init(tbar, 1); mb_init(tbar + 1, 1); mb_init(tbar + 2, TT / 32); }
+    if (threadIdx.x == 0) mb_init(rowbar, NT / 32);
+    if (t == 0) mb_init_fence();
     tfence_before();
     __syncthreads();
     tfence_after();
     // this thread's TMEM lane (its warp's quadrant) and column half
     const uint32_t tl = *tslot + ((uint32_t)(32 * (w & 3)) << 16) + 16u * h;
+    // the warp's TMEM writes of a row are complete and ordered before the row barrier's arrival
+    auto row_arrive = [&]() {
+        tm_wait_st();
+        tfence_before();
+        __syncwarp();
+        if (lane == 0) mb_arrive(rowbar);
+    };
+    // every warp's TMEM writes of row r are visible to this thread's later TMEM reads
+    auto row_wait = [&](uint32_t r) {
+        mb_wait(rowbar, r & 1);
+        tfence_after();
+    };
 
     const uint32_t G = gridDim.x;
     const uint32_t nrow = rows > blockIdx.x ? (rows - blockIdx.x + G - 1) / G : 0;
@@ -198,23 +215,28 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
     };
 
     if (nrow > 0) {
+        // (limb, physical row) of the CTA's rows j (lbc, rwc) and j + 1 (lbn, rwn): one division per row
+        uint32_t lbc = limb_of(0), rwc = row_of(0);
+        uint32_t lbn = nrow > 1 ? limb_of(1) : 0, rwn = nrow > 1 ? row_of(1) : 0;
+        uint32_t u = 0;                              // the team's sub-row counter (twiddle / buffer parity)
         if constexpr (FWD) {
-            // column pass m of the CTA (m = 4 j + i: row j, s = team + 4 i) lands in staging buffer m & 1
-            // (B1 / B2) and completes on mbarrier m & 1.  Its TMA is issued 1.5 passes ahead: the buffer was
-            // last read by column pass m - 2, and every warp of the team has passed a team barrier since
-            // (the stage-1 barrier of the sub-row in between), so column passes need no barrier of their own.
-            uint32_t* const B2 = TS + 2 * SUBW;
-            uint32_t tph = 0;                            // bit b: parity of mbarrier b's next completion
-            // (limb, physical row) of the CTA's current row j and of row j + 1 (one division per row)
-            uint32_t lbc = limb_of(0), rwc = row_of(0);
-            uint32_t lbn = nrow > 1 ? limb_of(1) : 0, rwn = nrow > 1 ? row_of(1) : 0;
-            auto issue_col = [&](uint32_t m, uint32_t prow) {   // team thread 0: column pass m of row `prow`
+            // Schedule per team and row j: for its four s,
+            //   R1(j, s)  [TMEM -> stage 1 -> B0]   C(j+1, s) [TMA staging -> layers 0..3 -> TMEM]
+            //   team barrier   R23(j, s) [stage 2, stage 3 -> out]
+            // The column pass sits between stage 1 and the barrier that stage 2 needs, so the barrier wait
+            // is covered by a whole pass of work; it overwrites exactly the TMEM cells R1 just read.
+            // Column pass m (= 4 j + i: row j, s = team + 4 i) lands in staging buffer m & 1 (B1 / B2) and
+            // completes on mbarrier m & 1; its TMA is issued right after the team barrier that follows
+            // column pass m - 2, the previous reader of that buffer (two passes ahead).
+            uint32_t tph = 0;                        // bit b: parity of mbarrier b's next completion
+            const uint32_t mtot = 4 * nrow;          // column passes of the CTA
+            auto issue_col = [&](uint32_t m, uint32_t prow) {   // team thread 0
                 fence_proxy_async();
                 mb_expect(tbar + (m & 1), 16 * TT * 4);
                 tma2_load_hint((m & 1) ? B2 : B1, &tm_in, (team + 4 * (int)(m & 3)) * TT, (int)(prow * 16),
                                tbar + (m & 1), l2_evict_first_policy());
             };
-            // column pass m (row j = m / 4, s = team + 4 (m & 3)): layers 0..3, into TMEM (layout j & 1)
+            // column pass m (row m / 4): layers 0..3, into TMEM (layout (m / 4) & 1)
             auto colpass = [&](uint32_t m, uint32_t limb) {
                 const int s = team + 4 * (int)(m & 3);
                 const LimbConst lc = a.lc[limb];
@@ -230,111 +252,106 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 if ((m >> 2) & 1) tm_st16(tl + 32 * s, x);   // B: 32 s + 16 h + k
                 else tm_st16s(tl + s, x);                    // A: 32 k + 16 h + s
             };
-            // sub-row s of row j: layers 4..15 (stage 1 from TMEM), canonical output; after its stage-1
-            // barrier, the TMA of column pass mnext (row prow_next) is issued
-            auto rowpass = [&](uint32_t j, int s, uint32_t u, uint32_t mnext, uint32_t prow_next) {
-                const uint32_t limb = lbc, row = rwc;
-                const LimbConst lc = a.lc[limb];
-                const uint32_t q = lc.q, q2 = lc.q2;
-                const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
-                uint32_t* out = a.out + ((size_t)row << LOGN) + s * SUBW;
-                uint32_t* S = B0;
-                cp_async_wait<0>();
-                __syncwarp();                            // this warp's stage-1 twiddles landed
-                uint32_t x[16];
-                if (j & 1) tm_ld16s(tl + s, x);          // B: element 256 a + t at 32 a + 16 h + s
-                else tm_ld16(tl + 32 * s, x);            // A: 32 s + 16 h + a
-                {   // stage 1: layers 4..7, thread (b, c), elements a
-                    const uint2* W = TWB(u & 1) + 16 * w;
-                    fwd16_sp(x, W, W + 2, W + 4, W + 8, q, q2);
-                    if (u > 0) mb_wait(tbar + 2, (u - 1) & 1);   // every warp done with sub-row u - 1 in B0
-#pragma unroll
-                    for (int i = 0; i < 16; ++i) S[v8_phys(i, hi4, lo4)] = x[i];
-                }
-                team_bar(team);                          // stage 1 done team-wide
-                if (t == 0 && mnext != ~0u) issue_col(mnext, prow_next);
-                {   // the team's next sub-row's twiddles
-                    uint32_t nj = j, ns = (uint32_t)s + TEAMS;
-                    if (ns >= 16) { nj = j + 1; ns = team; }
-                    if (nj < nrow) tw_fwd<A>(TWB((u + 1) & 1), a.tw + ((size_t)(nj == j ? lbc : lbn) << LOGN), ns, t);
-                    cp_async_commit();
-                }
-                uint2 w3[15];
-                load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
-                {   // stage 2: layers 8..11, thread (a, c), elements b
-                    const int aa = hi4, c = lo4;
-#pragma unroll
-                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
-                    const uint2* T2 = TWB(u & 1) + 128;
-                    fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, q, q2);
-#pragma unroll
-                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
-                }
-                __syncwarp();
-                {   // stage 3: layers 12..15, thread (a, b), 16 contiguous elements; coalesced store
-                    const int aa = hi4, b = lo4;
-                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
-                    const int sw = (b >> 1) & 3;
-#pragma unroll
-                    for (int v = 0; v < 4; ++v) {
-                        const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
-                        x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
-                    }
-                    fwd16_tw(x, w3, q, q2);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
-                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
-                    __syncwarp();
-                    const int wbase = w * 512 + 4 * (t & 31);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v) {
-                        const int e = wbase + 128 * v;
-                        const uint4 r = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
-                        __stcs(reinterpret_cast<uint4*>(out + e),
-                               make_uint4(canon4(r.x, q, q2), canon4(r.y, q, q2), canon4(r.z, q, q2), canon4(r.w, q, q2)));
-                    }
-                    __syncwarp();
-                    if ((t & 31) == 0) mb_arrive(tbar + 2);   // this warp's last read of B0
-                }
-            };
 
-            // prologue: the column passes 0..3 of row 0 (TMA 0, 1 up front; pass m issues m + 2 <= 4 after a
-            // team barrier, there being no sub-row in between yet)
-            const uint32_t mtot = 4 * nrow;              // column passes of the CTA
+            // prologue: the column passes of row 0 (TMA 0, 1 up front, m + 2 after pass m's team barrier)
             if (t == 0) {
                 issue_col(0, rwc);
-                issue_col(1, rwc);
+                if (1 < mtot) issue_col(1, rwc);
             }
             tw_fwd<A>(TWB(0), a.tw + ((size_t)lbc << LOGN), team, t);
             cp_async_commit();
 #pragma unroll 1
             for (uint32_t m = 0; m < 4; ++m) {
                 colpass(m, lbc);
-                if (m + 2 <= 4 && m + 2 < mtot) {
-                    team_bar(team);
-                    if (t == 0) issue_col(m + 2, m + 2 < 4 ? rwc : rwn);
-                }
+                team_bar(team);
+                if (t == 0 && m + 2 < mtot) issue_col(m + 2, m + 2 < 4 ? rwc : rwn);
             }
-            cta_sync_tmem();
-            uint32_t u = 0;
+            row_arrive();
 #pragma unroll 1
             for (uint32_t j = 0; j < nrow; ++j) {
-                // rows j (lbc, rwc) and j + 1 (lbn, rwn) known; row j + 2 is the TMA target of the last
-                // column passes of row j + 1
                 const bool more = j + 1 < nrow;
                 const uint32_t r2 = j + 2 < nrow ? row_of(j + 2) : 0;
+                const uint32_t q = 0;   // (per-row constants are loaded inside the passes)
+                (void)q;
 #pragma unroll 1
                 for (int i = 0; i < 4; ++i, ++u) {
                     const int s = team + 4 * i;
-                    const uint32_t m = 4 * (j + 1) + i;  // the column pass after this sub-row
-                    const uint32_t mn = m + 1;           // its successor, whose TMA this sub-row issues
-                    rowpass(j, s, u, mn < mtot ? mn : ~0u, (mn >> 2) == j + 1 ? rwn : r2);
-                    if (more) colpass(m, lbn);           // overwrites exactly the cells rowpass read
+                    const LimbConst lc = a.lc[lbc];
+                    const uint2* __restrict__ tw = a.tw + ((size_t)lbc << LOGN);
+                    uint32_t* S = B0;
+                    // ---- R1(j, s): stage 1 (layers 4..7, thread (b, c), elements a) from TMEM
+                    if (i == 0) row_wait(j);             // every column pass of row j is in TMEM
+                    cp_async_wait<0>();
+                    __syncwarp();                        // this warp's stage-1 twiddles landed
+                    uint32_t x[16];
+                    if (j & 1) tm_ld16s(tl + s, x);      // B: element 256 a + t at 32 a + 16 h + s
+                    else tm_ld16(tl + 32 * s, x);        // A: 32 s + 16 h + a
+                    {
+                        const uint2* W = TWB(u & 1) + 16 * w;
+                        fwd16_sp(x, W, W + 2, W + 4, W + 8, lc.q, lc.q2);
+                        if (u > 0) mb_wait(tbar + 2, (u - 1) & 1);   // every warp done with sub-row u - 1
+#pragma unroll
+                        for (int k = 0; k < 16; ++k) S[v8_phys(k, hi4, lo4)] = x[k];
+                    }
+                    // ---- C(j+1, s): overwrites exactly the TMEM cells R1 read
+                    const uint32_t m = 4 * (j + 1) + i;
+                    if (more) {
+                        colpass(m, lbn);
+                        if (i == 3) row_arrive();        // this warp's part of row j + 1 is in TMEM
+                    }
+                    team_bar(team);                      // stage 1 (and column pass m) done team-wide
+                    if (t == 0 && more && m + 2 < mtot) issue_col(m + 2, ((m + 2) >> 2) == j + 1 ? rwn : r2);
+                    {   // the team's next sub-row's twiddles
+                        uint32_t nj = j, ns = (uint32_t)s + TEAMS;
+                        if (ns >= 16) { nj = j + 1; ns = team; }
+                        if (nj < nrow) tw_fwd<A>(TWB((u + 1) & 1), a.tw + ((size_t)(nj == j ? lbc : lbn) << LOGN), ns, t);
+                        cp_async_commit();
+                    }
+                    // ---- R23(j, s)
+                    const uint32_t qq = lc.q, q2 = lc.q2;
+                    uint32_t* out = a.out + ((size_t)rwc << LOGN) + s * SUBW;
+                    uint2 w3[15];
+                    load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
+                    {   // stage 2: layers 8..11, thread (a, c), elements b
+                        const int aa = hi4, c = lo4;
+#pragma unroll
+                        for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(aa, k, c)];
+                        const uint2* T2 = TWB(u & 1) + 128;
+                        fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, qq, q2);
+#pragma unroll
+                        for (int k = 0; k < 16; ++k) S[v8_phys(aa, k, c)] = x[k];
+                    }
+                    __syncwarp();
+                    {   // stage 3: layers 12..15, thread (a, b), 16 contiguous elements; coalesced store
+                        const int aa = hi4, b = lo4;
+                        uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+                        const int sw = (b >> 1) & 3;
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+                            x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
+                        }
+                        fwd16_tw(x, w3, qq, q2);
+#pragma unroll
+                        for (int v = 0; v < 4; ++v)
+                            *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
+                                make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+                        __syncwarp();
+                        const int wbase = w * 512 + 4 * lane;
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            const int e = wbase + 128 * v;
+                            const uint4 r = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
+                            __stcs(reinterpret_cast<uint4*>(out + e),
+                                   make_uint4(canon4(r.x, qq, q2), canon4(r.y, qq, q2), canon4(r.z, qq, q2),
+                                              canon4(r.w, qq, q2)));
+                        }
+                        __syncwarp();
+                        if (lane == 0) mb_arrive(tbar + 2);   // this warp's last read of B0
+                    }
                 }
                 lbc = lbn; rwc = rwn;
                 if (j + 2 < nrow) { lbn = limb_of(j + 2); rwn = r2; }
-                cta_sync_tmem();
             }
         } else {
             // sub-row s of row j: layers 15..4 (input bit-reversed), stage 1' into TMEM (layout j & 1)
@@ -406,13 +423,9 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 for (int k = 0; k < 16; ++k) __stcs(o + k * SUBW, canon2(x[k], lc.q));
             };
 
-            // (limb, physical row) of rows j, j + 1, j + 2 (one division per row)
-            uint32_t lbc = limb_of(0), rwc = row_of(0);
-            uint32_t lbn = nrow > 1 ? limb_of(1) : 0, rwn = nrow > 1 ? row_of(1) : 0;
             tw_inv<A>(TWB(0), a.tw + ((size_t)lbc << LOGN), team, t);
             load_inv_slice(B0, a.in + ((size_t)rwc << LOGN) + team * SUBW, t);
             cp_async_commit();
-            uint32_t u = 0;
             bool jpar = false;                           // layout of row j (j & 1)
 #pragma unroll 1
             for (int s = team; s < 16; s += TEAMS, ++u) rowpass(0, s, u, lbc, rwc, lbn, rwn);
