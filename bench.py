@@ -549,10 +549,14 @@ def main():
     stream = torch.cuda.current_stream()
     sp = stream.cuda_stream
 
+    kern = {}
+
     def step():
         wdntt.wd_ntt_forward(plan.handle, x, y, batch, sp)
         lf = wdntt.wd_ntt_last_launches()
+        kern["forward"] = wdntt.wd_ntt_last_kernel()
         wdntt.wd_ntt_inverse(plan.handle, y, z, batch, sp)
+        kern["inverse"] = wdntt.wd_ntt_last_kernel()
         return lf + wdntt.wd_ntt_last_launches()
 
     for _ in range(max(3, args.warmup)):
@@ -718,7 +722,9 @@ def main():
                               else "eager launches, CUDA events around every launch")},
         "fwd_kops": rows * world / (fwd_ms / 1e3) / 1e3, "inv_kops": rows * world / (inv_ms / 1e3) / 1e3,
         "fwd_ms": fwd_ms, "inv_ms": inv_ms,
-        "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": achieved, "peak": hbm, "unit": "GB/s",
+        "kernels": kern,
+        "roofline": {"bound": "hbm", "kernel": "%s (%s)" % (dom_name, kern.get(dom_name, "?")), "achieved": achieved,
+                     "peak": hbm, "unit": "GB/s",
                      "frac": achieved / hbm, "traffic": traffic, "traffic_source": traffic_src,
                      "peak_kind": "%s (MEASURED_PEAKS.json hbm_gbs copy bandwidth)" % pk_kind,
                      "algorithmic_bytes_per_launch": alg_bytes},
@@ -727,12 +733,12 @@ def main():
         "roofline_tensor": {"bound": "tensor", "achieved": tmacs, "peak": i8_pk, "unit": "TMAC/s (int8)",
                             "frac": tmacs / i8_pk, "n64_peak": i8_pk64, "peak_kind": i8_kind,
                             "macs_per_launch": {"forward": macs_f, "inverse": macs_i},
-                            "note": "0 for modes without tcgen05 work (cuda = v8 butterflies)"},
+                            "note": "0 for modes without tcgen05 work (cuda = tm / v8 butterflies)"},
         # the bound that actually limits a Shoup-butterfly kernel on B200: the fma pipe (IMAD.HI at
         # quarter rate + 2 IMAD per butterfly); peak = the measured butterfly rate of a pure
         # register-resident butterfly loop (scripts/int_probe.cu, profiles/r01/int_probe.jsonl:
         # 13.6 butterflies/clk/SM) x SMs x the SM clock measured during the timed region
-        "roofline_alu": {"bound": "alu", "kernel": dom_name,
+        "roofline_alu": {"bound": "alu", "kernel": "%s (%s)" % (dom_name, kern.get(dom_name, "?")),
                          "achieved": (n // 2) * logn * rows / (dom_ms / 1e3) / 1e9,
                          "peak": BFLY_PER_CLK_SM * sms * (clk.summary()["sm_mhz"] or 1965) / 1e3,
                          "unit": "G butterflies/s",

@@ -244,6 +244,12 @@ int wd_ntt_plan_autotune(wd_ntt_plan* plan, uint32_t batch, wd_stream_t stream, 
 /* Kernel launches issued by the last forward/inverse call on this thread. */
 uint32_t wd_ntt_last_launches(void);
 
+/* Name of the kernel family the last forward/inverse call on this thread dispatched to (a static
+ * string, never NULL; "" before the first call): "tm" (TMEM-resident rows, N = 2^16), "v8/cl1",
+ * "v8/cl2", "v8/cl4", "v8/cl8" (v8 with 1..8-CTA clusters per row), "v5", "v1", "small", "tc4", "tensor",
+ * "fused", "cuda_gemm", "ftc".  Diagnostics for benches and tests: which path AUTO took. */
+const char* wd_ntt_last_kernel(void);
+
 /* Diagnostics only: while dev_buf (device memory, 20480 uint64 words) is set, every WD_MODE_TC4 launch
  * records clock64() timestamps of CTA 0's pipeline events into it (loads, MMAs, accumulator
  * hand-over, staging hand-over, stores; ntt_tc4.cuh TR_*).  NULL switches it off.  Process-wide. */

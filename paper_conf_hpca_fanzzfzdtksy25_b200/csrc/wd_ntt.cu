@@ -26,6 +26,7 @@ using namespace wd;
 namespace {
 thread_local int g_last_error = WD_OK;
 thread_local uint32_t g_last_launches = 0;
+thread_local const char* g_last_kernel = "";
 int set_err(int e) { g_last_error = e; return e; }
 }  // namespace
 
@@ -116,8 +117,11 @@ int ensure_tensor_tables(wd_ntt_plan* p) {
 // AUTO / CUDA: the measured default CUDA-core kernel per N and row count
 int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t rows, cudaStream_t s) {
     const uint32_t logN = p->logN, sm = (uint32_t)p->sm_count;
-    if (logN < 12) { launch_v1(logN, fwd, a, rows, s); return 1; }
+    if (logN < 12) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "small"; return 1; }
     int ver = p->kernel_ver;
+    // N = 2^16 with at least two rows per SM: tm, the TMEM-resident kernel (one CTA per SM, one row in
+    // flight per SM; below 2 x SM rows its row rounds leave SMs idle and v8's clusters win)
+    if (ver == 0 && logN == 16 && rows >= 2 * sm) ver = 20;
     if (ver == 0) {
         if ((logN == 15 || logN == 16) && rows < sm / 4) ver = 5;        // v5: the row in a cluster's DSMEM
         else if (rows >= sm || logN >= 15) ver = 8;
@@ -125,11 +129,11 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     }
     if (ver == 20 && logN == 16) {                                     // tm: TMEM-resident rows
         const int n = launch_tmr(fwd, a, rows, p->sm_count, s);
-        if (n > 0) return n;
+        if (n > 0) { g_last_kernel = "tm"; return n; }
         ver = 8;
     }
-    if (ver == 5 && logN >= 14) { launch_v5(logN, fwd, a, rows, p->sm_count, s); return 1; }
-    if (ver == 1 || ver == 5) { launch_v1(logN, fwd, a, rows, s); return 1; }
+    if (ver == 5 && logN >= 14) { launch_v5(logN, fwd, a, rows, p->sm_count, s); g_last_kernel = "v5"; return 1; }
+    if (ver == 1 || ver == 5) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "v1"; return 1; }
     int cl = p->v8_cl;
     if (!cl) {
         cl = 2;
@@ -142,6 +146,10 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
         else if (logN >= 15 && rows <= sm) cl = 4;
     }
     launch_v8(logN, fwd, a, rows, cl, 0, p->occ, p->v8_tma, s);
+    {
+        const int cm = std::max(1, std::min(cl, 1 << std::min<int>(3, (int)logN - 12)));   // launch_v8's clamp
+        g_last_kernel = cm == 8 ? "v8/cl8" : cm == 4 ? "v8/cl4" : cm == 2 ? "v8/cl2" : "v8/cl1";
+    }
     return 1;
 }
 
@@ -174,7 +182,7 @@ int run_mode(const wd_ntt_plan* p, int mode, float share, bool fwd, const uint32
         launches = launch_cuda_core(p, fwd, a, rows, s);
     } else if (mode == WD_MODE_TC4) {
         if (!p->t4.ok) return set_err(WD_EUNSUPPORTED);
-        if (fwd) launches = launch_tc4(fwd, a, p->t4, rows, p->sm_count, s);
+        if (fwd) { launches = launch_tc4(fwd, a, p->t4, rows, p->sm_count, s); g_last_kernel = "tc4"; }
         else launches = launch_cuda_core(p, fwd, a, rows, s);          // inverse kernel: not yet built
         if (launches == -2) return set_err(WD_ECUDA);
         if (launches < 0) return set_err(WD_EUNSUPPORTED);
@@ -183,11 +191,15 @@ int run_mode(const wd_ntt_plan* p, int mode, float share, bool fwd, const uint32
         if (mode == WD_MODE_CUDA_GEMM) {
             launch_wdcuda(fwd, a, p->tc, rows, p->sm_count, s);
             launches = 1;
+            g_last_kernel = "cuda_gemm";
         } else if (mode == WD_MODE_TENSOR) {
             launches = launch_tensor(fwd, a, p->tc, rows, p->sm_count, s);
+            g_last_kernel = "tensor";
         } else if (mode == WD_MODE_FUSED) {
             launches = launch_fused(fwd, a, p->tc, rows, p->sm_count, share, s);
+            g_last_kernel = "fused";
         } else if (mode == WD_MODE_FTC) {
+            g_last_kernel = "ftc";
             // WD-FTC: split at a polynomial boundary (rows stay limb-aligned), WD-Tensor on the first
             // bt polynomials in a forked stream, WD-CUDA on the rest in `s`, then join.
             const uint32_t bt = std::min<uint32_t>(batch, (uint32_t)std::lround(p->ftc_share * batch));
@@ -779,6 +791,7 @@ int wd_ntt_plan_autotune(wd_ntt_plan* p, uint32_t batch, wd_stream_t st, float* 
 }
 
 uint32_t wd_ntt_last_launches(void) { return g_last_launches; }
+const char* wd_ntt_last_kernel(void) { return g_last_kernel; }
 
 void wd_ntt_debug_tc4_trace(void* dev_buf) { tc4_set_trace(dev_buf); }
 

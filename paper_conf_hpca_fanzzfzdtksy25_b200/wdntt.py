@@ -64,6 +64,7 @@ _SIGS = {
     "wd_ntt_plan_autotune": (_i32, [_vp, _u32, _vp, ctypes.POINTER(ctypes.c_float)]),
     "wd_ntt_plan_get_mode": (_i32, [_vp]),
     "wd_ntt_last_launches": (_u32, []),
+    "wd_ntt_last_kernel": (ctypes.c_char_p, []),
     "wd_ntt_debug_tc4_trace": (None, [_vp]),
     "wd_ntt_last_error": (_i32, []),
     "wd_ntt_strerror": (ctypes.c_char_p, [_i32]),
@@ -216,6 +217,10 @@ def wd_ntt_plan_get_mode(plan: int) -> int:
 
 def wd_ntt_last_launches() -> int:
     return _lib.wd_ntt_last_launches()
+
+
+def wd_ntt_last_kernel() -> str:
+    return _lib.wd_ntt_last_kernel().decode()
 
 
 def wd_ntt_last_error() -> int:

@@ -181,12 +181,14 @@ def test_config4_n131072_l48(wd):
 
 
 # -------------------------------------------------------------- AUTO's decision boundaries
-# AUTO picks the kernel (v1 / v5 / v8) and v8's cluster size (8, 4, 2, 1 CTAs per row) from N and
-# the row count, with thresholds at SM/4, SM/2, SM and 8 x SM rows (wd_ntt.cu launch_cuda_core).
+# AUTO picks the kernel (v1 / v5 / v8 / tm) and v8's cluster size (8, 4, 2, 1 CTAs per row) from N and
+# the row count, with thresholds at SM/4, SM/2, SM, 2 x SM (tm at N = 2^16) and 8 x SM rows (wd_ntt.cu
+# launch_cuda_core).
 # Every N, every threshold +-1, every row of both directions against the oracle.
 def _boundary_rows():
     sm = torch.cuda.get_device_properties(0).multi_processor_count if torch.cuda.is_available() else 148
-    pts = {1, sm // 4 - 1, sm // 4, sm // 2, sm // 2 + 1, sm - 1, sm, sm + 1, 8 * sm - 1, 8 * sm}
+    pts = {1, sm // 4 - 1, sm // 4, sm // 2, sm // 2 + 1, sm - 1, sm, sm + 1, 2 * sm - 1, 2 * sm, 2 * sm + 1,
+           8 * sm - 1, 8 * sm}
     return sorted(pts)
 
 
@@ -198,6 +200,8 @@ def test_auto_decision_boundaries(wd, logn):
         x = inputs.uniform_residues(primes, n, rows, 7000 + logn * 10007 + rows)
         plan = wd.Plan(n, primes)
         y = gpu_fwd(wd, plan, x)
+        sm = torch.cuda.get_device_properties(0).multi_processor_count
+        assert (wd.wd_ntt_last_kernel() == "tm") == (logn == 16 and rows >= 2 * sm), (logn, rows)
         assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, rows)
         assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (logn, rows)
         plan.close()
@@ -330,6 +334,38 @@ def test_v8_column_feeds(wd, feed, logn, cl, monkeypatch):
     plan.inverse(t, t)
     torch.cuda.synchronize()
     assert np.array_equal(to_host(t), x), (feed, logn, cl)
+
+
+# tm, the TMEM-resident kernel (WD_NTT_KERNEL=tm; AUTO at N = 2^16 with >= 2 x SM rows): fewer rows than
+# SMs (idle CTAs), one row, ragged row counts against the SM count (CTAs with one row more than others),
+# both layouts of the TMEM ping-pong (odd and even rows per CTA), the natural row order (WD_NTT_LM=0),
+# edge inputs, in place; every row of both directions against the oracle
+@pytest.mark.parametrize("L,batch,lm", [(1, 1, "1"), (3, 1, "1"), (36, 5, "1"), (4, 83, "1"), (60, 7, "1"),
+                                        (5, 61, "0"), (36, 9, "0")])
+def test_tm_kernel(wd, L, batch, lm, monkeypatch):
+    monkeypatch.setenv("WD_NTT_KERNEL", "tm")
+    monkeypatch.setenv("WD_NTT_LM", lm)
+    n = 1 << 16
+    primes = [P[(7 * i + L) % 60] for i in range(L)]
+    x = inputs.uniform_residues(primes, n, batch, 5500 + L * 131 + batch)
+    plan = wd.Plan(n, primes, mode="cuda")
+    y = gpu_fwd(wd, plan, x)
+    assert wd.wd_ntt_last_kernel() == "tm"
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (L, batch)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (L, batch)
+    t = to_dev(x)
+    plan.forward(t, t)                                   # in place
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(t), y), (L, batch)
+    plan.inverse(t, t)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(t), x), (L, batch)
+    for kind in ("zeros", "qminus1"):
+        e = np.zeros_like(x) if kind == "zeros" else np.broadcast_to(
+            np.array(primes, dtype=np.uint32)[None, :, None] - 1, x.shape).copy()
+        assert np.array_equal(gpu_fwd(wd, plan, e), oracle.ntt_forward(e, primes)), (L, batch, kind)
+        assert np.array_equal(gpu_inv(wd, plan, e), oracle.ntt_inverse(e, primes)), (L, batch, kind)
+    plan.close()
 
 
 # Primes across the range the ABI accepts (the lazy bounds [0, 4q) < 2^32 hold for any q < 2^30).
