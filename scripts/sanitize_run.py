@@ -1,6 +1,6 @@
 """Drive every launch path of libwdntt.so once on small shapes, for compute-sanitizer
 (memcheck / racecheck / synccheck).  Usage: python scripts/sanitize_run.py [group ...]
-Groups: v8 v8feeds cc cl small tensor fused ftc gemm tc4 rns host.  Each group prints one line; the round trip
+Groups: v8 v8feeds tm cc cl small tensor fused ftc gemm tc4 rns host.  Each group prints one line; the round trip
 is checked (INTT(NTT(x)) == x) so a wrong result under the sanitizer is visible too."""
 import os
 import sys
@@ -42,6 +42,19 @@ def group_v8feeds():
             rt(p, 1 << logn, pr, batch)
             p.close()
     os.environ.pop("WD_NTT_V8_TMA"); os.environ.pop("WD_NTT_CL")
+
+
+def group_tm():
+    # tm, the TMEM-resident kernel (N = 2^16): fewer rows than SMs, and CTAs with 2 and 3 rows (both
+    # TMEM layouts, the row mbarrier handoff, the cross-row TMA / cp.async prefetches)
+    os.environ["WD_NTT_KERNEL"] = "tm"
+    for L, batch in ((2, 3), (4, 40), (3, 100)):
+        pr = inputs.bench_primes(L)
+        p = wdntt.Plan(1 << 16, pr)
+        rt(p, 1 << 16, pr, batch)
+        assert wdntt.wd_ntt_last_kernel() == "tm"
+        p.close()
+    os.environ.pop("WD_NTT_KERNEL")
 
 
 def group_cc():
