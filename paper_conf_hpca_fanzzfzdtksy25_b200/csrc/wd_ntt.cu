@@ -119,9 +119,13 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     const uint32_t logN = p->logN, sm = (uint32_t)p->sm_count;
     if (logN < 12) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "small"; return 1; }
     int ver = p->kernel_ver;
-    // N = 2^16 with at least two rows per SM: tm, the TMEM-resident kernel (one CTA per SM, one row in
-    // flight per SM; below 2 x SM rows its row rounds leave SMs idle and v8's clusters win)
-    if (ver == 0 && logN == 16 && rows >= 2 * sm) ver = 20;
+    // N = 2^16: tm, the TMEM-resident kernel (one CTA per SM, one row in flight per SM), when its rounds
+    // of SM-count rows are at least 85% full; a last round with fewer rows leaves whole SMs idle, while
+    // v8's 4 CTAs per SM absorb such a tail (scripts/gpu_tm_rows.sh: rows 148 / 296 / 444 / 4608 tm
+    // 1.19 / 1.06 / 1.06 / 1.08 x v8; rows 152 / 300 v8 1.22 / 1.12 x tm)
+    if (ver == 0 && logN == 16 && rows >= sm &&
+        (uint64_t)rows * 20 >= (uint64_t)sm * ((rows + sm - 1) / sm) * 17)
+        ver = 20;
     if (ver == 0) {
         if ((logN == 15 || logN == 16) && rows < sm / 4) ver = 5;        // v5: the row in a cluster's DSMEM
         else if (rows >= sm || logN >= 15) ver = 8;
