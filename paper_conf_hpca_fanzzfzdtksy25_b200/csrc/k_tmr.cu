@@ -1,5 +1,5 @@
-// k_tmr.cu -- launcher of the TMEM-resident CUDA-core NTT "tm" (N = 2^16; kernels in ntt_tmr.cuh,
-// DESIGN.md 5.1a).
+// k_tmr.cu -- launcher of the TMEM-resident CUDA-core NTT "tm" (N = 2^14..2^16; kernels in ntt_tmr.cuh
+// and ntt_tms.cuh).
 // This unit compiles the Harvey butterflies with their X + t / X + Y adds pinned to the ALU pipe
 // (modarith.cuh WD_BFLY_ALU: min(x + t, 4q), one VIADDMNMX instead of an IMAD.IADD on the fma pipe).
 // In the TMEM-resident kernel the fma pipe is the busiest one (ncu math_pipe_throttle); measured on
@@ -10,33 +10,49 @@
 #include <algorithm>
 #include <cstring>
 #include "launch.h"
-#include "ntt_tmr.cuh"
+#include "ntt_tms.cuh"
 
 namespace wd {
 
-int prep_tmr() {
-    for (auto k : {tmr::ntt_tmr16<true>, tmr::ntt_tmr16<false>}) {
-        if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, tmr::SMEM) != cudaSuccess ||
-            cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
-            return 4;
-    }
+namespace {
+template <typename K>
+int set_attr(K k, int smem) {
+    if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
+        cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+        return 4;
     return 0;
+}
+}  // namespace
+
+int prep_tmr() {
+    return set_attr(tmr::ntt_tmr16<true>, tmr::SMEM) | set_attr(tmr::ntt_tmr16<false>, tmr::SMEM) |
+           set_attr(tms::ntt_tms<2, true>, tms::SMEM) | set_attr(tms::ntt_tms<2, false>, tms::SMEM) |
+           set_attr(tms::ntt_tms<3, true>, tms::SMEM) | set_attr(tms::ntt_tms<3, false>, tms::SMEM);
 }
 
 // plain transforms only (contiguous [batch][L][N] rows, no pointwise product / store maps / copies);
 // returns launches (1), -1 if the arguments need v8, -2 if the tensor map cannot be encoded
-int launch_tmr(bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
-    if (a.in2 || a.aux || a.cpy || a.in_ls || a.out_ls || rows % a.L) return -1;
+int launch_tmr(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
+    if (logN < 14 || logN > 16 || a.in2 || a.aux || a.cpy || a.in_ls || a.out_ls || rows % a.L) return -1;
+    const uint32_t R = 1u << (logN - 12);
     alignas(64) CUtensorMap tm;
     std::memset(&tm, 0, sizeof(tm));
-    if (fwd) {   // the column passes: inner dimension the 4096 columns, one line per (row, k); box 256 x 16
-        const cuuint64_t dims[2] = {tmr::SUBW, (cuuint64_t)rows * 16}, strides[1] = {tmr::SUBW * 4};
-        const cuuint32_t box[2] = {tmr::TT, 16};
+    if (fwd) {   // the column passes: inner dimension the 4096 columns, one line per (row, k); box 256 x R
+        const cuuint64_t dims[2] = {tmr::SUBW, (cuuint64_t)rows * R}, strides[1] = {tmr::SUBW * 4};
+        const cuuint32_t box[2] = {tmr::TT, R};
         if (!tma_encode_u32(&tm, a.in, 2, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_NONE)) return -2;
     }
     const uint32_t grid = std::min<uint32_t>(rows, (uint32_t)sm_count);
-    if (fwd) tmr::ntt_tmr16<true><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows, tm);
-    else tmr::ntt_tmr16<false><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows, tm);
+    if (logN == 16) {
+        if (fwd) tmr::ntt_tmr16<true><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows, tm);
+        else tmr::ntt_tmr16<false><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows, tm);
+    } else if (logN == 15) {
+        if (fwd) tms::ntt_tms<3, true><<<grid, tmr::NT, tms::SMEM, s>>>(a, rows, tm);
+        else tms::ntt_tms<3, false><<<grid, tmr::NT, tms::SMEM, s>>>(a, rows, tm);
+    } else {
+        if (fwd) tms::ntt_tms<2, true><<<grid, tmr::NT, tms::SMEM, s>>>(a, rows, tm);
+        else tms::ntt_tms<2, false><<<grid, tmr::NT, tms::SMEM, s>>>(a, rows, tm);
+    }
     return 1;
 }
 

@@ -119,11 +119,13 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     const uint32_t logN = p->logN, sm = (uint32_t)p->sm_count;
     if (logN < 12) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "small"; return 1; }
     int ver = p->kernel_ver;
-    // N = 2^16: tm, the TMEM-resident kernel (one CTA per SM, one row in flight per SM), when its rounds
-    // of SM-count rows are at least 85% full; a last round with fewer rows leaves whole SMs idle, while
-    // v8's 4 CTAs per SM absorb such a tail (scripts/gpu_tm_rows.sh: rows 148 / 296 / 444 / 4608 tm
-    // 1.19 / 1.06 / 1.06 / 1.08 x v8; rows 152 / 300 v8 1.22 / 1.12 x tm)
-    if (ver == 0 && logN == 16 && rows >= sm &&
+    // N = 2^15, 2^16: tm, the TMEM-resident kernels (one CTA per SM, one (2^16) or two (2^15) rows in
+    // flight per SM), when their rounds of SM-count rows are at least 85% full; a last round with fewer
+    // rows leaves whole SMs idle, while v8's 4 CTAs per SM absorb such a tail (scripts/gpu_tm_rows.sh,
+    // gpu_tm_rows2.sh: N = 2^16 rows 148 / 296 / 444 / 4608 tm 1.19 / 1.06 / 1.06 / 1.08 x v8, rows
+    // 152 / 300 v8 1.22 / 1.12 x tm; N = 2^15 rows 576 .. 9216 tm 1.02 - 1.04 x v8).  N = 2^14 keeps v8
+    // (tm within -0.4 .. +3%, selectable with WD_NTT_KERNEL=tm).
+    if (ver == 0 && (logN == 15 || logN == 16) && rows >= sm &&
         (uint64_t)rows * 20 >= (uint64_t)sm * ((rows + sm - 1) / sm) * 17)
         ver = 20;
     if (ver == 0) {
@@ -131,8 +133,8 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
         else if (rows >= sm || logN >= 15) ver = 8;
         else ver = 1;                                                   // N <= 2^14, few rows
     }
-    if (ver == 20 && logN == 16) {                                     // tm: TMEM-resident rows
-        const int n = launch_tmr(fwd, a, rows, p->sm_count, s);
+    if (ver == 20 && logN >= 14 && logN <= 16) {                      // tm: TMEM-resident rows
+        const int n = launch_tmr(logN, fwd, a, rows, p->sm_count, s);
         if (n > 0) { g_last_kernel = "tm"; return n; }
         ver = 8;
     }
@@ -460,7 +462,8 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (cudaStreamCreateWithFlags(&p->fs, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->fe) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     if (prep_cc(p->logN) || prep_v8(p->logN, p->sm_count, &p->occ) || prep_rns() ||
-        (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4() || prep_tmr()))) {
+        (p->logN >= 14 && p->logN <= 16 && prep_tmr()) ||
+        (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4()))) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
     p->mode = WD_MODE_AUTO;

@@ -1,6 +1,6 @@
-"""A/B of the TMEM-resident kernel "tm" against v8 at N = 2^16: bit-exact agreement (and sampled rows vs
-the oracle) at several batch sizes, in place, then forward / inverse ms of both at config 3.
-usage: python scripts/tm_check.py [L] [reps]"""
+"""A/B of the TMEM-resident kernel "tm" against v8 (N = 2^16 by default): bit-exact agreement (and
+sampled rows vs the oracle) at several batch sizes, in place, then forward / inverse ms of both at
+128 polynomials.  usage: python scripts/tm_check.py [L] [reps] [logN]"""
 import os
 import sys
 
@@ -13,7 +13,8 @@ from paper_conf_hpca_fanzzfzdtksy25_b200 import inputs, wdntt  # noqa: E402
 
 L = int(sys.argv[1]) if len(sys.argv) > 1 else 36
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 20
-n = 1 << 16
+logn = int(sys.argv[3]) if len(sys.argv) > 3 else 16
+n = 1 << logn
 primes = inputs.bench_primes(L)
 
 
@@ -49,6 +50,7 @@ for b in (1, 2, 3, 5, 128):
     wdntt.wd_ntt_inverse(pt.handle, w, w, b, sp)
     torch.cuda.synchronize()
     ip_i = torch.equal(w, x)
+    assert wdntt.wd_ntt_last_kernel() == "tm", wdntt.wd_ntt_last_kernel()
     print("batch %3d: fwd==v8 %s  roundtrip %s  oracle fwd %s inv %s  in-place fwd %s inv %s" % (
         b, f_eq, rt, o_ok, oi_ok, ip_f, ip_i), flush=True)
     ok &= f_eq and rt and o_ok and oi_ok and ip_f and ip_i
@@ -77,5 +79,5 @@ def timeit(plan, b):
 for b in (128, 2):
     for name, pl in (("v8", p8), ("tm", pt), ("v8", p8), ("tm", pt)):
         f, i, k = timeit(pl, b)
-        print("%s batch %3d L %d: fwd %.4f ms inv %.4f ms KOPS %.0f" % (name, b, L, f, i, k), flush=True)
+        print("%s logN %d batch %3d L %d: fwd %.4f ms inv %.4f ms KOPS %.0f" % (name, logn, b, L, f, i, k), flush=True)
 print("ALL OK" if ok else "MISMATCH")
