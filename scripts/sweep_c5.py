@@ -34,6 +34,7 @@ def main():
                 y, z = torch.empty_like(x), torch.empty_like(x)
                 for _ in range(2):
                     wdntt.wd_ntt_forward(plan.handle, x, y, b, sp)
+                    kern = wdntt.wd_ntt_last_kernel()
                     wdntt.wd_ntt_inverse(plan.handle, y, z, b, sp)
                 torch.cuda.synchronize()
                 assert torch.equal(z, x), (logn, L, nct)
@@ -61,7 +62,7 @@ def main():
                 fms = ev[0].elapsed_time(ev[1]) / args.reps
                 ims = ev[1].elapsed_time(ev[2]) / args.reps
                 rows = b * L
-                print(json.dumps({"logN": logn, "L": L, "ciphertexts": nct, "rows": rows,
+                print(json.dumps({"logN": logn, "L": L, "ciphertexts": nct, "rows": rows, "kernel": kern,
                                   "fwd_ms": fms, "inv_ms": ims,
                                   "fwd_kops": rows / fms, "inv_kops": rows / ims,
                                   "hbm_frac_fwd": rows * 8.0 * n / (fms * 1e-3) / 1e9 / peak,
