@@ -11,11 +11,12 @@
 // of ntt_tmr.cuh: one CTA per SM, four teams of 256 threads; team tau owns sub-rows tau + 4 i (R / 4 of
 // them per row) and column passes tau + 4 i (four per row, in steps of 16 / R passes per sub-row).
 //   forward, row j:  R1(j, s) [stage 1 from slot j & 1]  C(j+1, ...) [TMA staging -> layers 0..A-1 ->
-//                    slot (j+1) & 1]  team barrier  R23(j, s) [stages 2, 3 -> out]; one CTA barrier per row
+//                    slot (j+1) & 1]  team barrier  R23(j, s) [stages 2, 3 -> out]
 //   inverse, row j:  C'(j, ...) [slot j & 1 -> layers A-1..0 with N^-1 -> out]  R'(j+1, s) [cp.async ->
-//                    stages 3', 2' -> team barrier -> stage 1' -> slot (j+1) & 1]; one CTA barrier per row
-// The CTA barrier per row orders both the row handoff (every column pass / sub-row of the next row is in
-// TMEM before it is read) and the slot reuse (row j's cells are read before row j + 2 overwrites them).
+//                    stages 3', 2' -> team barrier -> stage 1' -> slot (j+1) & 1]
+// Two CTA mbarriers order the row handoff (every column pass / sub-row of row j is in TMEM before it is
+// read) and the slot reuse (every warp has read row j - 1 before row j + 1 overwrites its slot), so
+// teams may drift apart by up to a row.
 #pragma once
 #include "ntt_tmr.cuh"
 
@@ -23,7 +24,7 @@ namespace wd {
 namespace tms {
 
 using tmr::TEAMS; using tmr::TT; using tmr::NT; using tmr::SUBW; using tmr::TWW; using tmr::TEAM_W;
-constexpr int SMEM = TEAMS * TEAM_W * 4 + 320;   // + 9 mbarriers per team + the TMEM base slot
+constexpr int SMEM = TEAMS * TEAM_W * 4 + 320;   // + 9 mbarriers per team, 2 CTA mbarriers, the TMEM slot
 
 // 16 cells at column offsets ta + R a, a = 0..15 (complete on return: the wait carries x as in/out
 // operands, so no use of x is scheduled before it)
@@ -94,7 +95,10 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
     auto TWB = [&](int b) { return reinterpret_cast<uint2*>(TS + 3 * SUBW + b * TWW); };
     // per team: tbar[0..NB-1] the forward TMA stagings, tbar[8] "B0 free"
     uint64_t* tbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + 9 * team;
-    uint32_t* tslot = reinterpret_cast<uint32_t*>(reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + 9 * TEAMS);
+    // CTA: rowbar "every warp's part of row r is in TMEM", slotbar "every warp has read row r's slot"
+    uint64_t* rowbar = reinterpret_cast<uint64_t*>(smem + TEAMS * TEAM_W) + 9 * TEAMS;
+    uint64_t* slotbar = rowbar + 1;
+    uint32_t* tslot = reinterpret_cast<uint32_t*>(rowbar + 2);
 
     if (threadIdx.x < 32) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" :: "r"(smem_u32(tslot)));
@@ -103,12 +107,24 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
     if (t == 0) {
         for (int i = 0; i < NB; ++i) mb_init(tbar + i, 1);
         mb_init(tbar + 8, TT / 32);
+        if (team == 0) { mb_init(rowbar, NT / 32); mb_init(slotbar, NT / 32); }
         mb_init_fence();
     }
     tmr::tfence_before();
     __syncthreads();
     tmr::tfence_after();
     const uint32_t tl = *tslot + ((uint32_t)(32 * (w & 3)) << 16) + 256u * h;   // lane quadrant, column half
+    // this warp's earlier TMEM accesses are complete and ordered before its arrival on b
+    auto warp_arrive_tmem = [&](uint64_t* b) {
+        tmr::tm_wait_st();
+        tmr::tfence_before();
+        __syncwarp();
+        if (lane == 0) mb_arrive(b);
+    };
+    auto wait_tmem = [&](uint64_t* b, uint32_t r) {   // phase r of b completed; later TMEM accesses after it
+        mb_wait(b, r & 1);
+        tmr::tfence_after();
+    };
 
     const uint32_t G = gridDim.x;
     const uint32_t nrow = rows > blockIdx.x ? (rows - blockIdx.x + G - 1) / G : 0;
@@ -165,7 +181,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                         if (mm < mtot) issue_col(mm, (mm >> 2) == 0 ? rwc : (mm >> 2) == 1 ? rwn : row_of(mm >> 2));
                     }
             }
-            tmr::cta_sync_tmem();
+            warp_arrive_tmem(rowbar);                    // this warp's passes of row 0 are in TMEM
 #pragma unroll 1
             for (uint32_t j = 0; j < nrow; ++j) {
                 const bool more = j + 1 < nrow;
@@ -181,6 +197,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                     cp_async_wait<0>();
                     __syncwarp();                        // this warp's stage-1 twiddles landed
                     uint32_t x[16];
+                    if (i == 0) wait_tmem(rowbar, j);    // every column pass of row j is in TMEM
                     ld16_stride<R>(tl + SLOT * (j & 1) + s, x);
                     {
                         const uint2* W = TWB(u & 1) + 16 * w;
@@ -192,10 +209,16 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                     // ---- C(j+1, ...): the step's PPS column passes of the next row
                     const uint32_t m0 = 4 * (j + 1) + i * PPS;
                     if (more) {
+                        // slot (j + 1) & 1 last held row j - 1: every warp has read it
+                        if (i == 0 && j > 0) wait_tmem(slotbar, j - 1);
 #pragma unroll 1
                         for (uint32_t q = 0; q < (uint32_t)PPS; ++q) colpass(m0 + q, lbn);
+                        if (i == NST - 1) warp_arrive_tmem(rowbar);   // this warp's passes of row j + 1
                     }
                     tmr::team_bar(team);                 // stage 1 (and the step's passes) done team-wide
+                    // this warp's reads of row j's slot are done (arrived only after this row's slot wait,
+                    // so a waiter never sees the barrier two phases ahead)
+                    if (i == NST - 1) warp_arrive_tmem(slotbar);
                     if (t == 0 && more)
                         for (uint32_t q = 0; q < (uint32_t)PPS; ++q) {
                             const uint32_t mm = m0 + NB + q;
@@ -255,7 +278,6 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                 }
                 lbc = lbn; rwc = rwn;
                 if (j + 2 < nrow) { lbn = limb_of(j + 2); rwn = r2; }
-                tmr::cta_sync_tmem();                    // row j + 1 in TMEM; slot j & 1 consumed
             }
         } else {
             // sub-row s of row jr: stages 3', 2' (team barrier) stage 1' into slot jr & 1
@@ -331,19 +353,27 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
             cp_async_commit();
 #pragma unroll 1
             for (int i = 0; i < NST; ++i) rowpass(0, team + 4 * i, lbc, rwc, lbn, rwn, i);
-            tmr::cta_sync_tmem();
+            warp_arrive_tmem(rowbar);                    // this warp's sub-rows of row 0 are in TMEM
 #pragma unroll 1
             for (uint32_t j = 0; j < nrow; ++j) {
                 const bool more = j + 1 < nrow;
                 const uint32_t lb2 = j + 2 < nrow ? limb_of(j + 2) : 0, rw2 = j + 2 < nrow ? row_of(j + 2) : 0;
 #pragma unroll 1
                 for (int i = 0; i < NST; ++i) {
+                    if (i == 0) wait_tmem(rowbar, j);    // every sub-row of row j is in TMEM
 #pragma unroll 1
                     for (int q = 0; q < PPS; ++q) colpass(j, team + 4 * (i * PPS + q), lbc, rwc);
-                    if (more) rowpass(j + 1, team + 4 * i, lbn, rwn, lb2, rw2, i);
+                    if (more) {
+                        // slot (j + 1) & 1 last held row j - 1: every warp has read it
+                        if (i == 0 && j > 0) wait_tmem(slotbar, j - 1);
+                        rowpass(j + 1, team + 4 * i, lbn, rwn, lb2, rw2, i);
+                    }
                 }
+                // this warp's sub-rows of row j + 1 are in TMEM, and its reads of row j are done (both
+                // arrivals after this row's waits, so a waiter never sees a barrier two phases ahead)
+                if (more) warp_arrive_tmem(rowbar);
+                warp_arrive_tmem(slotbar);
                 lbc = lbn; rwc = rwn; lbn = lb2; rwn = rw2;
-                tmr::cta_sync_tmem();                    // row j + 1 in TMEM; slot j & 1 consumed
             }
         }
     }
