@@ -119,13 +119,13 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     const uint32_t logN = p->logN, sm = (uint32_t)p->sm_count;
     if (logN < 12) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "small"; return 1; }
     int ver = p->kernel_ver;
-    // N = 2^15, 2^16: tm, the TMEM-resident kernels (one CTA per SM, one (2^16) or two (2^15) rows in
-    // flight per SM), when their rounds of SM-count rows are at least 85% full; a last round with fewer
-    // rows leaves whole SMs idle, while v8's 4 CTAs per SM absorb such a tail (scripts/gpu_tm_rows.sh,
-    // gpu_tm_rows2.sh: N = 2^16 rows 148 / 296 / 444 / 4608 tm 1.19 / 1.06 / 1.06 / 1.08 x v8, rows
-    // 152 / 300 v8 1.22 / 1.12 x tm; N = 2^15 rows 576 .. 9216 tm 1.02 - 1.04 x v8).  N = 2^14 keeps v8
-    // (tm within -0.4 .. +3%, selectable with WD_NTT_KERNEL=tm).
-    if (ver == 0 && (logN == 15 || logN == 16) && rows >= sm &&
+    // N = 2^14..2^16: tm, the TMEM-resident kernels (one CTA per SM, one (2^16) or two (2^14, 2^15) rows
+    // in flight per SM), when their rounds of SM-count rows are at least 85% full; a last round with
+    // fewer rows leaves whole SMs idle, while v8's 4 CTAs per SM absorb such a tail
+    // (scripts/gpu_tm_rows.sh, gpu_tm_rows2.sh: N = 2^16 rows 148 / 296 / 444 / 4608 tm 1.19 / 1.06 /
+    // 1.06 / 1.08 x v8, rows 152 / 300 v8 1.22 / 1.12 x tm; N = 2^15, 2^14 rows 576 .. 9216 tm 1.05 -
+    // 1.09 x v8, rows 216 v8 1.20 / 1.14 x tm)
+    if (ver == 0 && logN >= 14 && logN <= 16 && rows >= sm &&
         (uint64_t)rows * 20 >= (uint64_t)sm * ((rows + sm - 1) / sm) * 17)
         ver = 20;
     if (ver == 0) {

@@ -182,7 +182,7 @@ def test_config4_n131072_l48(wd):
 
 # -------------------------------------------------------------- AUTO's decision boundaries
 # AUTO picks the kernel (v1 / v5 / v8 / tm) and v8's cluster size (8, 4, 2, 1 CTAs per row) from N and
-# the row count, with thresholds at SM/4, SM/2, SM, 8 x SM rows and, at N = 2^15 / 2^16, the fill of tm's
+# the row count, with thresholds at SM/4, SM/2, SM, 8 x SM rows and, at N = 2^14..2^16, the fill of tm's
 # last round of SM-count rows (wd_ntt.cu launch_cuda_core).
 # Every N, every threshold +-1, every row of both directions against the oracle.
 def _boundary_rows():
@@ -201,7 +201,7 @@ def test_auto_decision_boundaries(wd, logn):
         plan = wd.Plan(n, primes)
         y = gpu_fwd(wd, plan, x)
         sm = torch.cuda.get_device_properties(0).multi_processor_count
-        tm_auto = logn in (15, 16) and rows >= sm and rows * 20 >= sm * (-(-rows // sm)) * 17   # rounds >= 85% full
+        tm_auto = 14 <= logn <= 16 and rows >= sm and rows * 20 >= sm * (-(-rows // sm)) * 17   # rounds >= 85% full
         assert (wd.wd_ntt_last_kernel() == "tm") == tm_auto, (logn, rows)
         assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, rows)
         assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (logn, rows)
@@ -337,8 +337,7 @@ def test_v8_column_feeds(wd, feed, logn, cl, monkeypatch):
     assert np.array_equal(to_host(t), x), (feed, logn, cl)
 
 
-# tm, the TMEM-resident kernels (WD_NTT_KERNEL=tm at N = 2^14..2^16; AUTO at N = 2^15, 2^16 from SM-count
-# rows on): fewer rows than
+# tm, the TMEM-resident kernels (WD_NTT_KERNEL=tm; AUTO at N = 2^14..2^16 from SM-count rows on): fewer rows than
 # SMs (idle CTAs), one row, ragged row counts against the SM count (CTAs with one row more than others),
 # both layouts of the TMEM ping-pong (odd and even rows per CTA), the natural row order (WD_NTT_LM=0),
 # edge inputs, in place; every row of both directions against the oracle
