@@ -29,8 +29,8 @@ void launch_v8(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int cl,
 int prep_wdcuda();
 void launch_wdcuda(bool fwd, const NttArgs& a, const TensorTables& tc, uint32_t rows, int sm_count, cudaStream_t s);
 
-// ---- k_tmr.cu: "tm", the TMEM-resident CUDA-core kernels (N = 2^14..2^16, plain transforms;
-//      ntt_tmr.cuh, ntt_tms.cuh)
+// ---- k_tmr.cu: "tm", the TMEM-resident CUDA-core kernels (N = 2^13..2^16, plain transforms;
+//      ntt_tmr.cuh, ntt_tms.cuh, ntt_tmt.cuh)
 int prep_tmr();
 // returns launches (1), -1 if the size or the arguments need v8 (pointwise product, store maps, strided
 // rows), -2 if the tensor map cannot be encoded

@@ -45,4 +45,10 @@ __device__ __forceinline__ void tma2_load_hint(void* dst, const CUtensorMap* m, 
                  " [%0], [%1, {%2, %3}], [%4], %5;"
                  :: "r"(smem_u32(dst)), "l"(m), "r"(c0), "r"(c1), "r"(smem_u32(b)), "l"(pol) : "memory");
 }
+__device__ __forceinline__ void tma3_load_hint(void* dst, const CUtensorMap* m, int c0, int c1, int c2, uint64_t* b,
+                                               uint64_t pol) {
+    asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                 " [%0], [%1, {%2, %3, %4}], [%5], %6;"
+                 :: "r"(smem_u32(dst)), "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(b)), "l"(pol) : "memory");
+}
 }  // namespace wd

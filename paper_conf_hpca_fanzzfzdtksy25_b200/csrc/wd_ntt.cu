@@ -119,21 +119,22 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     const uint32_t logN = p->logN, sm = (uint32_t)p->sm_count;
     if (logN < 12) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "small"; return 1; }
     int ver = p->kernel_ver;
-    // N = 2^14..2^16: tm, the TMEM-resident kernels (one CTA per SM, one (2^16) or two (2^14, 2^15) rows
-    // in flight per SM), when their rounds of SM-count rows are at least 85% full; a last round with
-    // fewer rows leaves whole SMs idle, while v8's 4 CTAs per SM absorb such a tail
-    // (scripts/gpu_tm_rows.sh, gpu_tm_rows2.sh: N = 2^16 rows 148 / 296 / 444 / 4608 tm 1.19 / 1.06 /
-    // 1.06 / 1.08 x v8, rows 152 / 300 v8 1.22 / 1.12 x tm; N = 2^15, 2^14 rows 576 .. 9216 tm 1.05 -
-    // 1.09 x v8, rows 216 v8 1.20 / 1.14 x tm)
-    if (ver == 0 && logN >= 14 && logN <= 16 && rows >= sm &&
-        (uint64_t)rows * 20 >= (uint64_t)sm * ((rows + sm - 1) / sm) * 17)
-        ver = 20;
+    // N = 2^13..2^16: tm, the TMEM-resident kernels, when their rounds of rows are at least 85% full.
+    // A round is one row per SM (2^14..2^16: one CTA per SM, one or two rows in flight) or four
+    // (2^13: one row per team); a last round with fewer rows leaves whole SMs idle, while v8's 4 CTAs
+    // per SM absorb such a tail (scripts/gpu_tm_rows*.sh, profiles/r02/tm/: at filled row counts tm is
+    // 1.05 - 1.19 x v8 at 2^14..2^16 and 1.09 - 1.15 x at 2^13; rows 152 / 300 at 2^16, 216 at
+    // 2^14 / 2^15 and 648 at 2^13 favour v8)
+    if (ver == 0 && logN >= 13 && logN <= 16) {
+        const uint64_t unit = (uint64_t)sm * (logN == 13 ? 4 : 1);
+        if ((uint64_t)rows * 20 >= unit * ((rows + unit - 1) / unit) * 17) ver = 20;
+    }
     if (ver == 0) {
         if ((logN == 15 || logN == 16) && rows < sm / 4) ver = 5;        // v5: the row in a cluster's DSMEM
         else if (rows >= sm || logN >= 15) ver = 8;
         else ver = 1;                                                   // N <= 2^14, few rows
     }
-    if (ver == 20 && logN >= 14 && logN <= 16) {                      // tm: TMEM-resident rows
+    if (ver == 20 && logN >= 13 && logN <= 16) {                      // tm: TMEM-resident rows
         const int n = launch_tmr(logN, fwd, a, rows, p->sm_count, s);
         if (n > 0) { g_last_kernel = "tm"; return n; }
         ver = 8;
@@ -462,7 +463,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (cudaStreamCreateWithFlags(&p->fs, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->fe) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     if (prep_cc(p->logN) || prep_v8(p->logN, p->sm_count, &p->occ) || prep_rns() ||
-        (p->logN >= 14 && p->logN <= 16 && prep_tmr()) ||
+        (p->logN >= 13 && p->logN <= 16 && prep_tmr()) ||
         (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4()))) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }

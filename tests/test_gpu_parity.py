@@ -182,13 +182,13 @@ def test_config4_n131072_l48(wd):
 
 # -------------------------------------------------------------- AUTO's decision boundaries
 # AUTO picks the kernel (v1 / v5 / v8 / tm) and v8's cluster size (8, 4, 2, 1 CTAs per row) from N and
-# the row count, with thresholds at SM/4, SM/2, SM, 8 x SM rows and, at N = 2^14..2^16, the fill of tm's
+# the row count, with thresholds at SM/4, SM/2, SM, 8 x SM rows and, at N = 2^13..2^16, the fill of tm's
 # last round of SM-count rows (wd_ntt.cu launch_cuda_core).
 # Every N, every threshold +-1, every row of both directions against the oracle.
 def _boundary_rows():
     sm = torch.cuda.get_device_properties(0).multi_processor_count if torch.cuda.is_available() else 148
     pts = {1, sm // 4 - 1, sm // 4, sm // 2, sm // 2 + 1, sm - 1, sm, sm + 1, 2 * sm - 1, 2 * sm, 2 * sm + 1,
-           8 * sm - 1, 8 * sm}
+           4 * sm - 1, 4 * sm, 4 * sm + 1, 8 * sm - 1, 8 * sm}
     return sorted(pts)
 
 
@@ -201,7 +201,8 @@ def test_auto_decision_boundaries(wd, logn):
         plan = wd.Plan(n, primes)
         y = gpu_fwd(wd, plan, x)
         sm = torch.cuda.get_device_properties(0).multi_processor_count
-        tm_auto = 14 <= logn <= 16 and rows >= sm and rows * 20 >= sm * (-(-rows // sm)) * 17   # rounds >= 85% full
+        unit = sm * (4 if logn == 13 else 1)     # tm processes rows in rounds of `unit`
+        tm_auto = 13 <= logn <= 16 and rows * 20 >= unit * (-(-rows // unit)) * 17   # rounds >= 85% full
         assert (wd.wd_ntt_last_kernel() == "tm") == tm_auto, (logn, rows)
         assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, rows)
         assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (logn, rows)
@@ -337,14 +338,15 @@ def test_v8_column_feeds(wd, feed, logn, cl, monkeypatch):
     assert np.array_equal(to_host(t), x), (feed, logn, cl)
 
 
-# tm, the TMEM-resident kernels (WD_NTT_KERNEL=tm; AUTO at N = 2^14..2^16 from SM-count rows on): fewer rows than
+# tm, the TMEM-resident kernels (WD_NTT_KERNEL=tm; AUTO at N = 2^13..2^16 when its row rounds are full): fewer rows than
 # SMs (idle CTAs), one row, ragged row counts against the SM count (CTAs with one row more than others),
 # both layouts of the TMEM ping-pong (odd and even rows per CTA), the natural row order (WD_NTT_LM=0),
 # edge inputs, in place; every row of both directions against the oracle
 @pytest.mark.parametrize("logn,L,batch,lm", [(16, 1, 1, "1"), (16, 3, 1, "1"), (16, 36, 5, "1"), (16, 4, 83, "1"),
                                              (16, 60, 7, "1"), (16, 5, 61, "0"), (16, 36, 9, "0"),
                                              (15, 1, 1, "1"), (15, 36, 5, "1"), (15, 4, 83, "1"), (15, 5, 61, "0"),
-                                             (14, 2, 1, "1"), (14, 36, 9, "1"), (14, 7, 100, "1"), (14, 3, 97, "0")])
+                                             (14, 2, 1, "1"), (14, 36, 9, "1"), (14, 7, 100, "1"), (14, 3, 97, "0"),
+                                             (13, 1, 1, "1"), (13, 36, 9, "1"), (13, 5, 150, "1"), (13, 3, 211, "0")])
 def test_tm_kernel(wd, logn, L, batch, lm, monkeypatch):
     monkeypatch.setenv("WD_NTT_KERNEL", "tm")
     monkeypatch.setenv("WD_NTT_LM", lm)
