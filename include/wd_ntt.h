@@ -53,8 +53,12 @@ typedef struct CUstream_st* wd_stream_t;       /* == cudaStream_t */
 #define WD_ENOMEM        5   /* device or host allocation failed                        */
 
 /* execution modes (wd_ntt_plan_set_mode) */
-#define WD_MODE_AUTO     0   /* library default for this N                              */
-#define WD_MODE_CUDA     1   /* CUDA-core radix-2^k butterflies only (WD-BO role)       */
+#define WD_MODE_AUTO     0   /* library default for this N: = WD_MODE_CUDA on B200       */
+#define WD_MODE_CUDA     1   /* CUDA-core radix-2^k butterflies only (WD-BO role): the     *
+                              * TMEM-resident kernels "tm" at N = 2^13..2^16 when their    *
+                              * rounds of rows are >= 85% full (one row per SM, four per   *
+                              * SM at 2^13), else v8 / v5 / v1 (wd_ntt_last_kernel names   *
+                              * the one a call ran)                   */
 #define WD_MODE_TENSOR   2   /* tcgen05 kind::i8 inner DFTs + CUDA-core epilogue        */
 #define WD_MODE_FUSED    3   /* both paths concurrently on the same SMs (WD-FUSE role)  */
 #define WD_MODE_CUDA_GEMM 4  /* inner DFTs as 32-bit GEMMs on the CUDA cores (WD-CUDA,   *
