@@ -27,6 +27,11 @@ struct NttArgs {
     uint32_t* cpy = nullptr;
     uint32_t cpy_ls = 0;
     uint32_t limb_major = 0;         // v8: walk rows limb by limb (rows must be a multiple of L)
+    // a launch over a part of a bigger batch's schedule (tm + v8 tail, wd_ntt.cu launch_cuda_core): the
+    // launch covers schedule slots slot0 .. slot0 + rows - 1 of a batch of nb_total polynomials (0: the
+    // launch's own rows / L); the slot -> row map (limb-major) is the whole batch's
+    uint32_t slot0 = 0;
+    uint32_t nb_total = 0;
 };
 
 __device__ __forceinline__ uint32_t row_map(uint32_t row, uint32_t L, uint32_t ls) {

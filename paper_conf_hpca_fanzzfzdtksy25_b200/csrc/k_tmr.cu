@@ -34,17 +34,21 @@ int prep_tmr() {
 // plain transforms only (contiguous [batch][L][N] rows, no pointwise product / store maps / copies);
 // returns launches (1), -1 if the arguments need v8, -2 if the tensor map cannot be encoded
 int launch_tmr(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s) {
-    if (logN < 13 || logN > 16 || a.in2 || a.aux || a.cpy || a.in_ls || a.out_ls || rows % a.L) return -1;
+    // rows_all: the whole batch's rows (the launch may cover its first `rows` schedule slots only)
+    const uint64_t rows_all = a.nb_total ? (uint64_t)a.nb_total * a.L : rows;
+    if (logN < 13 || logN > 16 || a.in2 || a.aux || a.cpy || a.in_ls || a.out_ls || rows_all % a.L || a.slot0 ||
+        rows > rows_all)
+        return -1;                               // (the tm kernels start at schedule slot 0)
     const uint32_t R = 1u << (logN - 12);
     alignas(64) CUtensorMap tm;
     std::memset(&tm, 0, sizeof(tm));
     if (fwd && logN == 13) {   // {256 columns, 16 passes, one line per (row, k)}; box: 8 passes x 2 lines
-        const cuuint64_t dims[3] = {tmr::TT, 16, (cuuint64_t)rows * R};
+        const cuuint64_t dims[3] = {tmr::TT, 16, (cuuint64_t)rows_all * R};
         const cuuint64_t strides[2] = {tmr::TT * 4, tmr::SUBW * 4};
         const cuuint32_t box[3] = {tmr::TT, 8, R};
         if (!tma_encode_u32(&tm, a.in, 3, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_NONE)) return -2;
     } else if (fwd) {   // the column passes: inner dimension the 4096 columns, one line per (row, k); box 256 x R
-        const cuuint64_t dims[2] = {tmr::SUBW, (cuuint64_t)rows * R}, strides[1] = {tmr::SUBW * 4};
+        const cuuint64_t dims[2] = {tmr::SUBW, (cuuint64_t)rows_all * R}, strides[1] = {tmr::SUBW * 4};
         const cuuint32_t box[2] = {tmr::TT, R};
         if (!tma_encode_u32(&tm, a.in, 2, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_NONE)) return -2;
     }

@@ -88,9 +88,9 @@ void launch_k(bool fwd, const NttArgs& a, uint32_t rows, int ncl, int tma, cudaS
         std::memset(&tm, 0, sizeof(tm));
         const int smem = V8_SMEM_K;
         if constexpr (tm_ok<LOGN>() && EPI == 0) {
-            if ((tma & 1) && fwd && encode_v8_cols(&tm, LOGN, a.in, a.in_ls, a.L, rows)) {
+            if ((tma & 1) && fwd && encode_v8_cols(&tm, LOGN, a.in, a.in_ls, a.L, a.nb_total ? a.nb_total * a.L : rows)) {
                 k = ntt_v8<LOGN, true, false, CL, 0, 1>;
-            } else if ((tma & 2) && !fwd && !a.in2 && encode_v8_cols(&tm, LOGN, a.out, a.out_ls, a.L, rows)) {
+            } else if ((tma & 2) && !fwd && !a.in2 && encode_v8_cols(&tm, LOGN, a.out, a.out_ls, a.L, a.nb_total ? a.nb_total * a.L : rows)) {
                 k = ntt_v8<LOGN, false, false, CL, 0, 1>;
             } else if ((tma & 4) && !fwd && !a.in2) {
                 k = ntt_v8<LOGN, false, false, CL, 0, 2>;

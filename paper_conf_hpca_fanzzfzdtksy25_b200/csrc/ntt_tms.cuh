@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
 
     const uint32_t G = gridDim.x;
     const uint32_t nrow = rows > blockIdx.x ? (rows - blockIdx.x + G - 1) / G : 0;
-    const uint32_t nb = rows / a.L;
+    const uint32_t nb = a.nb_total ? a.nb_total : rows / a.L;   // polynomials of the schedule
     auto limb_of = [&](uint32_t j) {
         const uint32_t sr = blockIdx.x + j * G;
         return a.limb_major ? sr / nb : sr % a.L;

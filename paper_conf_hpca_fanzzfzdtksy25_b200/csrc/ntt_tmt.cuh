@@ -64,11 +64,11 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
     auto vslot = [&](uint32_t j) { return 4 * blockIdx.x + (threadIdx.x >> 8) + j * 4 * gridDim.x; };
     const uint32_t nrow = rows > vslot(0) ? (rows - vslot(0) + 4 * gridDim.x - 1) / (4 * gridDim.x) : 0;
     auto limb_of = [&](uint32_t j) {
-        const uint32_t sr = vslot(j), nb = rows / a.L;
+        const uint32_t sr = vslot(j), nb = a.nb_total ? a.nb_total : rows / a.L;
         return a.limb_major ? sr / nb : sr % a.L;
     };
     auto row_of = [&](uint32_t j) {
-        const uint32_t sr = vslot(j), nb = rows / a.L;
+        const uint32_t sr = vslot(j), nb = a.nb_total ? a.nb_total : rows / a.L;
         if (!a.limb_major) return sr;
         const uint32_t lb = sr / nb;
         return (sr - lb * nb) * a.L + lb;

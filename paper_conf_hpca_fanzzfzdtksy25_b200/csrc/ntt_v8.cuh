@@ -239,7 +239,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
     const int t = threadIdx.x;
     const int hi4 = t >> 4, lo4 = t & 15;
 
-    const uint32_t nb = rows / a.L;              // polynomials in the launch
+    const uint32_t nb = a.nb_total ? a.nb_total : rows / a.L;   // polynomials of the schedule
+    const uint32_t send = a.slot0 + rows;        // the launch covers schedule slots slot0 .. send - 1
     static_assert(TM != 1 || (EPI == 0 && !PW && A >= 1 && R <= 16), "TMA column phase: EPI 0, no PW, 2 <= R <= 16");
     static_assert(TM != 2 || (!FWD && EPI == 0 && A >= 1), "early sub-row prefetch: inverse with a column phase");
     constexpr int PF = ((NS - 1) & 1) ^ 1;       // TM: the buffer free during a row's last sub-row
@@ -256,8 +257,8 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
         if (t == 0) {
             mb_init(&tbar[0], 1); mb_init(&tbar[1], 1);
             mb_init_fence();
-            const uint32_t sr = blockIdx.x / CL;
-            if (FWD && sr < rows) {              // the CTA's first column pass
+            const uint32_t sr = a.slot0 + blockIdx.x / CL;
+            if (FWD && sr < send) {              // the CTA's first column pass
                 mb_expect(&tbar[PF], R * V8_T * 4);
                 tma2_load_hint(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R), &tbar[PF],
                                l2_evict_first_policy());
@@ -267,7 +268,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
     }
     bool sub0_ready = false;                     // TM inverse: this row's first sub-row already requested
 #pragma unroll 1
-    for (uint32_t srow = blockIdx.x / CL; srow < rows; srow += gridDim.x / CL) {
+    for (uint32_t srow = a.slot0 + blockIdx.x / CL; srow < send; srow += gridDim.x / CL) {
         // limb-major schedule (a.limb_major): the rows in flight at any time share a few limbs,
         // so their twiddle tables (N x 8 bytes per limb and direction) stay a small part of L2
         // next to the L2-resident intermediates; the data layout is unchanged
@@ -353,7 +354,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                     v8_load_fwd_slice(smem + ((s + 1 - s0) & 1) * V8_SUBW, src + (s + 1) * V8_SUBW);
                 } else if constexpr (TM == 1) {               // the next row's first column pass
                     const uint32_t sr = srow + gridDim.x / CL;
-                    if (t == 0 && sr < rows) {
+                    if (t == 0 && sr < send) {
                         fence_proxy_async();
                         mb_expect(&tbar[PF], R * V8_T * 4);
                         tma2_load_hint(smem + PF * V8_SUBW, &tm_in, p0 * V8_T, (int)(row_map(map_row(sr), a.L, a.in_ls) * R),
@@ -506,7 +507,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                 const int orow = (int)(row_map(row, a.L, a.out_ls) * R);
                 if constexpr (TM == 2) {                 // the register-fed column phase leaves both buffers
                     const uint32_t sr = srow + gridDim.x / CL;     // idle: next row's first sub-row now
-                    if (sr < rows) {
+                    if (sr < send) {
                         const uint32_t nl = a.limb_major ? sr / nb : sr % a.L;
                         v8_tw_inv<A>(TWB(0), a.tw + ((size_t)nl << LOGN), s0);
                         v8_load_inv_slice(smem, a.in + ((size_t)row_map(map_row(sr), a.L, a.in_ls) << LOGN) + s0 * V8_SUBW);
@@ -539,7 +540,7 @@ __global__ void __launch_bounds__(V8_T, 4) ntt_v8(NttArgs a, uint32_t rows, cons
                         static_assert((NP & 1) == 0, "the last pass reads buffer 1: buffer 0 is free");
                         if (pass + 1 == p0 + NP) {            // the next row's first sub-row into buffer 0
                             const uint32_t sr = srow + gridDim.x / CL;
-                            if (sr < rows) {
+                            if (sr < send) {
                                 const uint32_t nl = a.limb_major ? sr / nb : sr % a.L;
                                 v8_tw_inv<A>(TWB(0), a.tw + ((size_t)nl << LOGN), s0);
                                 v8_load_inv_slice(smem, a.in + ((size_t)row_map(map_row(sr), a.L, a.in_ls) << LOGN) +

@@ -119,15 +119,19 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     const uint32_t logN = p->logN, sm = (uint32_t)p->sm_count;
     if (logN < 12) { launch_v1(logN, fwd, a, rows, s); g_last_kernel = "small"; return 1; }
     int ver = p->kernel_ver;
-    // N = 2^13..2^16: tm, the TMEM-resident kernels, when their rounds of rows are at least 85% full.
-    // A round is one row per SM (2^14..2^16: one CTA per SM, one or two rows in flight) or four
-    // (2^13: one row per team); a last round with fewer rows leaves whole SMs idle, while v8's 4 CTAs
-    // per SM absorb such a tail (scripts/gpu_tm_rows*.sh, profiles/r02/tm/: at filled row counts tm is
-    // 1.05 - 1.19 x v8 at 2^14..2^16 and 1.09 - 1.15 x at 2^13; rows 152 / 300 at 2^16, 216 at
-    // 2^14 / 2^15 and 648 at 2^13 favour v8)
+    // N = 2^13..2^16: tm, the TMEM-resident kernels.  They process rows in rounds of `unit` (one row per
+    // SM; four per SM at 2^13), so a last, partly filled round leaves SMs idle for a whole row time.
+    //  * a small remainder (<= unit / 4 rows): tm runs the full rounds and v8, with the most CTAs per row,
+    //    the remaining schedule slots right after it (the same limb-major slot -> row map);
+    //  * otherwise tm alone when its rounds are at least 85% full, else v8, whose 4 CTAs per SM absorb
+    //    such a tail (scripts/gpu_tm_rows*.sh, profiles/r02/tm/)
+    bool tm_tail = false;
+    uint64_t tm_unit = 0;
     if (ver == 0 && logN >= 13 && logN <= 16) {
-        const uint64_t unit = (uint64_t)sm * (logN == 13 ? 4 : 1);
-        if ((uint64_t)rows * 20 >= unit * ((rows + unit - 1) / unit) * 17) ver = 20;
+        tm_unit = (uint64_t)sm * (logN == 13 ? 4 : 1);
+        const uint64_t tail = rows % tm_unit;
+        if (rows >= tm_unit && tail * 4 <= tm_unit) { ver = 20; tm_tail = tail != 0; }
+        else if ((uint64_t)rows * 20 >= tm_unit * ((rows + tm_unit - 1) / tm_unit) * 17) ver = 20;
     }
     if (ver == 0) {
         if ((logN == 15 || logN == 16) && rows < sm / 4) ver = 5;        // v5: the row in a cluster's DSMEM
@@ -135,8 +139,22 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
         else ver = 1;                                                   // N <= 2^14, few rows
     }
     if (ver == 20 && logN >= 13 && logN <= 16) {                      // tm: TMEM-resident rows
-        const int n = launch_tmr(logN, fwd, a, rows, p->sm_count, s);
-        if (n > 0) { g_last_kernel = "tm"; return n; }
+        if (tm_tail) {
+            const uint32_t tail = (uint32_t)(rows % tm_unit);
+            NttArgs am = a;
+            am.nb_total = rows / a.L;                                   // the whole batch's slot map
+            const int n = launch_tmr(logN, fwd, am, rows - tail, p->sm_count, s);
+            if (n > 0) {
+                NttArgs at = am;
+                at.slot0 = rows - tail;
+                launch_v8(logN, fwd, at, tail, std::min(8, 1 << ((int)logN - 12)), 0, p->occ, p->v8_tma, s);
+                g_last_kernel = "tm+v8";
+                return n + 1;
+            }
+        } else {
+            const int n = launch_tmr(logN, fwd, a, rows, p->sm_count, s);
+            if (n > 0) { g_last_kernel = "tm"; return n; }
+        }
         ver = 8;
     }
     if (ver == 5 && logN >= 14) { launch_v5(logN, fwd, a, rows, p->sm_count, s); g_last_kernel = "v5"; return 1; }

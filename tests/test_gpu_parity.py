@@ -182,8 +182,8 @@ def test_config4_n131072_l48(wd):
 
 # -------------------------------------------------------------- AUTO's decision boundaries
 # AUTO picks the kernel (v1 / v5 / v8 / tm) and v8's cluster size (8, 4, 2, 1 CTAs per row) from N and
-# the row count, with thresholds at SM/4, SM/2, SM, 8 x SM rows and, at N = 2^13..2^16, the fill of tm's
-# last round of SM-count rows (wd_ntt.cu launch_cuda_core).
+# the row count, with thresholds at SM/4, SM/2, SM, 8 x SM rows and, at N = 2^13..2^16, tm's rounds of
+# rows: full rounds with a small remainder run as tm + a v8 tail launch (wd_ntt.cu launch_cuda_core).
 # Every N, every threshold +-1, every row of both directions against the oracle.
 def _boundary_rows():
     sm = torch.cuda.get_device_properties(0).multi_processor_count if torch.cuda.is_available() else 148
@@ -202,11 +202,40 @@ def test_auto_decision_boundaries(wd, logn):
         y = gpu_fwd(wd, plan, x)
         sm = torch.cuda.get_device_properties(0).multi_processor_count
         unit = sm * (4 if logn == 13 else 1)     # tm processes rows in rounds of `unit`
-        tm_auto = 13 <= logn <= 16 and rows * 20 >= unit * (-(-rows // unit)) * 17   # rounds >= 85% full
-        assert (wd.wd_ntt_last_kernel() == "tm") == tm_auto, (logn, rows)
+        tail = rows % unit
+        split = 13 <= logn <= 16 and rows >= unit and tail * 4 <= unit          # full rounds + v8 tail
+        tm_alone = 13 <= logn <= 16 and not split and rows * 20 >= unit * (-(-rows // unit)) * 17
+        want = "tm+v8" if split and tail else "tm" if split or tm_alone else None
+        got = wd.wd_ntt_last_kernel()
+        assert (got == want) if want else not got.startswith("tm"), (logn, rows, got)
         assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, rows)
         assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (logn, rows)
         plan.close()
+
+
+# AUTO's tm + v8-tail split (full rounds of rows on tm, a remainder <= a quarter round on v8 with the
+# same limb-major slot map) at row counts that are not multiples of L's: every row of both directions
+@pytest.mark.parametrize("logn,L,batch", [(16, 36, 5), (16, 7, 43), (15, 5, 61), (14, 9, 33), (13, 11, 55)])
+def test_auto_tm_tail_split(wd, logn, L, batch):
+    n = 1 << logn
+    sm = torch.cuda.get_device_properties(0).multi_processor_count
+    unit = sm * (4 if logn == 13 else 1)
+    rows = batch * L
+    primes = [P[(11 * i + L) % 60] for i in range(L)]
+    x = inputs.uniform_residues(primes, n, batch, 5900 + logn * 7 + batch)
+    plan = wd.Plan(n, primes)
+    y = gpu_fwd(wd, plan, x)
+    tail = rows % unit
+    if rows >= unit and 0 < tail * 4 <= unit:
+        assert wd.wd_ntt_last_kernel() == "tm+v8", (logn, rows)
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, L, batch)
+    assert np.array_equal(gpu_inv(wd, plan, x), oracle.ntt_inverse(x, primes)), (logn, L, batch)
+    t = to_dev(x)
+    plan.forward(t, t)                                   # in place
+    plan.inverse(t, t)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(t), x), (logn, L, batch)
+    plan.close()
 
 
 @pytest.mark.parametrize("logn,L", [(12, 1), (13, 60), (14, 17), (15, 9), (16, 60), (17, 2)])
