@@ -8,7 +8,7 @@ mkdir -p gpurun_out
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"ntt|rns|tc4" -c 400 --csv --log-file gpurun_out/launches_$TAG.csv \
   python bench.py --steps 2 --warmup 1 --no-cpu --e2e-steps 0 > gpurun_out/launches_${TAG}_bench.txt 2>&1
 echo "launch list rc=$?"
-timeout 900 ncu --set full --import-source on --clock-control none -k regex:"ntt_v8|ntt_tmr" -s 2 -c 2 -o gpurun_out/prof_$TAG \
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:"ntt_v8|ntt_tmr" -s 4 -c 4 -o gpurun_out/prof_$TAG \
   python scripts/one_step.py 128 auto > gpurun_out/prof_${TAG}_run.txt 2>&1
 echo "full rc=$?"
 python scripts/ncu_summary.py gpurun_out/prof_$TAG.ncu-rep > gpurun_out/ncu_$TAG.txt 2>&1
