@@ -157,6 +157,85 @@ __device__ __forceinline__ void load_inv_slice(uint32_t* S, const uint32_t* src,
 }
 
 // the forward twiddle areas / stage bodies shared by the two directions are written out in each branch
+// ---------------------------------------------------------------- row-phase stages shared by the tm kernels
+// v8's sub-row layout (ntt_v8.cuh v8_phys) in a 4096-word shared-memory buffer S; team thread t.
+// Forward stages 2 (twiddles T2 = the sub-row's stage-2 area) and 3 (twiddles w3), then the coalesced
+// canonical store of the sub-row to out and this warp's arrival on b0free (its last read of S).
+__device__ __forceinline__ void fwd_stages23(uint32_t* S, uint32_t* x, const uint2* T2, const uint2* w3, uint32_t q,
+                                             uint32_t q2, uint32_t* out, int t, uint64_t* b0free) {
+    const int hi4 = t >> 4, lo4 = t & 15, w = t >> 5, lane = t & 31;
+    {   // stage 2: thread (a, c), elements b
+        const int aa = hi4, c = lo4;
+#pragma unroll
+        for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(aa, k, c)];
+        fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, q, q2);
+#pragma unroll
+        for (int k = 0; k < 16; ++k) S[v8_phys(aa, k, c)] = x[k];
+    }
+    __syncwarp();
+    {   // stage 3: thread (a, b), 16 contiguous elements; coalesced store through the warp's own slots
+        const int aa = hi4, b = lo4;
+        uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+        const int sw = (b >> 1) & 3;
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+            x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
+        }
+        fwd16_tw(x, w3, q, q2);
+#pragma unroll
+        for (int v = 0; v < 4; ++v)
+            *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) = make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+        __syncwarp();
+        const int wbase = w * 512 + 4 * lane;
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const int e = wbase + 128 * v;
+            const uint4 r = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
+            __stcs(reinterpret_cast<uint4*>(out + e),
+                   make_uint4(canon4(r.x, q, q2), canon4(r.y, q, q2), canon4(r.z, q, q2), canon4(r.w, q, q2)));
+        }
+        __syncwarp();
+        if (lane == 0) mb_arrive(b0free);
+    }
+}
+// Inverse stages 3' (twiddles w3) and 2' (this warp's twiddle copies in TW, tw_inv's layout) in S
+__device__ __forceinline__ void inv_stages32(uint32_t* S, uint32_t* x, const uint2* w3, const uint2* TW, const LimbConst& lc,
+                                             int t) {
+    const int hi4 = t >> 4, lo4 = t & 15, w = t >> 5;
+    {   // stage 3': thread (a, b), 16 contiguous elements
+        const int aa = hi4, b = lo4;
+        uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
+        const int sw = (b >> 1) & 3;
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
+            x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
+        }
+        inv16_tw(x, w3, lc.q, lc.q2);
+#pragma unroll
+        for (int v = 0; v < 4; ++v)
+            *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) = make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
+    }
+    __syncwarp();
+    {   // stage 2': thread (a, c), elements b
+        const int aa = hi4, c = lo4;
+#pragma unroll
+        for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(aa, k, c)];
+        const uint2* W = TW + 32 * w + (aa & 1);
+        inv16_sp<false>(x, W, W + 2 + (aa & 1), W + 6 + 3 * (aa & 1), W + 14 + 7 * (aa & 1), lc);
+#pragma unroll
+        for (int k = 0; k < 16; ++k) S[v8_phys(aa, k, c)] = x[k];
+    }
+}
+// Inverse stage 1' (twiddles TW + 256): x <- thread (b, c)'s 16 elements a, lazy in [0, 2q)
+__device__ __forceinline__ void inv_stage1(const uint32_t* S, uint32_t* x, const uint2* TW, const LimbConst& lc, int t) {
+#pragma unroll
+    for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(k, t >> 4, t & 15)];
+    const uint2* T1 = TW + 256;
+    inv16_sp<false>(x, T1, T1 + 2, T1 + 4, T1 + 8, lc);
+}
+
 template <bool FWD>
 __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, const __grid_constant__ CUtensorMap tm_in) {
     constexpr int LOGN = 16, A = 4;
@@ -312,43 +391,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                     uint32_t* out = a.out + ((size_t)rwc << LOGN) + s * SUBW;
                     uint2 w3[15];
                     load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
-                    {   // stage 2: layers 8..11, thread (a, c), elements b
-                        const int aa = hi4, c = lo4;
-#pragma unroll
-                        for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(aa, k, c)];
-                        const uint2* T2 = TWB(u & 1) + 128;
-                        fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, qq, q2);
-#pragma unroll
-                        for (int k = 0; k < 16; ++k) S[v8_phys(aa, k, c)] = x[k];
-                    }
-                    __syncwarp();
-                    {   // stage 3: layers 12..15, thread (a, b), 16 contiguous elements; coalesced store
-                        const int aa = hi4, b = lo4;
-                        uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
-                        const int sw = (b >> 1) & 3;
-#pragma unroll
-                        for (int v = 0; v < 4; ++v) {
-                            const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
-                            x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
-                        }
-                        fwd16_tw(x, w3, qq, q2);
-#pragma unroll
-                        for (int v = 0; v < 4; ++v)
-                            *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
-                                make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
-                        __syncwarp();
-                        const int wbase = w * 512 + 4 * lane;
-#pragma unroll
-                        for (int v = 0; v < 4; ++v) {
-                            const int e = wbase + 128 * v;
-                            const uint4 r = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
-                            __stcs(reinterpret_cast<uint4*>(out + e),
-                                   make_uint4(canon4(r.x, qq, q2), canon4(r.y, qq, q2), canon4(r.z, qq, q2),
-                                              canon4(r.w, qq, q2)));
-                        }
-                        __syncwarp();
-                        if (lane == 0) mb_arrive(tbar + 2);   // this warp's last read of B0
-                    }
+                    fwd_stages23(S, x, TWB(u & 1) + 128, w3, qq, q2, out, t, tbar + 2);
                 }
                 lbc = lbn; rwc = rwn;
                 if (j + 2 < nrow) { lbn = limb_of(j + 2); rwn = r2; }
@@ -366,31 +409,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 cp_async_wait<0>();
                 __syncwarp();                            // this warp's slice of sub-row s landed
                 uint32_t x[16];
-                {   // stage 3': layers 15..12, thread (a, b), 16 contiguous elements
-                    const int aa = hi4, b = lo4;
-                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
-                    const int sw = (b >> 1) & 3;
-#pragma unroll
-                    for (int v = 0; v < 4; ++v) {
-                        const uint4 r = *reinterpret_cast<const uint4*>(base + ((v ^ sw) << 2));
-                        x[4 * v] = r.x; x[4 * v + 1] = r.y; x[4 * v + 2] = r.z; x[4 * v + 3] = r.w;
-                    }
-                    inv16_tw(x, w3, q, q2);
-#pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        *reinterpret_cast<uint4*>(base + ((v ^ sw) << 2)) =
-                            make_uint4(x[4 * v], x[4 * v + 1], x[4 * v + 2], x[4 * v + 3]);
-                }
-                __syncwarp();
-                {   // stage 2': layers 11..8, thread (a, c), elements b
-                    const int aa = hi4, c = lo4;
-#pragma unroll
-                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(aa, i, c)];
-                    const uint2* W = TWB(u & 1) + 32 * w + (aa & 1);
-                    inv16_sp<false>(x, W, W + 2 + (aa & 1), W + 6 + 3 * (aa & 1), W + 14 + 7 * (aa & 1), lc);
-#pragma unroll
-                    for (int i = 0; i < 16; ++i) S[v8_phys(aa, i, c)] = x[i];
-                }
+                inv_stages32(S, x, w3, TWB(u & 1), lc, t);
                 team_bar(team);                          // stage 2' done team-wide; the other buffer is free
                 {   // the team's next sub-row: data and twiddles into the other buffer
                     uint32_t nj = j, ns = (uint32_t)s + TEAMS, nl = limb, nr = row_self;
@@ -401,11 +420,8 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                     }
                     cp_async_commit();
                 }
-                {   // stage 1': layers 7..4, thread (b, c), elements a -> TMEM (lazy, in [0, 2q))
-#pragma unroll
-                    for (int i = 0; i < 16; ++i) x[i] = S[v8_phys(i, hi4, lo4)];
-                    const uint2* T1 = TWB(u & 1) + 256;
-                    inv16_sp<false>(x, T1, T1 + 2, T1 + 4, T1 + 8, lc);
+                {   // stage 1': layers A+3..A, thread (b, c), elements a -> TMEM (lazy, in [0, 2q))
+                    inv_stage1(S, x, TWB(u & 1), lc, t);
                     if (j & 1) tm_st16s(tl + s, x);      // B: element 256 a + t at 32 a + 16 h + s
                     else tm_st16(tl + 32 * s, x);        // A: 32 s + 16 h + a
                 }

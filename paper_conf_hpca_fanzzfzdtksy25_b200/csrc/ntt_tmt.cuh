@@ -150,43 +150,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
                     uint32_t* out = a.out + ((size_t)rwc << LOGN) + s * SUBW;
                     uint2 w3[15];
                     load_tw16(w3, tw, A + 8, (uint32_t)s * 256 + t);
-                    {   // stage 2: layers 5..8, thread (a, c), elements b
-                        const int aa = hi4, c = lo4;
-#pragma unroll
-                        for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(aa, k, c)];
-                        const uint2* T2 = TWB(u & 1) + 128;
-                        fwd16_sp(x, T2 + aa, T2 + 16 + 2 * aa, T2 + 48 + 4 * aa, T2 + 112 + 8 * aa, qq, q2);
-#pragma unroll
-                        for (int k = 0; k < 16; ++k) S[v8_phys(aa, k, c)] = x[k];
-                    }
-                    __syncwarp();
-                    {   // stage 3: layers 9..12, thread (a, b), 16 contiguous elements; coalesced store
-                        const int aa = hi4, b = lo4;
-                        uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
-                        const int sw = (b >> 1) & 3;
-#pragma unroll
-                        for (int vv = 0; vv < 4; ++vv) {
-                            const uint4 r = *reinterpret_cast<const uint4*>(base + ((vv ^ sw) << 2));
-                            x[4 * vv] = r.x; x[4 * vv + 1] = r.y; x[4 * vv + 2] = r.z; x[4 * vv + 3] = r.w;
-                        }
-                        fwd16_tw(x, w3, qq, q2);
-#pragma unroll
-                        for (int vv = 0; vv < 4; ++vv)
-                            *reinterpret_cast<uint4*>(base + ((vv ^ sw) << 2)) =
-                                make_uint4(x[4 * vv], x[4 * vv + 1], x[4 * vv + 2], x[4 * vv + 3]);
-                        __syncwarp();
-                        const int wbase = w * 512 + 4 * lane;
-#pragma unroll
-                        for (int vv = 0; vv < 4; ++vv) {
-                            const int e = wbase + 128 * vv;
-                            const uint4 r = *reinterpret_cast<const uint4*>(S + v8_phys(e >> 8, (e >> 4) & 15, e & 15));
-                            __stcs(reinterpret_cast<uint4*>(out + e),
-                                   make_uint4(canon4(r.x, qq, q2), canon4(r.y, qq, q2), canon4(r.z, qq, q2),
-                                              canon4(r.w, qq, q2)));
-                        }
-                        __syncwarp();
-                        if (lane == 0) mb_arrive(tbar + 2);   // this warp's last read of B0
-                    }
+                    tmr::fwd_stages23(S, x, TWB(u & 1) + 128, w3, qq, q2, out, t, tbar + 2);
                 }
                 lbc = lbn; rwc = rwn;
                 if (j + 2 < nrow) { lbn = limb_of(j + 2); rwn = r2; }
@@ -204,31 +168,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
                 cp_async_wait<0>();
                 __syncwarp();                            // this warp's slice of the sub-row landed
                 uint32_t x[16];
-                {   // stage 3': layers 12..9, thread (a, b), 16 contiguous elements
-                    const int aa = hi4, b = lo4;
-                    uint32_t* base = S + aa * 256 + ((b ^ (aa & 1)) << 4);
-                    const int sw = (b >> 1) & 3;
-#pragma unroll
-                    for (int vv = 0; vv < 4; ++vv) {
-                        const uint4 r = *reinterpret_cast<const uint4*>(base + ((vv ^ sw) << 2));
-                        x[4 * vv] = r.x; x[4 * vv + 1] = r.y; x[4 * vv + 2] = r.z; x[4 * vv + 3] = r.w;
-                    }
-                    inv16_tw(x, w3, q, q2);
-#pragma unroll
-                    for (int vv = 0; vv < 4; ++vv)
-                        *reinterpret_cast<uint4*>(base + ((vv ^ sw) << 2)) =
-                            make_uint4(x[4 * vv], x[4 * vv + 1], x[4 * vv + 2], x[4 * vv + 3]);
-                }
-                __syncwarp();
-                {   // stage 2': layers 8..5, thread (a, c), elements b
-                    const int aa = hi4, c = lo4;
-#pragma unroll
-                    for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(aa, k, c)];
-                    const uint2* W = TWB(u & 1) + 32 * w + (aa & 1);
-                    inv16_sp<false>(x, W, W + 2 + (aa & 1), W + 6 + 3 * (aa & 1), W + 14 + 7 * (aa & 1), lc);
-#pragma unroll
-                    for (int k = 0; k < 16; ++k) S[v8_phys(aa, k, c)] = x[k];
-                }
+                tmr::inv_stages32(S, x, w3, TWB(u & 1), lc, t);
                 tmr::team_bar(team);                     // stage 2' done team-wide; the other buffer is free
                 {   // the team's next sub-row: data and twiddles into the other buffer
                     uint32_t nj = jr, ns = (uint32_t)s + 1, nl = limb, nr = row_self;
@@ -239,11 +179,8 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
                     }
                     cp_async_commit();
                 }
-                {   // stage 1': layers 4..1, thread (b, c), elements a -> slot jr & 1 (lazy, in [0, 2q))
-#pragma unroll
-                    for (int k = 0; k < 16; ++k) x[k] = S[v8_phys(k, hi4, lo4)];
-                    const uint2* T1 = TWB(u & 1) + 256;
-                    inv16_sp<false>(x, T1, T1 + 2, T1 + 4, T1 + 8, lc);
+                {   // stage 1': layers A+3..A, thread (b, c), elements a -> TMEM (lazy, in [0, 2q))
+                    tmr::inv_stage1(S, x, TWB(u & 1), lc, t);
                     tms::st16_stride<R>(tl + SLOT * (jr & 1) + s, x);
                 }
                 ++u;
