@@ -40,6 +40,22 @@ constexpr int TWW = 768;                        // words per twiddle area (<= 38
 constexpr int TEAM_W = 3 * SUBW + 2 * TWW;
 constexpr int SMEM = TEAMS * TEAM_W * 4 + 128;  // + 3 mbarriers per team, the row mbarrier, the TMEM slot
 
+// ---------------------------------------------------------------- debug checks (compute-sanitizer is closed
+// on the GPU pool this round): a -DWD_TM_DEBUG build traps on a TMEM access outside the warp's lane
+// quadrant or the 512 allocated columns, on a row index outside the batch, and on an mbarrier wait that
+// does not complete (tma.cuh); tests/test_gpu_parity.py runs the tm shapes against it
+#ifdef WD_TM_DEBUG
+#define TM_ASSERT(c) do { if (!(c)) __trap(); } while (0)
+#else
+#define TM_ASSERT(c) do { } while (0)
+#endif
+// a TMEM access of `span` consecutive columns from ta by this thread's warp
+__device__ __forceinline__ void tm_check(uint32_t ta, uint32_t span) {
+    TM_ASSERT((ta >> 16) == 32u * ((threadIdx.x >> 5) & 3));
+    TM_ASSERT((ta & 0xFFFFu) + span <= 512u);
+    (void)ta; (void)span;
+}
+
 // ---------------------------------------------------------------- tensor memory
 __device__ __forceinline__ void tfence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tfence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -47,6 +63,7 @@ __device__ __forceinline__ void tm_wait_st() { asm volatile("tcgen05.wait::st.sy
 // 16 consecutive columns of the warp's lanes -> x[0..15]; complete on return (wait::ld in the same asm,
 // so no use of x can be scheduled before it)
 __device__ __forceinline__ void tm_ld16(uint32_t ta, uint32_t* x) {
+    tm_check(ta, 16);
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x16.b32 "
                  "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n\t"
                  "tcgen05.wait::ld.sync.aligned;"
@@ -56,6 +73,7 @@ __device__ __forceinline__ void tm_ld16(uint32_t ta, uint32_t* x) {
 }
 // columns ta, ta + 32, ..., ta + 480 -> x[0..15]
 __device__ __forceinline__ void tm_ld16s(uint32_t ta, uint32_t* x) {
+    tm_check(ta, 481);
     asm volatile("{\n\t"
                  "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%16];\n\t"
                  "tcgen05.ld.sync.aligned.32x32b.x1.b32 {%1}, [%16+32];\n\t"
@@ -79,6 +97,7 @@ __device__ __forceinline__ void tm_ld16s(uint32_t ta, uint32_t* x) {
                  : "r"(ta) : "memory");
 }
 __device__ __forceinline__ void tm_st16(uint32_t ta, const uint32_t* x) {
+    tm_check(ta, 16);
     asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
                  "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};"
                  :: "r"(ta), "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7]),
@@ -86,6 +105,7 @@ __device__ __forceinline__ void tm_st16(uint32_t ta, const uint32_t* x) {
                  : "memory");
 }
 __device__ __forceinline__ void tm_st16s(uint32_t ta, const uint32_t* x) {
+    tm_check(ta, 481);
     asm volatile("{\n\t"
                  "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};\n\t"
                  "tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+32], {%2};\n\t"
@@ -288,6 +308,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
     };
     auto row_of = [&](uint32_t j) {
         const uint32_t sr = blockIdx.x + j * G;
+        TM_ASSERT(sr < nb * a.L);                // a schedule slot of the batch
         if (!a.limb_major) return sr;
         const uint32_t lb = sr / nb;
         return (sr - lb * nb) * a.L + lb;

@@ -45,6 +45,7 @@ __device__ __forceinline__ void st1_at(uint32_t ta, const uint32_t* x) {
 }
 template <int R>
 __device__ __forceinline__ void ld16_stride(uint32_t ta, uint32_t* x) {
+    tmr::tm_check(ta, 15 * R + 1);
     ld1_at<R, 0>(ta, x);
     asm volatile("tcgen05.wait::ld.sync.aligned;"
                  : "+r"(x[0]), "+r"(x[1]), "+r"(x[2]), "+r"(x[3]), "+r"(x[4]), "+r"(x[5]), "+r"(x[6]), "+r"(x[7]),
@@ -52,10 +53,14 @@ __device__ __forceinline__ void ld16_stride(uint32_t ta, uint32_t* x) {
                  :: "memory");
 }
 template <int R>
-__device__ __forceinline__ void st16_stride(uint32_t ta, const uint32_t* x) { st1_at<R, 0>(ta, x); }
+__device__ __forceinline__ void st16_stride(uint32_t ta, const uint32_t* x) {
+    tmr::tm_check(ta, 15 * R + 1);
+    st1_at<R, 0>(ta, x);
+}
 // R contiguous cells
 template <int R>
 __device__ __forceinline__ void stR(uint32_t ta, const uint32_t* x) {
+    tmr::tm_check(ta, R);
     if constexpr (R == 8)
         asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
                      :: "r"(ta), "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7])
@@ -66,6 +71,7 @@ __device__ __forceinline__ void stR(uint32_t ta, const uint32_t* x) {
 }
 template <int R>
 __device__ __forceinline__ void ldR(uint32_t ta, uint32_t* x) {
+    tmr::tm_check(ta, R);
     if constexpr (R == 8)
         asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];\n\t"
                      "tcgen05.wait::ld.sync.aligned;"
@@ -135,6 +141,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
     };
     auto row_of = [&](uint32_t j) {
         const uint32_t sr = blockIdx.x + j * G;
+        TM_ASSERT(sr < nb * a.L);                // a schedule slot of the batch
         if (!a.limb_major) return sr;
         const uint32_t lb = sr / nb;
         return (sr - lb * nb) * a.L + lb;

@@ -69,6 +69,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
     };
     auto row_of = [&](uint32_t j) {
         const uint32_t sr = vslot(j), nb = a.nb_total ? a.nb_total : rows / a.L;
+        TM_ASSERT(sr < nb * a.L);                // a schedule slot of the batch
         if (!a.limb_major) return sr;
         const uint32_t lb = sr / nb;
         return (sr - lb * nb) * a.L + lb;

@@ -12,9 +12,21 @@ __device__ __forceinline__ void mb_init(uint64_t* b, uint32_t n) {
 }
 __device__ __forceinline__ void mb_init_fence() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 __device__ __forceinline__ void mb_wait(uint64_t* b, uint32_t parity) {
+#ifdef WD_TM_DEBUG
+    // debug builds: trap instead of hanging when a phase never completes (~2 s at B200 clocks)
+    const long long t0 = clock64();
+    for (;;) {
+        uint32_t ok;
+        asm volatile("{\n\t.reg .pred P1;\n\tmbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+                     "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(ok) : "r"(smem_u32(b)), "r"(parity) : "memory");
+        if (ok) break;
+        if (clock64() - t0 > (1LL << 32)) __trap();
+    }
+#else
     asm volatile("{\n\t.reg .pred P1;\n\tMBW_%=:\n\t"
                  "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
                  "@!P1 bra MBW_%=;\n\t}\n" :: "r"(smem_u32(b)), "r"(parity) : "memory");
+#endif
 }
 __device__ __forceinline__ void mb_arrive(uint64_t* b) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(b)) : "memory");
