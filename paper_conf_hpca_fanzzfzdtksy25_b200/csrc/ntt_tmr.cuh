@@ -17,15 +17,20 @@
 // TMEM cell (lane t % 128, column col(p, k, h)).  Two layouts alternate from row to row,
 //   A: col(p, k, h) = 32 k + 16 h + p          B: col(p, k, h) = 32 p + 16 h + k,
 // so that the 32 cells sub-row s of row j has consumed are exactly the cells column pass s of row j+1
-// writes, by the same thread (forward; the inverse mirrors it).  A team therefore interleaves
-//   forward:  R(j, s) C(j+1, s)  for its four s, then one CTA barrier per row,
-//   inverse:  C'(j, s) R'(j+1, s) for its four s, then one CTA barrier per row,
-// with the column pass of the next row overwriting the sub-row just consumed -- the classic in-place
-// ping-pong.  In each row one of the two accesses is 16 contiguous columns (one tcgen05.ld/st .x16),
-// the other 16 strided ones (.x1).
-// Forward column passes are fed by TMA (one 256 x 16 box per pass, issued one pass ahead); inverse
-// sub-rows by 16-byte cp.async, double-buffered as in v8; forward outputs leave by coalesced 512-byte
-// STG from the sub-row buffer, inverse outputs straight from registers (128-byte lines per warp).
+// writes, by the same thread (forward; the inverse mirrors it).  A team therefore interleaves, for its
+// four s,
+//   forward:  R1(j, s) [stage 1 from TMEM]  C(j+1, s) [column pass into the cells R1 just read]  team
+//             barrier  R23(j, s); rows hand over through a CTA mbarrier (arrive after a warp's last
+//             column pass of row j+1, wait before its first stage-1 read of that row),
+//   inverse:  C'(j, s) R'(j+1, s) [stages 3', 2', team barrier, stage 1' into the cells C' read], then
+//             one CTA barrier per row,
+// the classic in-place ping-pong.  In each row one of the two accesses is 16 contiguous columns (one
+// tcgen05.ld/st .x16), the other 16 strided ones (.x1).  The column pass between stage 1 and the
+// stage-1 barrier covers that barrier's wait.
+// Forward column passes are fed by TMA (one 256 x 16 box per pass, two staging buffers per team, issued
+// two passes ahead); inverse sub-rows by 16-byte cp.async, double-buffered as in v8; forward outputs
+// leave by coalesced 512-byte STG from the sub-row buffer, inverse outputs straight from registers
+// (128-byte lines per warp).  Ablations and measurements: DESIGN.md 5.1a.
 #pragma once
 #include "ntt_v8.cuh"
 
