@@ -28,7 +28,8 @@ int prep_tmr() {
     return set_attr(tmr::ntt_tmr16<true>, tmr::SMEM) | set_attr(tmr::ntt_tmr16<false>, tmr::SMEM) |
            set_attr(tms::ntt_tms<2, true>, tms::SMEM) | set_attr(tms::ntt_tms<2, false>, tms::SMEM) |
            set_attr(tms::ntt_tms<3, true>, tms::SMEM) | set_attr(tms::ntt_tms<3, false>, tms::SMEM) |
-           set_attr(tmt::ntt_tmt13<true>, tmt::SMEM) | set_attr(tmt::ntt_tmt13<false>, tmt::SMEM);
+           set_attr(tmt::ntt_tmt13<true>, tmt::SMEM) | set_attr(tmt::ntt_tmt13<false>, tmt::SMEM) |
+           set_attr(tmr::ntt_tmr16<true, true>, tmr::SMEM);
 }
 
 // plain transforms only (contiguous [batch][L][N] rows, no pointwise product / store maps / copies);
@@ -67,6 +68,19 @@ int launch_tmr(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int sm_
         if (fwd) tmt::ntt_tmt13<true><<<g13, tmr::NT, tmt::SMEM, s>>>(a, rows, tm);
         else tmt::ntt_tmt13<false><<<g13, tmr::NT, tmt::SMEM, s>>>(a, rows, tm);
     }
+    return 1;
+}
+
+int launch_tmr17(const NttArgs& a, uint32_t rows2, int sm_count, cudaStream_t s) {
+    alignas(64) CUtensorMap tm;
+    std::memset(&tm, 0, sizeof(tm));
+    // the 2^17 input as lines of 4096 words (32 per row, 16 per half-row); a column pass loads two 256 x 16
+    // boxes (both halves of its columns)
+    const cuuint64_t dims[2] = {tmr::SUBW, (cuuint64_t)rows2 * 16}, strides[1] = {tmr::SUBW * 4};
+    const cuuint32_t box[2] = {tmr::TT, 16};
+    if (!tma_encode_u32(&tm, a.in, 2, dims, strides, box, CU_TENSOR_MAP_SWIZZLE_NONE)) return -2;
+    const uint32_t grid = std::min<uint32_t>(rows2, (uint32_t)sm_count);
+    tmr::ntt_tmr16<true, true><<<grid, tmr::NT, tmr::SMEM, s>>>(a, rows2, tm);
     return 1;
 }
 

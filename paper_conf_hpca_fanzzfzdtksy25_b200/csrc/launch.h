@@ -35,6 +35,9 @@ int prep_tmr();
 // returns launches (1), -1 if the size or the arguments need v8 (pointwise product, store maps, strided
 // rows), -2 if the tensor map cannot be encoded
 int launch_tmr(uint32_t logN, bool fwd, const NttArgs& a, uint32_t rows, int sm_count, cudaStream_t s);
+// N = 2^17 forward on its two 2^16 halves: `a` is the virtual half plan (2 L limbs, the re-indexed twiddles
+// and LimbConst of wd_ntt.cu), rows2 = 2 x the 2^17 rows; a.in / a.out the 2^17 data
+int launch_tmr17(const NttArgs& a, uint32_t rows2, int sm_count, cudaStream_t s);
 
 // ---- k_tensor.cu: the round-1 tensor path (TENSOR, FUSED modes; N = 2^16)
 int prep_tensor();

@@ -261,8 +261,15 @@ __device__ __forceinline__ void inv_stage1(const uint32_t* S, uint32_t* x, const
     inv16_sp<false>(x, T1, T1 + 2, T1 + 4, T1 + 8, lc);
 }
 
-template <bool FWD>
+// H17 (forward only): N = 2^17 as two independent 2^16 halves.  After the first merged-psi layer (pairs j,
+// j + 2^16, twiddle Psi17[1]) the halves never interact again, and half h is the 2^16 network whose layer-l
+// group-g twiddle is Psi17[2^(l+1) + h 2^l + g].  The host passes a virtual plan: 2 L limbs (limb' = 2 l + h,
+// re-indexed twiddle tables, LimbConst with (Psi17[1], Shoup) in pad_[0..1]) and 2 rows per 2^17 row, so
+// one CTA holds one half in TMEM.  Only the column pass differs: it loads both halves' lines of its columns
+// (two TMA boxes, 32 KB, single-buffered, issued one pass ahead) and applies layer 0 before layers 1..4.
+template <bool FWD, bool H17 = false>
 __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, const __grid_constant__ CUtensorMap tm_in) {
+    static_assert(FWD || !H17, "H17: forward only");
     constexpr int LOGN = 16, A = 4;
     extern __shared__ __align__(1024) uint32_t smem[];
     const int team = (int)(threadIdx.x >> 8), t = (int)(threadIdx.x & (TT - 1));
@@ -337,31 +344,51 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
             const uint32_t mtot = 4 * nrow;          // column passes of the CTA
             auto issue_col = [&](uint32_t m, uint32_t prow) {   // team thread 0
                 fence_proxy_async();
-                mb_expect(tbar + (m & 1), 16 * TT * 4);
-                tma2_load_hint((m & 1) ? B2 : B1, &tm_in, (team + 4 * (int)(m & 3)) * TT, (int)(prow * 16),
-                               tbar + (m & 1), l2_evict_first_policy());
+                if constexpr (H17) {                 // both halves' lines of the 2^17 row prow / 2 -> B1, B2
+                    mb_expect(tbar, 32 * TT * 4);
+                    const int line = (int)((prow >> 1) * 32), c0 = (team + 4 * (int)(m & 3)) * TT;
+                    tma2_load_hint(B1, &tm_in, c0, line, tbar, l2_evict_first_policy());
+                    tma2_load_hint(B2, &tm_in, c0, line + 16, tbar, l2_evict_first_policy());
+                } else {
+                    mb_expect(tbar + (m & 1), 16 * TT * 4);
+                    tma2_load_hint((m & 1) ? B2 : B1, &tm_in, (team + 4 * (int)(m & 3)) * TT, (int)(prow * 16),
+                                   tbar + (m & 1), l2_evict_first_policy());
+                }
             };
             // column pass m (row m / 4): layers 0..3, into TMEM (layout (m / 4) & 1)
             auto colpass = [&](uint32_t m, uint32_t limb) {
                 const int s = team + 4 * (int)(m & 3);
                 const LimbConst lc = a.lc[limb];
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
-                const uint32_t b = m & 1;
-                mb_wait(tbar + b, (tph >> b) & 1);
-                tph ^= 1u << b;
-                const uint32_t* SB = b ? B2 : B1;
                 uint32_t x[16];
+                if constexpr (H17) {
+                    mb_wait(tbar, m & 1);            // one staging buffer, one completion per pass
+                    const uint2 w0 = make_uint2(lc.pad_[0], lc.pad_[1]);
+                    const bool upper = limb & 1;     // half h = limb' & 1
 #pragma unroll
-                for (int k = 0; k < 16; ++k) x[k] = SB[k * TT + t];
+                    for (int k = 0; k < 16; ++k) {   // layer 0 of 2^17: (x_j, x_j+2^16) -> this half's value
+                        const uint32_t lo = umin32(B1[k * TT + t], B1[k * TT + t] - lc.q2);
+                        const uint32_t tt = shoup_mul(B2[k * TT + t], w0.x, w0.y, lc.q);
+                        x[k] = upper ? lo - tt + lc.q2 : lo + tt;
+                    }
+                } else {
+                    const uint32_t b = m & 1;
+                    mb_wait(tbar + b, (tph >> b) & 1);
+                    tph ^= 1u << b;
+                    const uint32_t* SB = b ? B2 : B1;
+#pragma unroll
+                    for (int k = 0; k < 16; ++k) x[k] = SB[k * TT + t];
+                }
                 fwd_radix<A>(x, tw, 0, 0, lc.q, lc.q2);
                 if ((m >> 2) & 1) tm_st16(tl + 32 * s, x);   // B: 32 s + 16 h + k
                 else tm_st16s(tl + s, x);                    // A: 32 k + 16 h + s
             };
 
             // prologue: the column passes of row 0 (TMA 0, 1 up front, m + 2 after pass m's team barrier)
+            constexpr uint32_t AHEAD = H17 ? 1 : 2;  // passes a TMA runs ahead (staging buffers)
             if (t == 0) {
                 issue_col(0, rwc);
-                if (1 < mtot) issue_col(1, rwc);
+                if (!H17 && 1 < mtot) issue_col(1, rwc);
             }
             tw_fwd<A>(TWB(0), a.tw + ((size_t)lbc << LOGN), team, t);
             cp_async_commit();
@@ -369,7 +396,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
             for (uint32_t m = 0; m < 4; ++m) {
                 colpass(m, lbc);
                 team_bar(team);
-                if (t == 0 && m + 2 < mtot) issue_col(m + 2, m + 2 < 4 ? rwc : rwn);
+                if (t == 0 && m + AHEAD < mtot) issue_col(m + AHEAD, m + AHEAD < 4 ? rwc : rwn);
             }
             row_arrive();
 #pragma unroll 1
@@ -405,7 +432,8 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                         if (i == 3) row_arrive();        // this warp's part of row j + 1 is in TMEM
                     }
                     team_bar(team);                      // stage 1 (and column pass m) done team-wide
-                    if (t == 0 && more && m + 2 < mtot) issue_col(m + 2, ((m + 2) >> 2) == j + 1 ? rwn : r2);
+                    if (t == 0 && more && m + AHEAD < mtot)
+                        issue_col(m + AHEAD, ((m + AHEAD) >> 2) == j + 1 ? rwn : r2);
                     {   // the team's next sub-row's twiddles
                         uint32_t nj = j, ns = (uint32_t)s + TEAMS;
                         if (ns >= 16) { nj = j + 1; ns = team; }

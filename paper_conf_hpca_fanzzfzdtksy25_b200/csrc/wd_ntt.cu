@@ -51,6 +51,11 @@ struct wd_ntt_plan {
     uint2* d_fwd = nullptr;        // [L][N]  (psi^brv(i), Shoup)
     uint2* d_inv = nullptr;        // [L][N]  (psi^-brv(i), Shoup)
     LimbConst* d_lc = nullptr;     // [L]
+    // N = 2^17 forward through tm (ntt_tmr.cuh H17): the two 2^16 halves as a virtual plan of 2 L limbs,
+    // limb' = 2 l + h: [L][2][2^16] re-indexed forward twiddles (local index 2^k + g of half h = Psi[2^(k+1)
+    // + h 2^k + g]) and [2 L] LimbConst carrying the first layer's (Psi[1], Shoup) in pad_[0..1]
+    uint2* d_fwd17 = nullptr;
+    LimbConst* d_lc17 = nullptr;
     uint4* d_rs = nullptr;         // [L] RESCALE constants vs the last prime (ntt_rns.cuh); L >= 2
     uint32_t rs_thr = 0;           // q_last - floor(q_last / 2)
     bool rs_ok = false;            // L >= 2 and q_last differs from every other prime
@@ -125,6 +130,21 @@ int launch_cuda_core(const wd_ntt_plan* p, bool fwd, const NttArgs& a, uint32_t 
     //    the remaining schedule slots right after it (the same limb-major slot -> row map);
     //  * otherwise tm alone when its rounds are at least 85% full, else v8, whose 4 CTAs per SM absorb
     //    such a tail (scripts/gpu_tm_rows*.sh, profiles/r02/tm/)
+    // N = 2^17 forward: tm on the two 2^16 halves of every row (ntt_tmr.cuh H17; 2 rows per 2^17 row),
+    // when those half-row rounds are at least 85% full.  Out of place only: both halves read the whole
+    // input row (the first layer pairs them) on different SMs at different times, so in place one half's
+    // output could overwrite input the other still has to read.  The inverse stays on v8 (its last layer
+    // joins the halves).
+    if ((ver == 0 || ver == 20) && logN == 17 && fwd && p->d_fwd17 && a.in != a.out && !a.in2 && !a.aux && !a.cpy &&
+        !a.in_ls && !a.out_ls && !a.slot0 && !a.nb_total) {
+        const uint64_t r2 = 2ull * rows, u = (uint64_t)sm;
+        if ((ver == 20 || (r2 >= u && r2 * 20 >= u * ((r2 + u - 1) / u) * 17)) && r2 <= 0x7fffffffull) {
+            NttArgs ah = a;
+            ah.L = 2 * a.L; ah.tw = p->d_fwd17; ah.lc = p->d_lc17;
+            const int n = launch_tmr17(ah, (uint32_t)r2, p->sm_count, s);
+            if (n > 0) { g_last_kernel = "tm17"; return n; }
+        }
+    }
     bool tm_tail = false;
     uint64_t tm_unit = 0;
     if (ver == 0 && logN >= 13 && logN <= 16) {
@@ -320,6 +340,7 @@ void free_plan(wd_ntt_plan* p) {
         cudaGetDevice(&cur);
         if (cur != p->device) cudaSetDevice(p->device);
         cudaFree(p->d_fwd); cudaFree(p->d_inv); cudaFree(p->d_lc); cudaFree(p->d_rs);
+        cudaFree(p->d_fwd17); cudaFree(p->d_lc17);
         free_tensor_tables(p->tc);
         free_tc4_tables(p->t4);
         for (auto& s : p->hs) if (s) cudaStreamDestroy(s);
@@ -459,6 +480,32 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
         cudaMemcpy(p->d_lc, lc.data(), sizeof(LimbConst) * L, cudaMemcpyHostToDevice) != cudaSuccess) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }
+    if (p->logN == 17) {   // the virtual half plan of the tm forward (same table bytes as d_fwd)
+        try {
+            const uint32_t H = N / 2;
+            std::vector<uint2> h17((size_t)L * N);
+            std::vector<LimbConst> l17(2 * (size_t)L);
+            for (uint32_t l = 0; l < L; ++l) {
+                const uint2* f = fwd.data() + (size_t)l * N;
+                for (uint32_t hh = 0; hh < 2; ++hh) {
+                    uint2* d = h17.data() + ((size_t)l * 2 + hh) * H;
+                    d[0] = make_uint2(0, 0);
+                    for (uint32_t k = 0; (1u << k) < H; ++k)
+                        for (uint32_t g = 0; g < (1u << k); ++g) d[(1u << k) + g] = f[(2u << k) + (hh << k) + g];
+                    LimbConst c = lc[l];
+                    c.pad_[0] = f[1].x; c.pad_[1] = f[1].y;
+                    l17[2 * l + hh] = c;
+                }
+            }
+            if (cudaMalloc(&p->d_fwd17, tb) != cudaSuccess || cudaMalloc(&p->d_lc17, sizeof(LimbConst) * 2 * L) != cudaSuccess ||
+                cudaMemcpy(p->d_fwd17, h17.data(), tb, cudaMemcpyHostToDevice) != cudaSuccess ||
+                cudaMemcpy(p->d_lc17, l17.data(), sizeof(LimbConst) * 2 * L, cudaMemcpyHostToDevice) != cudaSuccess) {
+                cudaGetLastError(); free_plan(p); set_err(WD_ENOMEM); return nullptr;
+            }
+        } catch (const std::bad_alloc&) {
+            free_plan(p); set_err(WD_ENOMEM); return nullptr;
+        }
+    }
     // RESCALE constants (row f4): per limb i < L-1 {-q_last mod q_i, Shoup(1), q_last^-1 mod q_i, Shoup}
     if (L >= 2) {
         const uint32_t ql = primes[L - 1];
@@ -481,7 +528,7 @@ wd_ntt_plan* wd_ntt_plan_create(uint32_t N, const uint32_t* primes, uint32_t L) 
     if (cudaStreamCreateWithFlags(&p->fs, cudaStreamNonBlocking) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     for (auto& e : p->fe) if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) { free_plan(p); set_err(WD_ECUDA); return nullptr; }
     if (prep_cc(p->logN) || prep_v8(p->logN, p->sm_count, &p->occ) || prep_rns() ||
-        (p->logN >= 13 && p->logN <= 16 && prep_tmr()) ||
+        (p->logN >= 13 && p->logN <= 17 && prep_tmr()) ||
         (p->logN == 16 && (prep_tensor() || prep_wdcuda() || prep_tc4()))) {
         cudaGetLastError(); free_plan(p); set_err(WD_ECUDA); return nullptr;
     }

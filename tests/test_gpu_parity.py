@@ -206,6 +206,8 @@ def test_auto_decision_boundaries(wd, logn):
         split = 13 <= logn <= 16 and rows >= unit and tail * 4 <= unit          # full rounds + v8 tail
         tm_alone = 13 <= logn <= 16 and not split and rows * 20 >= unit * (-(-rows // unit)) * 17
         want = "tm+v8" if split and tail else "tm" if split or tm_alone else None
+        if logn == 17 and 2 * rows >= sm and 2 * rows * 20 >= sm * (-(-2 * rows // sm)) * 17:
+            want = "tm17"                        # the forward on the two 2^16 halves of every row
         got = wd.wd_ntt_last_kernel()
         assert (got == want) if want else not got.startswith("tm"), (logn, rows, got)
         assert np.array_equal(y, oracle.ntt_forward(x, primes)), (logn, rows)
@@ -399,6 +401,37 @@ def test_tm_kernel(wd, logn, L, batch, lm, monkeypatch):
             np.array(primes, dtype=np.uint32)[None, :, None] - 1, x.shape).copy()
         assert np.array_equal(gpu_fwd(wd, plan, e), oracle.ntt_forward(e, primes)), (L, batch, kind)
         assert np.array_equal(gpu_inv(wd, plan, e), oracle.ntt_inverse(e, primes)), (L, batch, kind)
+    plan.close()
+
+
+# N = 2^17 forward on its two 2^16 halves (tm17: AUTO when the half-row rounds are full, or WD_NTT_KERNEL=tm):
+# few half-rows, ragged counts, the natural order, in place, edge inputs; the inverse stays on v8
+@pytest.mark.parametrize("L,batch,lm,force", [(1, 74, "1", ""), (3, 50, "1", ""), (48, 4, "1", ""), (5, 1, "1", "tm"),
+                                              (7, 11, "0", "tm"), (48, 64, "1", "")])
+def test_tm17_forward(wd, L, batch, lm, force, monkeypatch):
+    if force:
+        monkeypatch.setenv("WD_NTT_KERNEL", force)
+    monkeypatch.setenv("WD_NTT_LM", lm)
+    n = 1 << 17
+    primes = [P[(13 * i + L) % 60] for i in range(L)]
+    x = inputs.uniform_residues(primes, n, batch, 6100 + L * 17 + batch)
+    plan = wd.Plan(n, primes)
+    y = gpu_fwd(wd, plan, x)
+    sm = torch.cuda.get_device_properties(0).multi_processor_count
+    r2 = 2 * batch * L
+    if force or (r2 >= sm and r2 * 20 >= sm * (-(-r2 // sm)) * 17):
+        assert wd.wd_ntt_last_kernel() == "tm17", wd.wd_ntt_last_kernel()
+    assert np.array_equal(y, oracle.ntt_forward(x, primes)), (L, batch)
+    t = to_dev(x)
+    plan.forward(t, t)                                   # in place
+    plan.inverse(t, t)
+    torch.cuda.synchronize()
+    assert np.array_equal(to_host(t), x), (L, batch)
+    if batch * L <= 200:
+        for kind in ("zeros", "qminus1"):
+            e = np.zeros_like(x) if kind == "zeros" else np.broadcast_to(
+                np.array(primes, dtype=np.uint32)[None, :, None] - 1, x.shape).copy()
+            assert np.array_equal(gpu_fwd(wd, plan, e), oracle.ntt_forward(e, primes)), (L, batch, kind)
     plan.close()
 
 
