@@ -403,8 +403,6 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
             for (uint32_t j = 0; j < nrow; ++j) {
                 const bool more = j + 1 < nrow;
                 const uint32_t r2 = j + 2 < nrow ? row_of(j + 2) : 0;
-                const uint32_t q = 0;   // (per-row constants are loaded inside the passes)
-                (void)q;
 #pragma unroll 1
                 for (int i = 0; i < 4; ++i, ++u) {
                     const int s = team + 4 * i;
@@ -455,7 +453,6 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
             auto rowpass = [&](uint32_t j, int s, uint32_t u, uint32_t limb, uint32_t row_self, uint32_t limb_next,
                                uint32_t row_next) {
                 const LimbConst lc = a.lc[limb];
-                const uint32_t q = lc.q, q2 = lc.q2;
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
                 uint32_t* S = (u & 1) ? B1 : B0;
                 uint2 w3[15];

@@ -255,7 +255,6 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
             auto rowpass = [&](uint32_t jr, int s, uint32_t limb, uint32_t row_self, uint32_t limb_next,
                                uint32_t row_next, int i) {
                 const LimbConst lc = a.lc[limb];
-                const uint32_t q = lc.q, q2 = lc.q2;
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
                 uint32_t* S = (u & 1) ? B1 : B0;
                 uint2 w3[15];

@@ -29,7 +29,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
     constexpr int SLOT = 32;                     // TMEM columns of one row per (lane, half) and team
     extern __shared__ __align__(1024) uint32_t smem[];
     const int team = (int)(threadIdx.x >> 8), t = (int)(threadIdx.x & (TT - 1));
-    const int w = t >> 5, h = w >> 2, hi4 = t >> 4, lo4 = t & 15, lane = t & 31;
+    const int w = t >> 5, h = w >> 2, hi4 = t >> 4, lo4 = t & 15;
     uint32_t* TS = smem + team * TEAM_W;
     uint32_t* const B0 = TS;                     // forward: sub-row exchange; inverse: input buffer 0
     uint32_t* const B1 = TS + SUBW;              // inverse: input buffer 1; forward: staging of even steps
@@ -161,7 +161,6 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
             auto rowpass = [&](uint32_t jr, int s, uint32_t limb, uint32_t row_self, uint32_t limb_next,
                                uint32_t row_next) {
                 const LimbConst lc = a.lc[limb];
-                const uint32_t q = lc.q, q2 = lc.q2;
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
                 uint32_t* S = (u & 1) ? B1 : B0;
                 uint2 w3[15];
