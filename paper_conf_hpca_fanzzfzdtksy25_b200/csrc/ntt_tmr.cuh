@@ -356,9 +356,13 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                 }
             };
             // column pass m (row m / 4): layers 0..3, into TMEM (layout (m / 4) & 1)
-            auto colpass = [&](uint32_t m, uint32_t limb) {
+            // qv = (q, 2q) of the limb, loaded once per row by the caller: a LimbConst load per pass
+            // (re-issued after every asm volatile TMEM access) stalls the first butterfly on its latency
+            auto colpass = [&](uint32_t m, uint32_t limb, uint2 qv) {
                 const int s = team + 4 * (int)(m & 3);
-                const LimbConst lc = a.lc[limb];
+                LimbConst lc;
+                if constexpr (H17) lc = a.lc[limb];  // + (Psi17[1], Shoup) in pad_
+                else { lc.q = qv.x; lc.q2 = qv.y; }
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
                 uint32_t x[16];
                 if constexpr (H17) {
@@ -394,7 +398,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
             cp_async_commit();
 #pragma unroll 1
             for (uint32_t m = 0; m < 4; ++m) {
-                colpass(m, lbc);
+                colpass(m, lbc, __ldg(reinterpret_cast<const uint2*>(a.lc + lbc)));
                 team_bar(team);
                 if (t == 0 && m + AHEAD < mtot) issue_col(m + AHEAD, m + AHEAD < 4 ? rwc : rwn);
             }
@@ -403,10 +407,13 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
             for (uint32_t j = 0; j < nrow; ++j) {
                 const bool more = j + 1 < nrow;
                 const uint32_t r2 = j + 2 < nrow ? row_of(j + 2) : 0;
+                const uint2 qc = __ldg(reinterpret_cast<const uint2*>(a.lc + lbc));   // (q, 2q) of rows j, j + 1
+                const uint2 qn = __ldg(reinterpret_cast<const uint2*>(a.lc + lbn));
 #pragma unroll 1
                 for (int i = 0; i < 4; ++i, ++u) {
                     const int s = team + 4 * i;
-                    const LimbConst lc = a.lc[lbc];
+                    LimbConst lc;                        // the row stages use q, 2q only
+                    lc.q = qc.x; lc.q2 = qc.y;
                     const uint2* __restrict__ tw = a.tw + ((size_t)lbc << LOGN);
                     uint32_t* S = B0;
                     // ---- R1(j, s): stage 1 (layers 4..7, thread (b, c), elements a) from TMEM
@@ -426,7 +433,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmr16(NttArgs a, uint32_t rows, con
                     // ---- C(j+1, s): overwrites exactly the TMEM cells R1 read
                     const uint32_t m = 4 * (j + 1) + i;
                     if (more) {
-                        colpass(m, lbn);
+                        colpass(m, lbn, qn);
                         if (i == 3) row_arrive();        // this warp's part of row j + 1 is in TMEM
                     }
                     team_bar(team);                      // stage 1 (and column pass m) done team-wide

@@ -160,9 +160,11 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                 tma2_load_hint(SB(m), &tm_in, (team + 4 * (int)(m & 3)) * TT, (int)(prow * R), tbar + m % NB,
                                l2_evict_first_policy());
             };
-            auto colpass = [&](uint32_t m, uint32_t limb) {   // layers 0..A-1 of pass m into slot (m / 4) & 1
+            // qv = (q, 2q) of the limb, loaded once per row by the caller (as in ntt_tmr.cuh)
+            auto colpass = [&](uint32_t m, uint32_t limb, uint2 qv) {   // layers 0..A-1 of pass m into slot (m / 4) & 1
                 const int p = team + 4 * (int)(m & 3);
-                const LimbConst lc = a.lc[limb];
+                LimbConst lc;
+                lc.q = qv.x; lc.q2 = qv.y;
                 const uint2* __restrict__ tw = a.tw + ((size_t)limb << LOGN);
                 mb_wait(tbar + m % NB, (m / NB) & 1);
                 const uint32_t* B = SB(m);
@@ -180,7 +182,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
 #pragma unroll 1
             for (uint32_t m0 = 0; m0 < 4; m0 += PPS) {
 #pragma unroll 1
-                for (uint32_t q = 0; q < (uint32_t)PPS; ++q) colpass(m0 + q, lbc);
+                for (uint32_t q = 0; q < (uint32_t)PPS; ++q) colpass(m0 + q, lbc, __ldg(reinterpret_cast<const uint2*>(a.lc + lbc)));
                 tmr::team_bar(team);
                 if (t == 0)
                     for (uint32_t q = 0; q < (uint32_t)PPS; ++q) {
@@ -194,10 +196,13 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                 const bool more = j + 1 < nrow;
                 const uint32_t r2 = j + 2 < nrow ? row_of(j + 2) : 0;
                 const uint32_t r3 = j + 3 < nrow ? row_of(j + 3) : 0;
+                const uint2 qc = __ldg(reinterpret_cast<const uint2*>(a.lc + lbc));   // (q, 2q) of rows j, j + 1
+                const uint2 qn = __ldg(reinterpret_cast<const uint2*>(a.lc + lbn));
 #pragma unroll 1
                 for (int i = 0; i < NST; ++i, ++u) {
                     const int s = team + 4 * i;
-                    const LimbConst lc = a.lc[lbc];
+                    LimbConst lc;                        // the row stages use q, 2q only
+                    lc.q = qc.x; lc.q2 = qc.y;
                     const uint2* __restrict__ tw = a.tw + ((size_t)lbc << LOGN);
                     uint32_t* S = B0;
                     // ---- R1(j, s): stage 1 (layers A..A+3, thread (b, c), elements a) from slot j & 1
@@ -219,7 +224,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tms(NttArgs a, uint32_t rows, const
                         // slot (j + 1) & 1 last held row j - 1: every warp has read it
                         if (i == 0 && j > 0) wait_tmem(slotbar, j - 1);
 #pragma unroll 1
-                        for (uint32_t q = 0; q < (uint32_t)PPS; ++q) colpass(m0 + q, lbn);
+                        for (uint32_t q = 0; q < (uint32_t)PPS; ++q) colpass(m0 + q, lbn, qn);
                         if (i == NST - 1) warp_arrive_tmem(rowbar);   // this warp's passes of row j + 1
                     }
                     tmr::team_bar(team);                 // stage 1 (and the step's passes) done team-wide

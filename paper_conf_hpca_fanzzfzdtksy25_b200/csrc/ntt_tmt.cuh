@@ -88,8 +88,10 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
                 tma3_load_hint(SB(m), &tm_in, 0, 8 * (int)(m & 1), (int)(prow * R), tbar + (m & 1),
                                l2_evict_first_policy());
             };
-            auto colstep = [&](uint32_t m, uint32_t limb) {   // layer 0 of 8 passes into slot (m / 2) & 1
-                const LimbConst lc = a.lc[limb];
+            // qv = (q, 2q) of the limb, loaded once per row by the caller (as in ntt_tmr.cuh)
+            auto colstep = [&](uint32_t m, uint32_t limb, uint2 qv) {   // layer 0 of 8 passes into slot (m / 2) & 1
+                LimbConst lc;
+                lc.q = qv.x; lc.q2 = qv.y;
                 const uint2 w0 = __ldg(a.tw + ((size_t)limb << LOGN) + 1);
                 mb_wait(tbar + (m & 1), (m >> 1) & 1);
                 const uint32_t* B = SB(m);
@@ -111,7 +113,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
             cp_async_commit();
 #pragma unroll 1
             for (uint32_t m = 0; m < 2; ++m) {       // prologue: row 0's column passes
-                colstep(m, lbc);
+                colstep(m, lbc, __ldg(reinterpret_cast<const uint2*>(a.lc + lbc)));
                 team_sync_tmem();
                 if (t == 0 && m + 2 < mtot) issue_step(m + 2, rwn);
             }
@@ -119,9 +121,12 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
             for (uint32_t j = 0; j < nrow; ++j) {
                 const bool more = j + 1 < nrow;
                 const uint32_t r2 = j + 2 < nrow ? row_of(j + 2) : 0;
+                const uint2 qc = __ldg(reinterpret_cast<const uint2*>(a.lc + lbc));   // (q, 2q) of rows j, j + 1
+                const uint2 qn = __ldg(reinterpret_cast<const uint2*>(a.lc + lbn));
 #pragma unroll 1
                 for (int s = 0; s < R; ++s, ++u) {
-                    const LimbConst lc = a.lc[lbc];
+                    LimbConst lc;                        // the row stages use q, 2q only
+                    lc.q = qc.x; lc.q2 = qc.y;
                     const uint2* __restrict__ tw = a.tw + ((size_t)lbc << LOGN);
                     uint32_t* S = B0;
                     // ---- R1(j, s): stage 1 (layers 1..4, thread (b, c), elements a) from slot j & 1
@@ -138,7 +143,7 @@ __global__ void __launch_bounds__(NT, 1) ntt_tmt13(NttArgs a, uint32_t rows, con
                     }
                     // ---- C(j+1, passes 8s .. 8s+7)
                     const uint32_t m = 2 * (j + 1) + s;
-                    if (more) colstep(m, lbn);
+                    if (more) colstep(m, lbn, qn);
                     team_sync_tmem();                    // stage 1, the step's passes done team-wide
                     if (t == 0 && more && m + 2 < mtot) issue_step(m + 2, r2);
                     {   // the team's next sub-row's twiddles
